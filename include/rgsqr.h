@@ -1,0 +1,163 @@
+/*
+ * rgsqr.h -- C ABI of the B200-native out-of-core recursive classical Gram-Schmidt QR.
+ *
+ * The operation (Zhang & Wu, ICPP'21, /root/reference/PAPER.md):
+ *   factor a tall matrix A (m x n, m >= n, "m is the number of rows and n is the
+ *   number of columns") into Q (orthonormal columns) and R (upper
+ *   triangular) with A = Q R, by classical Gram-Schmidt
+ *   (Eq. 1; CGS evaluation order PAPER.md:109) organised as the
+ *   column-halving recursion of Eq. 2:
+ *       [A1|A2] = [Q1|Q2] [[R11, R12], [0, R22]]
+ *       A1 = Q1 R11;  R12 = Q1^T A2;  A2 <- A2 - Q1 R12;  A2 = Q2 R22.
+ *   When A does not fit the device-memory budget the two products stream row
+ *   tiles host<->device with the copies overlapped by the math.
+ *
+ * Conventions (all functions):
+ *   - Return an int status: 0 = OK, > 0 = warning (outputs valid), < 0 = error
+ *     (outputs unspecified; message via rgsqr_last_error).
+ *   - Matrices are COLUMN-MAJOR. A, Q: element (i,j) at base[i + j*lda].
+ *     R: n x n, element (i,j) at R[i + j*n] (ldr = n), binary32, strict lower
+ *     triangle written as 0.
+ *   - Element type of A and Q is set by `precision`:
+ *       RGSQR_FP16   -> IEEE binary16 storage, fp16 tensor-core operands, fp32 accumulate
+ *       RGSQR_BF16   -> bfloat16 storage,       bf16 operands,               fp32 accumulate
+ *       RGSQR_TF32   -> binary32 storage,       tf32 operands,               fp32 accumulate
+ *       RGSQR_TF32X3 -> binary32 storage,       3-pass split tf32 (hi*hi + hi*lo + lo*hi)
+ *   - Stored-value rounding (Q, updated A2', R12 used as an MMA operand) is
+ *     round-to-nearest-even (reading R5).
+ *   - Ownership: the caller owns every buffer it passes; the library never frees
+ *     or reallocates them.  The library owns all device memory it allocates: a
+ *     single arena of at most `device_mem_budget` bytes (0 = all free memory
+ *     minus a 512 MiB reserve), so the budget is enforced by construction.
+ *   - Blocking: rgsqr_factor* return after Q and R are complete (host-synchronous).
+ *     A handle is not thread-safe; use one handle per thread / per GPU.
+ *   - Preconditions: 1 <= n <= m, lda >= m, lda*sizeof(elem) % 16 == 0, pointers
+ *     16-byte aligned.  Violations return RGSQR_ERR_INVALID_ARG.
+ *   - Rank deficiency (the paper assumes linearly independent columns,
+ *     PAPER.md:103): if some r_jj <= m * u_fp32 * ||a_j|| (or is not finite),
+ *     q_j = 0 and r_jj = 0 are written, the first such j is reported in
+ *     rgsqr_stats.first_breakdown_col, and RGSQR_WARN_RANK_DEFICIENT is returned.
+ */
+#ifndef RGSQR_H
+#define RGSQR_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct rgsqr_ctx* rgsqr_handle;
+
+enum rgsqr_precision { RGSQR_FP16 = 0, RGSQR_BF16 = 1, RGSQR_TF32 = 2, RGSQR_TF32X3 = 3 };
+
+enum rgsqr_status {
+  RGSQR_OK = 0,
+  RGSQR_WARN_RANK_DEFICIENT = 1,
+  RGSQR_ERR_INVALID_ARG = -1,
+  RGSQR_ERR_BUDGET_TOO_SMALL = -2,
+  RGSQR_ERR_CUDA = -3,
+  RGSQR_ERR_NCCL = -4,
+  RGSQR_ERR_UNSUPPORTED = -5,
+  RGSQR_ERR_HOST_MEM = -6
+};
+
+/* Option keys for rgsqr_set_option / rgsqr_get_option. */
+enum rgsqr_option {
+  RGSQR_OPT_LEAF_WIDTH = 1,     /* columns factored by the in-kernel CGS leaf (8..64, default 64) */
+  RGSQR_OPT_TILE_ROWS_MIN = 2,  /* OOC row-tile ramp start (paper: 2048; default 4096) */
+  RGSQR_OPT_TILE_ROWS_MAX = 3,  /* OOC row-tile cap (paper: 8192/16384; default 16384) */
+  RGSQR_OPT_RING_DEPTH = 4,     /* K device slots per OOC stream ring (>= 2, default 3) */
+  RGSQR_OPT_ALGO = 5,           /* 0 = recursive (Eq. 2, default), 1 = blocked */
+  RGSQR_OPT_BLOCK_COLS = 6,     /* panel width b of the blocked algorithm (default 8192) */
+  RGSQR_OPT_SERIALIZE = 7,      /* 1 = one stream, no overlap (the paper's "Synchronous" rows) */
+  RGSQR_OPT_REUSE = 8,          /* 1 = QR-level data reuse, default 1 */
+  RGSQR_OPT_LEAF_CTAS = 9,      /* CTAs of the leaf kernel (0 = automatic) */
+  RGSQR_OPT_SPLITK = 10         /* force split-K factor of the TN product (0 = automatic) */
+};
+
+/* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */
+typedef struct rgsqr_stats {
+  int64_t h2d_bytes;            /* all host->device bytes */
+  int64_t d2h_bytes;            /* all device->host bytes */
+  int64_t h2d_matrix_bytes;     /* A / A2' / Q words moved host->device */
+  int64_t d2h_matrix_bytes;     /* Q / A2' words moved device->host */
+  int64_t d2h_r_bytes;          /* R blocks moved device->host */
+  int64_t d2d_bytes;            /* device-to-device staging copies */
+  double  wall_ms;              /* host wall time of the factorization call */
+  double  h2d_busy_ms;          /* sum of H2D copy durations (CUDA events) */
+  double  d2h_busy_ms;          /* sum of D2H copy durations */
+  double  compute_busy_ms;      /* sum of compute-stream segment durations */
+  double  overlap_ratio;        /* (sum busy - wall) / (sum busy - max busy), R18 */
+  double  pin_ms;               /* cudaHostRegister time (excluded from wall_ms) */
+  int64_t arena_bytes;          /* size of the device arena */
+  int64_t arena_high_water;     /* peak arena bytes in use */
+  int64_t n_leaf_launches;
+  int64_t n_tn_launches;
+  int64_t n_nn_launches;
+  int64_t n_other_launches;
+  int64_t n_ooc_nodes;
+  int64_t n_incore_nodes;
+  int64_t first_breakdown_col;  /* -1 if none */
+  int64_t flops;                /* 2 m n^2 (BASELINE.json metric convention) */
+} rgsqr_stats;
+
+/* ---- lifetime -------------------------------------------------------------------- */
+int rgsqr_create(rgsqr_handle* h, int device);
+/* Multi-GPU (row-sharded, one process per GPU): rank 0 calls rgsqr_get_unique_id and
+ * broadcasts the 128 bytes; every rank then calls rgsqr_create_dist collectively. */
+int rgsqr_get_unique_id(unsigned char id[128]);
+int rgsqr_create_dist(rgsqr_handle* h, int device, int rank, int nranks, const unsigned char id[128]);
+int rgsqr_destroy(rgsqr_handle h);
+
+/* ---- the factorization ------------------------------------------------------------- */
+/* Host-resident out-of-core recursive CGS QR.  A_host: m x n (lda), host memory
+ * (pinned or pageable; pageable buffers are page-locked for the call, cost in
+ * stats.pin_ms).  Q_out: host, same element type and lda; may alias A_host (in
+ * place).  R_out: host n x n binary32 (rank 0 only when nranks > 1; others may pass
+ * NULL).  device_mem_budget: bytes of device memory the library may use (0 = all).
+ * With nranks > 1, m is the number of LOCAL rows of this rank's contiguous row block. */
+int rgsqr_factor(rgsqr_handle h, const void* A_host, int64_t lda, int64_t m, int64_t n,
+                 void* Q_out, float* R_out, int precision, size_t device_mem_budget);
+
+/* Same factorization with A, Q and R already resident in device memory (HBM).
+ * A_dev / Q_dev: device pointers (Q_dev may alias A_dev), R_dev: device n x n
+ * binary32.  device_mem_budget bounds the library's workspace only.  Runs on the
+ * handle's stream (rgsqr_set_stream). */
+int rgsqr_factor_device(rgsqr_handle h, const void* A_dev, int64_t lda, int64_t m, int64_t n,
+                        void* Q_dev, float* R_dev, int precision, size_t device_mem_budget);
+
+/* ---- hot-path operations (device pointers; used by the kernel parity tests) ------------ */
+/* Leaf CGS panel (Eq. 1) in place: P (m x w, ldp) -> Q; R11 (w x w,
+ * device, ldr) receives r_ij, 1 <= w <= 64.  Returns the first breakdown column via
+ * *breakdown (host int, -1 if none). */
+int rgsqr_op_leaf(rgsqr_handle h, void* P, int64_t ldp, int64_t m, int64_t w,
+                  float* R11, int64_t ldr, int precision, int* breakdown);
+/* Inner product R12 (+)= Q1^T A2: Q1 m x w1 (ldq), A2 m x w2 (lda),
+ * R12 binary32 w1 x w2 (ldr).  accumulate = 0: R12 = Q1^T A2; 1: R12 += Q1^T A2.
+ * R12op (optional, may be NULL): R12 rounded to the operand type, ld = w1. */
+int rgsqr_op_inner(rgsqr_handle h, const void* Q1, int64_t ldq, const void* A2, int64_t lda,
+                   int64_t m, int64_t w1, int64_t w2, float* R12, int64_t ldr,
+                   void* R12op, int accumulate, int precision);
+/* Outer product A2 <- A2 - Q1 R12op: Q1 m x w1 (ldq), R12op
+ * w1 x w2 operand-typed (ld = ldr), A2 m x w2 (lda) updated in place. */
+int rgsqr_op_outer(rgsqr_handle h, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr,
+                   void* A2, int64_t lda, int64_t m, int64_t w1, int64_t w2, int precision);
+
+/* ---- support ------------------------------------------------------------------------ */
+int rgsqr_set_stream(rgsqr_handle h, void* cuda_stream);      /* NULL = library's own stream */
+int rgsqr_get_stream(rgsqr_handle h, void** cuda_stream);
+int rgsqr_host_alloc(rgsqr_handle h, size_t bytes, void** p);  /* pinned, first-touch */
+int rgsqr_host_free(rgsqr_handle h, void* p);
+int rgsqr_set_option(rgsqr_handle h, int key, int64_t value);
+int rgsqr_get_option(rgsqr_handle h, int key, int64_t* value);
+int rgsqr_get_stats(rgsqr_handle h, rgsqr_stats* out);
+int rgsqr_version(void);                                        /* 100 * major + minor */
+const char* rgsqr_status_string(int status);
+const char* rgsqr_last_error(rgsqr_handle h);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RGSQR_H */

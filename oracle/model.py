@@ -118,3 +118,43 @@ def inner_overlap_condition(rg: float, rm: float, word_bytes: int = 4) -> float:
     """the streamed inner product hides its copies when
     (4mk+4nk)/Rm < 2mnk/Rg, i.e. (square case m = n) m > 4 Rg / Rm (fp32 words)."""
     return word_bytes * rg / rm
+
+
+def recursive_noreuse_split_words(m: int, n: int, b: int) -> dict:
+    """The no-reuse recursive traffic split into matrix words (A / Q / A2') and R words,
+    for an executor that keeps R12 resident between the two products (so the outer
+    product does not re-read R12; the paper's model of PAPER.md:147 does)."""
+    out = {"h2d_matrix": 0, "d2h_matrix": 0, "d2h_r": 0}
+
+    def rec(w):
+        if w <= b:
+            out["h2d_matrix"] += m * w
+            out["d2h_matrix"] += m * w
+            out["d2h_r"] += w * w
+            return
+        w1 = w // 2
+        w2 = w - w1
+        rec(w1)
+        out["h2d_matrix"] += 2 * m * (w1 + w2)      # inner + outer read Q1 and A2
+        out["d2h_matrix"] += m * w2                 # outer writes A2'
+        out["d2h_r"] += w1 * w2                     # R12 out once
+        rec(w2)
+
+    rec(n)
+    return out
+
+
+def blocked_noreuse_split_words(m: int, n: int, b: int) -> dict:
+    """PAPER.md:139 per-iteration terms without the R12 re-read, and with the last
+    panel (no trailing matrix) moving only its panel in and Q out."""
+    k = n // b
+    out = {"h2d_matrix": 0, "d2h_matrix": 0, "d2h_r": 0}
+    for i in range(1, k + 1):
+        rest = n - i * b
+        if rest == 0:
+            out["h2d_matrix"] += m * b
+        else:
+            out["h2d_matrix"] += m * b + m * b + m * rest + m * b + m * rest
+        out["d2h_matrix"] += m * b + m * rest
+        out["d2h_r"] += b * b + b * rest
+    return out

@@ -1,0 +1,357 @@
+// api.cu -- the extern "C" boundary declared in include/rgsqr.h.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <chrono>
+#include <climits>
+#include <cstring>
+#include <new>
+
+#include "engine.h"
+
+using namespace rgsqr;
+
+namespace rgsqr {
+
+int ensure_arena(Ctx* c, size_t want) {
+  if (c->arena.base && c->arena.size >= want && c->arena.size <= want + ((size_t)64 << 20)) {
+    c->arena.top = 0;
+    return RGSQR_OK;
+  }
+  if (c->arena.base) {
+    cudaFree(c->arena.base);
+    c->arena = Arena{};
+  }
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, want);
+  if (e != cudaSuccess)
+    return fail(c, RGSQR_ERR_CUDA, "arena cudaMalloc(" + std::to_string(want) + "): " + cudaGetErrorString(e));
+  c->arena.base = static_cast<char*>(p);
+  c->arena.size = want;
+  c->arena.top = 0;
+  c->arena.high = 0;
+  return RGSQR_OK;
+}
+
+size_t resolve_budget(Ctx* c, size_t budget) {
+  if (budget != 0) return budget;
+  size_t fr = 0, tot = 0;
+  cudaMemGetInfo(&fr, &tot);
+  size_t mine = c->arena.base ? c->arena.size : 0;
+  size_t avail = fr + mine;
+  const size_t reserve = (size_t)512 << 20;
+  return avail > reserve ? avail - reserve : avail / 2;
+}
+
+void reset_stats(Ctx* c) {
+  std::memset(&c->stats, 0, sizeof(c->stats));
+  c->stats.first_breakdown_col = -1;
+}
+
+int validate(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, const void* Q, int prec) {
+  if (!A || !Q) return fail(c, RGSQR_ERR_INVALID_ARG, "null A or Q");
+  if (n < 1 || m < n) return fail(c, RGSQR_ERR_INVALID_ARG, "need 1 <= n <= m");
+  if (lda < m) return fail(c, RGSQR_ERR_INVALID_ARG, "need lda >= m");
+  if (prec < RGSQR_FP16 || prec > RGSQR_TF32X3) return fail(c, RGSQR_ERR_INVALID_ARG, "bad precision");
+  if (prec == RGSQR_TF32X3) return fail(c, RGSQR_ERR_UNSUPPORTED, "TF32X3 not implemented yet");
+  const int s = elem_bytes(prec);
+  if ((lda * s) % 16 != 0) return fail(c, RGSQR_ERR_INVALID_ARG, "lda*sizeof(elem) must be a multiple of 16");
+  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(Q)) & 15)
+    return fail(c, RGSQR_ERR_INVALID_ARG, "A and Q must be 16-byte aligned");
+  return RGSQR_OK;
+}
+
+// A, Q, R in HBM; in-core recursion on Q (after copying A into Q when they differ).
+int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* Q, float* R, int prec,
+                  size_t budget) {
+  int rc = validate(c, A, lda, m, n, Q, prec);
+  if (rc < 0) return rc;
+  if (!R) return fail(c, RGSQR_ERR_INVALID_ARG, "null R");
+  reset_stats(c);
+  auto t0 = std::chrono::steady_clock::now();
+  const size_t ws = incore_workspace_bytes(c, prec, m, n);
+  const size_t cap = resolve_budget(c, budget);
+  if (ws > cap) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "workspace " + std::to_string(ws) + " > budget");
+  rc = ensure_arena(c, ws);
+  if (rc < 0) return rc;
+  cudaStream_t st = c->compute();
+  const int s = elem_bytes(prec);
+  if (Q != A)
+    RGSQR_CUDA(c, cudaMemcpy2DAsync(Q, lda * s, A, lda * s, m * s, n, cudaMemcpyDeviceToDevice, st));
+  RGSQR_CUDA(c, cudaMemsetAsync(R, 0, (size_t)n * n * sizeof(float), st));
+  RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), st));
+  rc = incore_factor(c, prec, Q, lda, m, n, R, n, 0, st);
+  if (rc < 0) return rc;
+  int brk = INT_MAX;
+  RGSQR_CUDA(c, cudaMemcpyAsync(&brk, c->d_breakdown, sizeof(int), cudaMemcpyDeviceToHost, st));
+  RGSQR_CUDA(c, cudaStreamSynchronize(st));
+  auto t1 = std::chrono::steady_clock::now();
+  c->stats.wall_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+  c->stats.arena_bytes = (int64_t)c->arena.size;
+  c->stats.arena_high_water = (int64_t)c->arena.high;
+  c->stats.flops = (int64_t)(2.0 * m * (double)n * n);
+  c->stats.first_breakdown_col = brk == 0x7f7f7f7f || brk == INT_MAX ? -1 : brk;
+  return c->stats.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;
+}
+
+}  // namespace rgsqr
+
+// ------------------------------------------------------------------------------------
+// NCCL (loaded at run time from the pip wheel torch uses; only for nranks > 1)
+// ------------------------------------------------------------------------------------
+namespace {
+struct NcclApi {
+  void* lib = nullptr;
+  int (*getUniqueId)(void*) = nullptr;
+  int (*commInitRank)(void**, int, const void*, int) = nullptr;
+  int (*commDestroy)(void*) = nullptr;
+  int (*allReduce)(const void*, void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  bool load() {
+    if (lib) return true;
+    const char* names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char* nm : names) {
+      lib = dlopen(nm, RTLD_NOW | RTLD_GLOBAL);
+      if (lib) break;
+    }
+    if (!lib) return false;
+    getUniqueId = reinterpret_cast<int (*)(void*)>(dlsym(lib, "ncclGetUniqueId"));
+    commInitRank = reinterpret_cast<int (*)(void**, int, const void*, int)>(dlsym(lib, "ncclCommInitRank"));
+    commDestroy = reinterpret_cast<int (*)(void*)>(dlsym(lib, "ncclCommDestroy"));
+    allReduce = reinterpret_cast<int (*)(const void*, void*, size_t, int, int, void*, cudaStream_t)>(
+        dlsym(lib, "ncclAllReduce"));
+    return getUniqueId && commInitRank && commDestroy && allReduce;
+  }
+};
+NcclApi g_nccl;
+
+int create_impl(rgsqr_handle* h, int device) {
+  if (!h) return RGSQR_ERR_INVALID_ARG;
+  *h = nullptr;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return RGSQR_ERR_CUDA;
+  if (device < 0 || device >= ndev) return RGSQR_ERR_INVALID_ARG;
+  if (cudaSetDevice(device) != cudaSuccess) return RGSQR_ERR_CUDA;
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return RGSQR_ERR_CUDA;
+  if (prop.major != 10) return RGSQR_ERR_UNSUPPORTED;  // sm_100a only
+  Ctx* c = new (std::nothrow) Ctx();
+  if (!c) return RGSQR_ERR_HOST_MEM;
+  c->device = device;
+  c->num_sms = prop.multiProcessorCount;
+  if (cudaStreamCreateWithFlags(&c->st_own, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->st_h2d, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
+      cudaMalloc(&c->d_counter, 256) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess) {
+    delete c;
+    return RGSQR_ERR_CUDA;
+  }
+  reset_stats(c);
+  *h = reinterpret_cast<rgsqr_handle>(c);
+  return RGSQR_OK;
+}
+
+Ctx* C(rgsqr_handle h) { return reinterpret_cast<Ctx*>(h); }
+}  // namespace
+
+extern "C" {
+
+int rgsqr_version(void) { return 100; }
+
+const char* rgsqr_status_string(int s) {
+  switch (s) {
+    case RGSQR_OK: return "RGSQR_OK";
+    case RGSQR_WARN_RANK_DEFICIENT: return "RGSQR_WARN_RANK_DEFICIENT";
+    case RGSQR_ERR_INVALID_ARG: return "RGSQR_ERR_INVALID_ARG";
+    case RGSQR_ERR_BUDGET_TOO_SMALL: return "RGSQR_ERR_BUDGET_TOO_SMALL";
+    case RGSQR_ERR_CUDA: return "RGSQR_ERR_CUDA";
+    case RGSQR_ERR_NCCL: return "RGSQR_ERR_NCCL";
+    case RGSQR_ERR_UNSUPPORTED: return "RGSQR_ERR_UNSUPPORTED";
+    case RGSQR_ERR_HOST_MEM: return "RGSQR_ERR_HOST_MEM";
+  }
+  return "RGSQR_UNKNOWN_STATUS";
+}
+
+int rgsqr_create(rgsqr_handle* h, int device) { return create_impl(h, device); }
+
+int rgsqr_get_unique_id(unsigned char id[128]) {
+  if (!id) return RGSQR_ERR_INVALID_ARG;
+  if (!g_nccl.load()) return RGSQR_ERR_NCCL;
+  return g_nccl.getUniqueId(id) == 0 ? RGSQR_OK : RGSQR_ERR_NCCL;
+}
+
+int rgsqr_create_dist(rgsqr_handle* h, int device, int rank, int nranks, const unsigned char id[128]) {
+  if (nranks < 1 || rank < 0 || rank >= nranks || !id) return RGSQR_ERR_INVALID_ARG;
+  int rc = create_impl(h, device);
+  if (rc < 0) return rc;
+  Ctx* c = C(*h);
+  c->rank = rank;
+  c->nranks = nranks;
+  if (nranks > 1) {
+    if (!g_nccl.load()) return fail(c, RGSQR_ERR_NCCL, "libnccl.so.2 not loadable");
+    if (g_nccl.commInitRank(&c->nccl_comm, nranks, id, rank) != 0)
+      return fail(c, RGSQR_ERR_NCCL, "ncclCommInitRank failed");
+  }
+  return RGSQR_OK;
+}
+
+int rgsqr_destroy(rgsqr_handle h) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  cudaDeviceSynchronize();
+  if (c->nccl_comm && g_nccl.commDestroy) g_nccl.commDestroy(c->nccl_comm);
+  if (c->arena.base) cudaFree(c->arena.base);
+  cudaFree(c->d_partials);
+  cudaFree(c->d_counter);
+  cudaFree(c->d_breakdown);
+  for (auto e : c->event_pool) cudaEventDestroy(e);
+  cudaStreamDestroy(c->st_own);
+  cudaStreamDestroy(c->st_h2d);
+  cudaStreamDestroy(c->st_d2h);
+  delete c;
+  return RGSQR_OK;
+}
+
+int rgsqr_factor(rgsqr_handle h, const void* A_host, int64_t lda, int64_t m, int64_t n, void* Q_out, float* R_out,
+                 int precision, size_t device_mem_budget) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  return factor_host(c, A_host, lda, m, n, Q_out, R_out, precision, device_mem_budget);
+}
+
+int rgsqr_factor_device(rgsqr_handle h, const void* A_dev, int64_t lda, int64_t m, int64_t n, void* Q_dev,
+                        float* R_dev, int precision, size_t device_mem_budget) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  return factor_device(c, A_dev, lda, m, n, Q_dev, R_dev, precision, device_mem_budget);
+}
+
+int rgsqr_op_leaf(rgsqr_handle h, void* P, int64_t ldp, int64_t m, int64_t w, float* R11, int64_t ldr,
+                  int precision, int* breakdown) {
+  Ctx* c = C(h);
+  if (!c || !P || !R11 || m < 1 || w < 1 || ldp < m || ldr < w) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  cudaStream_t st = c->compute();
+  RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), st));
+  int rc = op_leaf(c, precision, P, ldp, m, w, R11, ldr, 0, st);
+  if (rc < 0) return rc;
+  int brk = INT_MAX;
+  RGSQR_CUDA(c, cudaMemcpyAsync(&brk, c->d_breakdown, sizeof(int), cudaMemcpyDeviceToHost, st));
+  RGSQR_CUDA(c, cudaStreamSynchronize(st));
+  if (breakdown) *breakdown = (brk == 0x7f7f7f7f) ? -1 : brk;
+  return brk == 0x7f7f7f7f ? RGSQR_OK : RGSQR_WARN_RANK_DEFICIENT;
+}
+
+int rgsqr_op_inner(rgsqr_handle h, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m, int64_t w1,
+                   int64_t w2, float* R12, int64_t ldr, void* R12op, int accumulate, int precision) {
+  Ctx* c = C(h);
+  if (!c || !Q1 || !A2 || !R12 || m < 1 || w1 < 1 || w2 < 1 || ldr < w1) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  int rc = ensure_arena(c, (size_t)72 << 20);
+  if (rc < 0) return rc;
+  rc = op_inner(c, precision, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, w1, accumulate, c->compute());
+  if (rc < 0) return rc;
+  RGSQR_CUDA(c, cudaStreamSynchronize(c->compute()));
+  return RGSQR_OK;
+}
+
+int rgsqr_op_outer(rgsqr_handle h, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2,
+                   int64_t lda, int64_t m, int64_t w1, int64_t w2, int precision) {
+  Ctx* c = C(h);
+  if (!c || !Q1 || !A2 || !R12op || m < 1 || w1 < 1 || w2 < 1) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  int rc = op_outer(c, precision, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, c->compute());
+  if (rc < 0) return rc;
+  RGSQR_CUDA(c, cudaStreamSynchronize(c->compute()));
+  return RGSQR_OK;
+}
+
+int rgsqr_set_stream(rgsqr_handle h, void* s) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  c->st_user = static_cast<cudaStream_t>(s);
+  return RGSQR_OK;
+}
+
+int rgsqr_get_stream(rgsqr_handle h, void** s) {
+  Ctx* c = C(h);
+  if (!c || !s) return RGSQR_ERR_INVALID_ARG;
+  *s = c->compute();
+  return RGSQR_OK;
+}
+
+int rgsqr_host_alloc(rgsqr_handle h, size_t bytes, void** p) {
+  Ctx* c = C(h);
+  if (!c || !p) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  if (cudaHostAlloc(p, bytes, cudaHostAllocPortable) != cudaSuccess) return fail(c, RGSQR_ERR_HOST_MEM, "cudaHostAlloc");
+  return RGSQR_OK;
+}
+
+int rgsqr_host_free(rgsqr_handle h, void* p) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  return cudaFreeHost(p) == cudaSuccess ? RGSQR_OK : RGSQR_ERR_CUDA;
+}
+
+static int64_t* opt_slot(Ctx* c, int key) {
+  Options& o = c->opt;
+  switch (key) {
+    case RGSQR_OPT_LEAF_WIDTH: return &o.leaf_width;
+    case RGSQR_OPT_TILE_ROWS_MIN: return &o.tile_rows_min;
+    case RGSQR_OPT_TILE_ROWS_MAX: return &o.tile_rows_max;
+    case RGSQR_OPT_RING_DEPTH: return &o.ring_depth;
+    case RGSQR_OPT_ALGO: return &o.algo;
+    case RGSQR_OPT_BLOCK_COLS: return &o.block_cols;
+    case RGSQR_OPT_SERIALIZE: return &o.serialize;
+    case RGSQR_OPT_REUSE: return &o.reuse;
+    case RGSQR_OPT_LEAF_CTAS: return &o.leaf_ctas;
+    case RGSQR_OPT_SPLITK: return &o.splitk;
+  }
+  return nullptr;
+}
+
+int rgsqr_set_option(rgsqr_handle h, int key, int64_t value) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  int64_t* s = opt_slot(c, key);
+  if (!s) return fail(c, RGSQR_ERR_INVALID_ARG, "unknown option");
+  switch (key) {
+    case RGSQR_OPT_LEAF_WIDTH: if (value < 1 || value > LEAF_MAX_W) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_TILE_ROWS_MIN:
+    case RGSQR_OPT_TILE_ROWS_MAX: if (value < 128 || value % 128) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_RING_DEPTH: if (value < 2 || value > 16) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_ALGO: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_BLOCK_COLS: if (value < 8) return RGSQR_ERR_INVALID_ARG; break;
+    default: if (value < 0) return RGSQR_ERR_INVALID_ARG;
+  }
+  *s = value;
+  return RGSQR_OK;
+}
+
+int rgsqr_get_option(rgsqr_handle h, int key, int64_t* value) {
+  Ctx* c = C(h);
+  if (!c || !value) return RGSQR_ERR_INVALID_ARG;
+  int64_t* s = opt_slot(c, key);
+  if (!s) return RGSQR_ERR_INVALID_ARG;
+  *value = *s;
+  return RGSQR_OK;
+}
+
+int rgsqr_get_stats(rgsqr_handle h, rgsqr_stats* out) {
+  Ctx* c = C(h);
+  if (!c || !out) return RGSQR_ERR_INVALID_ARG;
+  *out = c->stats;
+  return RGSQR_OK;
+}
+
+const char* rgsqr_last_error(rgsqr_handle h) {
+  Ctx* c = C(h);
+  if (!c) return "invalid handle";
+  return c->last_error.c_str();
+}
+
+}  // extern "C"

@@ -1,0 +1,121 @@
+// engine.h -- host-side runtime: context, device arena, tensor maps, the hot-path ops,
+// the in-core recursion and the out-of-core executor.
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <functional>
+#include <string>
+#include <vector>
+
+#include "../../include/rgsqr.h"
+#include "kernels.h"
+
+namespace rgsqr {
+
+struct Options {
+  int64_t leaf_width = 64;
+  int64_t tile_rows_min = 4096;
+  int64_t tile_rows_max = 16384;
+  int64_t ring_depth = 3;
+  int64_t algo = 0;          // 0 recursive, 1 blocked
+  int64_t block_cols = 8192;
+  int64_t serialize = 0;
+  int64_t reuse = 1;
+  int64_t leaf_ctas = 0;
+  int64_t splitk = 0;
+};
+
+// Bump allocator over one cudaMalloc of at most the budget; LIFO release by mark.
+struct Arena {
+  char* base = nullptr;
+  size_t size = 0;
+  size_t top = 0;
+  size_t high = 0;
+  void* alloc(size_t bytes) {
+    size_t off = (top + 255) & ~size_t(255);
+    if (off + bytes > size) return nullptr;
+    top = off + bytes;
+    if (top > high) high = top;
+    return base + off;
+  }
+  size_t mark() const { return top; }
+  void release(size_t m) { top = m; }
+  size_t free_bytes() const { return size > top ? size - ((top + 255) & ~size_t(255)) : 0; }
+};
+
+struct TimedSeg {
+  int kind;                  // 0 h2d, 1 d2h, 2 compute
+  cudaEvent_t a, b;
+};
+
+struct Ctx {
+  int device = 0;
+  int rank = 0, nranks = 1;
+  int num_sms = 148;
+  cudaStream_t st_user = nullptr;   // set by rgsqr_set_stream
+  cudaStream_t st_own = nullptr;
+  cudaStream_t st_h2d = nullptr, st_d2h = nullptr;
+  Options opt;
+  rgsqr_stats stats{};
+  std::string last_error;
+  Arena arena;
+  size_t arena_alloc_size = 0;
+  // small persistent device buffers (leaf barrier/partials, breakdown flag)
+  float* d_partials = nullptr;
+  unsigned int* d_counter = nullptr;
+  int* d_breakdown = nullptr;
+  void* nccl_comm = nullptr;
+  std::vector<TimedSeg> segs;
+  std::vector<cudaEvent_t> event_pool;
+  size_t event_next = 0;
+  bool timing = false;
+
+  cudaStream_t compute() const { return st_user ? st_user : st_own; }
+  cudaEvent_t ev();
+};
+
+// status helpers
+int fail(Ctx* c, int status, const std::string& msg);
+#define RGSQR_CUDA(c, call)                                                        \
+  do {                                                                             \
+    cudaError_t _e = (call);                                                       \
+    if (_e != cudaSuccess)                                                         \
+      return fail((c), RGSQR_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(_e)); \
+  } while (0)
+
+int elem_bytes(int precision);
+bool encode_tmap_2d(CUtensorMap* map, int precision, const void* base, uint64_t inner, uint64_t outer,
+                    uint64_t outer_stride_bytes, uint32_t box_inner, uint32_t box_outer, std::string* err,
+                    bool atom32 = false);
+
+// ---- ops (device pointers, on stream st) ----
+int op_inner(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
+             int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate,
+             cudaStream_t st);
+int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2,
+             int64_t lda, int64_t m, int64_t w1, int64_t w2, cudaStream_t st);
+int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float* R11, int64_t ldr,
+            int64_t col_offset, cudaStream_t st);
+int leaf_width_for(Ctx* c, int64_t m);
+int64_t split_width(int64_t w, int64_t leaf);
+
+// ---- factorizations ----
+size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n);
+// Optional callbacks of the in-core recursion, used by the out-of-core executor to
+// overlap a node's column upload / Q download with its factorization:
+//   need(c)      -- called before any op that reads columns [0, c) of the node
+//   leaf_done(c) -- called after the leaf ending at column c (Q[:, 0:c) is final)
+struct IncoreHooks {
+  std::function<void(int64_t)> need;
+  std::function<void(int64_t)> leaf_done;
+};
+int incore_factor(Ctx* c, int prec, void* A, int64_t lda, int64_t m, int64_t n, float* R, int64_t ldr,
+                  int64_t col_offset, cudaStream_t st, IncoreHooks* hooks = nullptr);
+int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* Q, float* R, int prec,
+                  size_t budget);
+int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* Q, float* R, int prec,
+                size_t budget);
+
+}  // namespace rgsqr

@@ -1,0 +1,245 @@
+// gemm.cu -- the two tensor-core contractions of one recursion node (Eq. 2):
+//
+//   inner product (TN)  R12 (+)= Q1^T A2      M = w1, N = w2, K = m (rows)
+//   outer product (NN)  A2  <-  A2 - Q1 R12   M = m,  N = w2, K = w1
+//
+// One CTA computes a 128 x BN tile with tcgen05.mma (cta_group::1), operands staged by
+// TMA into a STAGES-deep shared-memory ring (128B swizzle), the fp32 accumulator in TMEM.
+// Warp roles: warp 0 = TMA producer (one elected lane), warp 1 = MMA issuer (one elected
+// lane), warp 2 = TMEM allocator; all four warps run the epilogue (TMEM -> registers ->
+// global), warp w owning TMEM lanes [32w, 32w+32).
+//
+// Column-major storage makes both TN operands K-major (rows are the contraction index);
+// in NN the Q1 operand is MN-major (its rows are the output rows) -- legal for
+// f16/bf16/tf32 UMMA.  The subtraction A2 - Q1 R12 is fused into the epilogue, so A2'
+// is written exactly once, rounded RN-even to the storage type (R5).
+#include "dtype.cuh"
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace rgsqr {
+
+template <typename T, bool kNN, int BN>
+struct GemmCfg {
+  static constexpr int BM = 128;
+  static constexpr int EPB = 128 / (int)sizeof(T);  // elements per 128-byte row
+  static constexpr int BK = EPB;                    // K per pipeline stage
+  static constexpr int UK = 32 / (int)sizeof(T);    // K per tcgen05.mma (16 f16, 8 tf32)
+  static constexpr int A_BYTES = BM * 128;
+  static constexpr int B_BYTES = BN * 128;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (196 * 1024) / STAGE_BYTES > 8 ? 8 : (196 * 1024) / STAGE_BYTES;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
+  static constexpr uint32_t IDESC = ptx::idesc_f32acc(Elem<T>::kUmmaFormat, kNN ? 1u : 0u, 0u, BM, BN);
+};
+
+template <typename T, bool kNN, int BN>
+__global__ void __launch_bounds__(128, 1)
+    gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                const GemmParams p) {
+  using C = GemmCfg<T, kNN, BN>;
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = ptx::smem_u32(smem_raw);
+  uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
+
+  const int warp = threadIdx.x >> 5;
+  const int64_t m0 = (int64_t)blockIdx.x * C::BM;
+  const int64_t n0 = (int64_t)blockIdx.y * BN;
+  const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;
+  const int64_t kb1 = min(p.kb_total, kb0 + p.kb_per_split);
+  const int nkb = (int)(kb1 - kb0);
+
+  if (warp == 0 && ptx::elect_one()) {
+    ptx::tma_prefetch_desc(&mapA);
+    ptx::tma_prefetch_desc(&mapB);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    ptx::mbar_init(tfull, 1);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 2) ptx::tmem_alloc<C::TMEM_COLS>(tslot);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0) {
+    // ---------------- TMA producer ----------------
+    if (ptx::elect_one()) {
+      for (int it = 0; it < nkb; ++it) {
+        const int s = it % C::STAGES;
+        const uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
+        ptx::mbar_wait(&empty[s], ph ^ 1u);
+        uint8_t* sA = smem + s * C::STAGE_BYTES;
+        uint8_t* sB = sA + C::A_BYTES;
+        const int32_t k0 = (int32_t)((kb0 + it) * C::BK);
+        ptx::mbar_arrive_expect_tx(&full[s], C::STAGE_BYTES);
+        if constexpr (kNN) {
+#pragma unroll
+          for (int mb = 0; mb < C::BM / C::EPB; ++mb)
+            ptx::tma_load_2d(sA + mb * C::BK * 128, &mapA, &full[s], (int32_t)(m0 + mb * C::EPB), k0);
+        } else {
+          ptx::tma_load_2d(sA, &mapA, &full[s], k0, (int32_t)m0);
+        }
+        ptx::tma_load_2d(sB, &mapB, &full[s], k0, (int32_t)n0);
+      }
+    }
+  } else if (warp == 1) {
+    // ---------------- MMA issuer ----------------
+    if (ptx::elect_one()) {
+      for (int it = 0; it < nkb; ++it) {
+        const int s = it % C::STAGES;
+        const uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
+        ptx::mbar_wait(&full[s], ph);
+        ptx::tc_fence_after();
+        const uint32_t aBase = ptx::smem_u32(smem + s * C::STAGE_BYTES);
+        const uint32_t bBase = aBase + C::A_BYTES;
+#pragma unroll
+        for (int kk = 0; kk < C::BK / C::UK; ++kk) {
+          uint64_t ad;
+          if constexpr (kNN && Elem<T>::kTF32)
+            ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 512, 1);
+          else if constexpr (kNN)
+            ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 1024);
+          else
+            ad = ptx::sdesc_sw128(aBase + kk * C::UK * (int)sizeof(T), 16, 1024);
+          const uint64_t bd = ptx::sdesc_sw128(bBase + kk * C::UK * (int)sizeof(T), 16, 1024);
+          ptx::umma<Elem<T>::kTF32>(tmem, ad, bd, C::IDESC, (it | kk) != 0 ? 1u : 0u);
+        }
+        ptx::umma_commit(&empty[s]);
+      }
+      ptx::umma_commit(tfull);
+    }
+  }
+  __syncwarp();
+
+  // ---------------- epilogue: all four warps ----------------
+  if (nkb > 0) ptx::mbar_wait(tfull, 0);
+  ptx::tc_fence_after();
+  const int lane = threadIdx.x & 31;
+  const int64_t i = m0 + warp * 32 + lane;
+  const bool row_ok = i < p.M;
+#pragma unroll 1
+  for (int cc = 0; cc < BN / 32; ++cc) {
+    uint32_t v[32];
+    if (nkb > 0) {
+      ptx::tmem_ld_32x32b_x32(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(cc * 32), v);
+      ptx::tmem_ld_wait();
+    } else {
+#pragma unroll
+      for (int j = 0; j < 32; ++j) v[j] = 0u;
+    }
+    if (!row_ok) continue;
+    const int64_t nb = n0 + cc * 32;
+#pragma unroll
+    for (int j = 0; j < 32; ++j) {
+      const int64_t n = nb + j;
+      if (n >= p.N) break;
+      const float x = __uint_as_float(v[j]);
+      if constexpr (kNN) {
+        T* a = reinterpret_cast<T*>(p.A2) + i + n * p.lda2;
+        *a = Elem<T>::store(Elem<T>::load(*a) - x);
+      } else {
+        if (p.P != nullptr) {
+          p.P[blockIdx.z * p.split_stride + i + n * p.ldp] = x;
+        } else {
+          float* c = p.C + i + n * p.ldc;
+          const float y = p.accumulate ? *c + x : x;
+          *c = y;
+          if (p.Cop != nullptr) reinterpret_cast<T*>(p.Cop)[i + n * p.ldop] = Elem<T>::store(y);
+        }
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<C::TMEM_COLS>(tmem);
+  }
+}
+
+// ---------------------------------------------------------------------------------
+// Deterministic split-K reduction: C = (accumulate ? C : 0) + sum_{s=0..S-1} P[s] in
+// a fixed order (no float atomics; R10), plus the optional operand copy.
+// ---------------------------------------------------------------------------------
+template <typename T>
+__global__ void splitk_reduce_kernel(const float* __restrict__ P, int64_t split_stride, int64_t ldp,
+                                     int splits, float* C, int64_t ldc, int accumulate, T* Cop,
+                                     int64_t ldop, int64_t M, int64_t N) {
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= M * N) return;
+  const int64_t i = idx % M, n = idx / M;
+  float acc = accumulate ? C[i + n * ldc] : 0.0f;
+  for (int s = 0; s < splits; ++s) acc += P[s * split_stride + i + n * ldp];
+  C[i + n * ldc] = acc;
+  if (Cop != nullptr) Cop[i + n * ldop] = Elem<T>::store(acc);
+}
+
+// ---------------------------------------------------------------------------------
+// host-side launch helpers
+// ---------------------------------------------------------------------------------
+template <typename T, bool kNN, int BN>
+static cudaError_t launch_gemm_t(const CUtensorMap& ma, const CUtensorMap& mb, const GemmParams& p,
+                                 int splits, cudaStream_t st) {
+  using C = GemmCfg<T, kNN, BN>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(gemm_kernel<T, kNN, BN>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  dim3 grid((unsigned)((p.M + C::BM - 1) / C::BM), (unsigned)((p.N + BN - 1) / BN), (unsigned)splits);
+  gemm_kernel<T, kNN, BN><<<grid, 128, C::SMEM, st>>>(ma, mb, p);
+  return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMap& mb,
+                        const GemmParams& p, int splits, cudaStream_t st) {
+  if (nn) {
+    if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, p, splits, st);
+    if (bn == 128) return launch_gemm_t<T, true, 128>(ma, mb, p, splits, st);
+    return launch_gemm_t<T, true, 64>(ma, mb, p, splits, st);
+  }
+  if (bn == 256) return launch_gemm_t<T, false, 256>(ma, mb, p, splits, st);
+  if (bn == 128) return launch_gemm_t<T, false, 128>(ma, mb, p, splits, st);
+  return launch_gemm_t<T, false, 64>(ma, mb, p, splits, st);
+}
+
+template <typename T>
+cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t ldp, int splits,
+                                 float* C, int64_t ldc, int accumulate, T* Cop, int64_t ldop,
+                                 int64_t M, int64_t N, cudaStream_t st) {
+  const int64_t total = M * N;
+  const int threads = 256;
+  splitk_reduce_kernel<T><<<(unsigned)((total + threads - 1) / threads), threads, 0, st>>>(
+      P, split_stride, ldp, splits, C, ldc, accumulate, Cop, ldop, M, N);
+  return cudaGetLastError();
+}
+
+int gemm_block_k(int elem_bytes) { return 128 / elem_bytes; }
+
+template cudaError_t launch_gemm<__half>(bool, int, const CUtensorMap&, const CUtensorMap&,
+                                         const GemmParams&, int, cudaStream_t);
+template cudaError_t launch_gemm<__nv_bfloat16>(bool, int, const CUtensorMap&, const CUtensorMap&,
+                                                const GemmParams&, int, cudaStream_t);
+template cudaError_t launch_gemm<float>(bool, int, const CUtensorMap&, const CUtensorMap&,
+                                        const GemmParams&, int, cudaStream_t);
+template cudaError_t launch_splitk_reduce<__half>(const float*, int64_t, int64_t, int, float*, int64_t,
+                                                  int, __half*, int64_t, int64_t, int64_t, cudaStream_t);
+template cudaError_t launch_splitk_reduce<__nv_bfloat16>(const float*, int64_t, int64_t, int, float*,
+                                                         int64_t, int, __nv_bfloat16*, int64_t, int64_t,
+                                                         int64_t, cudaStream_t);
+template cudaError_t launch_splitk_reduce<float>(const float*, int64_t, int64_t, int, float*, int64_t,
+                                                 int, float*, int64_t, int64_t, int64_t, cudaStream_t);
+
+}  // namespace rgsqr

@@ -1,0 +1,61 @@
+// kernels.h -- internal launch interface of the device kernels (not part of the C ABI).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace rgsqr {
+
+constexpr int LEAF_MAX_W = 64;
+constexpr size_t LEAF_SMEM_BUDGET = 200 * 1024;
+
+struct GemmParams {
+  int64_t M, N, K;          // D[M x N] = sum_k A[M x K] B[N x K]^T (see gemm.cu)
+  int64_t kb_total;         // K blocks of gemm_block_k() elements
+  int64_t kb_per_split;     // K blocks per grid.z slice
+  // inner product (TN) epilogue
+  float* C;                 // fp32 output, ldc
+  int64_t ldc;
+  int accumulate;           // C += result
+  void* Cop;                // optional operand-typed copy, ldop
+  int64_t ldop;
+  float* P;                 // split-K partials (non-null => write partials instead of C)
+  int64_t ldp;
+  int64_t split_stride;
+  // outer product (NN) epilogue: A2 <- A2 - result
+  void* A2;
+  int64_t lda2;
+};
+
+struct LeafParams {
+  void* P;                  // panel m x w (ldp), overwritten by Q
+  int64_t ldp;
+  int64_t m;
+  int w;
+  int rows_per_cta;
+  float* R;                 // w x w block of R (ldr)
+  int64_t ldr;
+  float* partials;          // [2][LEAF_MAX_W+2][grid]
+  unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
+  int* breakdown;           // device int, atomicMin of the first breakdown column
+  int64_t col_offset;       // global index of the panel's first column
+};
+
+int gemm_block_k(int elem_bytes);
+int leaf_max_smem_rows(int w);
+
+template <typename T>
+cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMap& mb,
+                        const GemmParams& p, int splits, cudaStream_t st);
+template <typename T>
+cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t ldp, int splits,
+                                 float* C, int64_t ldc, int accumulate, T* Cop, int64_t ldop,
+                                 int64_t M, int64_t N, cudaStream_t st);
+template <typename T>
+cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st);
+
+template <typename T>
+cudaError_t launch_cast(const float* src, int64_t lds, T* dst, int64_t ldd, int64_t M, int64_t N,
+                        cudaStream_t st);
+
+}  // namespace rgsqr

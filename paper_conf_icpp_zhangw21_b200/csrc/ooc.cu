@@ -1,0 +1,491 @@
+// ooc.cu -- host-resident (out-of-core) recursive CGS QR: the executor.
+//
+// The recursion of Eq. (2) is walked on the host.  A node whose
+// columns fit the device arena (the budget) is factored IN-CORE by the
+// device recursion of ops.cu, its columns uploaded in chunks that the recursion waits
+// on progressively, and its Q columns downloaded as soon as each leaf finishes
+// (cross-operation overlap).  A node that does not fit is OUT-OF-CORE:
+//
+//   left child  -> inner product R12 = Q1^T A2, row tiles streamed (Fig. 3)
+//               -> R12 out once at the end
+//               -> outer product A2 <- A2 - Q1 R12, R12 resident, row tiles in and out
+//                  (Fig. 5)
+//   right child
+//
+// Row tiles move through a K-slot device ring on three streams (h2d copy engine,
+// compute, d2h copy engine) chained by events: loaded[s] -> kernel -> done[s] -> d2h
+// -> free[s] -> next upload into s.  Tile height ramps from tile_rows_min up to the
+// slot size.  QR-level reuse, when it fits the budget:
+//   rule 1: the left child's Q1 stays resident after its in-core factorization, so
+//           both products stream only A2 tiles;
+//   rule 3: each A2' tile is written over the rows of Q1 it no longer needs (after
+//           Q1 was downloaded) instead of back to the host, so the right child starts
+//           in-core without re-reading A2'  (the paper's "fast in-core data
+//           transferring" D2D copy, used here to build the resident A2').
+// The blocked algorithm (option ALGO=1) reuses the same node primitives
+// with a fixed panel width instead of the recursion.
+#include <chrono>
+#include <climits>
+#include <cstring>
+#include <thread>
+#include <vector>
+
+#include "engine.h"
+
+namespace rgsqr {
+int ensure_arena(Ctx* c, size_t want);
+size_t resolve_budget(Ctx* c, size_t budget);
+void reset_stats(Ctx* c);
+int validate(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, const void* Q, int prec);
+
+namespace {
+
+struct Exec {
+  Ctx* c;
+  int prec;
+  int64_t s;
+  const char* A;
+  char* Q;
+  int64_t lda, m, n;
+  float* R;
+  cudaStream_t sc, sh, sd;
+  int K;
+  int64_t tmin, tmax;
+  bool reuse;
+
+  // ---- timing / accounting helpers ----
+  cudaEvent_t seg_begin(cudaStream_t st) {
+    cudaEvent_t e = c->ev();
+    cudaEventRecord(e, st);
+    return e;
+  }
+  void seg_end(int kind, cudaStream_t st, cudaEvent_t a) {
+    cudaEvent_t b = c->ev();
+    cudaEventRecord(b, st);
+    c->segs.push_back({kind, a, b});
+  }
+  void wait(cudaStream_t waiter, cudaStream_t signaller) {
+    if (waiter == signaller) return;
+    cudaEvent_t e = c->ev();
+    cudaEventRecord(e, signaller);
+    cudaStreamWaitEvent(waiter, e, 0);
+  }
+  void join_all() {
+    wait(sc, sh);
+    wait(sc, sd);
+    wait(sh, sc);
+    wait(sd, sc);
+  }
+  const char* hsrc(bool q) const { return q ? Q : A; }
+  const char* hptr(const char* base, int64_t r0, int64_t col) const { return base + (r0 + col * lda) * s; }
+
+  int h2d(void* dst, int64_t ldd, const char* base, int64_t r0, int64_t rows, int64_t c0, int64_t cols) {
+    cudaEvent_t a = seg_begin(sh);
+    RGSQR_CUDA(c, cudaMemcpy2DAsync(dst, ldd * s, hptr(base, r0, c0), lda * s, rows * s, cols,
+                                    cudaMemcpyHostToDevice, sh));
+    seg_end(0, sh, a);
+    c->stats.h2d_bytes += rows * cols * s;
+    c->stats.h2d_matrix_bytes += rows * cols * s;
+    return RGSQR_OK;
+  }
+  int d2h(char* base, int64_t r0, int64_t rows, int64_t c0, int64_t cols, const void* src, int64_t lds) {
+    cudaEvent_t a = seg_begin(sd);
+    RGSQR_CUDA(c, cudaMemcpy2DAsync(const_cast<char*>(hptr(base, r0, c0)), lda * s, src, lds * s, rows * s, cols,
+                                    cudaMemcpyDeviceToHost, sd));
+    seg_end(1, sd, a);
+    c->stats.d2h_bytes += rows * cols * s;
+    c->stats.d2h_matrix_bytes += rows * cols * s;
+    return RGSQR_OK;
+  }
+  int d2h_r(int64_t r0, int64_t c0, int64_t rows, int64_t cols, const float* src, int64_t lds) {
+    if (!R) return RGSQR_OK;  // non-zero ranks of a distributed run
+    cudaEvent_t a = seg_begin(sd);
+    RGSQR_CUDA(c, cudaMemcpy2DAsync(R + r0 + c0 * n, n * sizeof(float), src, lds * sizeof(float),
+                                    rows * sizeof(float), cols, cudaMemcpyDeviceToHost, sd));
+    seg_end(1, sd, a);
+    c->stats.d2h_bytes += rows * cols * 4;
+    c->stats.d2h_r_bytes += rows * cols * 4;
+    return RGSQR_OK;
+  }
+
+  // ---- sizing ----
+  size_t incore_need(int64_t w) const {
+    return (size_t)m * w * s + 256 + (size_t)w * w * 4 + 256 + incore_workspace_bytes(c, prec, m, w) + 4096;
+  }
+  std::vector<int64_t> tiles(int64_t t) const {
+    std::vector<int64_t> v;
+    int64_t r = 0, cur = std::min(tmin, t);
+    while (r < m) {
+      int64_t h = std::min(cur, m - r);
+      v.push_back(h);
+      r += h;
+      cur = std::min(t, cur * 2);  // ramp
+    }
+    return v;
+  }
+  int64_t pick_tile(size_t avail, int64_t cols_per_slot) const {
+    int64_t t = (int64_t)(avail / ((size_t)K * cols_per_slot * s));
+    t = std::min<int64_t>(t, tmax);
+    t = std::min<int64_t>(t, (m + 127) / 128 * 128);
+    t = t / 128 * 128;
+    return t;
+  }
+
+  // ---- in-core node: upload (unless resident), factor, stream Q and R out ----
+  int incore_node(int64_t c0, int64_t w, bool src_q, char* D, bool resident, cudaEvent_t* q_done) {
+    const size_t mark = c->arena.mark();
+    float* Rs = static_cast<float*>(c->arena.alloc((size_t)w * w * 4));
+    if (!Rs) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core node: no space for R block");
+    RGSQR_CUDA(c, cudaMemsetAsync(Rs, 0, (size_t)w * w * 4, sc));
+    const int64_t leaf = std::max(1, leaf_width_for(c, m));
+    int64_t cw = ((int64_t)32 << 20) / std::max<int64_t>(1, m * s);
+    cw = std::max<int64_t>(leaf, cw / 64 * 64);
+    std::vector<std::pair<int64_t, cudaEvent_t>> chunks;
+    if (!resident) {
+      for (int64_t a = 0; a < w; a += cw) {
+        const int64_t cols = std::min(cw, w - a);
+        int rc = h2d(D + a * m * s, m, hsrc(src_q), 0, m, c0 + a, cols);
+        if (rc < 0) return rc;
+        cudaEvent_t e = c->ev();
+        cudaEventRecord(e, sh);
+        chunks.push_back({a, e});
+      }
+    }
+    size_t next = 0;
+    int64_t flushed = 0;
+    int err = 0;
+    IncoreHooks hk;
+    hk.need = [&](int64_t col_end) {
+      while (next < chunks.size() && chunks[next].first < col_end) {
+        cudaStreamWaitEvent(sc, chunks[next].second, 0);
+        ++next;
+      }
+    };
+    hk.leaf_done = [&](int64_t col_end) {
+      if (col_end - flushed < cw && col_end < w) return;
+      wait(sd, sc);
+      int rc = d2h(Q, 0, m, c0 + flushed, col_end - flushed, D + flushed * m * s, m);
+      if (rc < 0) err = rc;
+      flushed = col_end;
+    };
+    cudaEvent_t a = seg_begin(sc);
+    int rc = incore_factor(c, prec, D, m, m, w, Rs, w, c0, sc, &hk);
+    if (rc < 0) return rc;
+    if (err < 0) return err;
+    seg_end(2, sc, a);
+    hk.need(w);  // (no-op unless the recursion skipped columns)
+    wait(sd, sc);
+    if (flushed < w) {
+      rc = d2h(Q, 0, m, c0 + flushed, w - flushed, D + flushed * m * s, m);
+      if (rc < 0) return rc;
+    }
+    rc = d2h_r(c0, c0, w, w, Rs, w);
+    if (rc < 0) return rc;
+    cudaEvent_t done = c->ev();
+    cudaEventRecord(done, sd);
+    if (q_done) *q_done = done;
+    // the R block lives in the arena: nobody may reuse it before its download finished
+    cudaStreamWaitEvent(sc, done, 0);
+    cudaStreamWaitEvent(sh, done, 0);
+    c->arena.release(mark);
+    return RGSQR_OK;
+  }
+
+  // ---- streamed inner product  R12 = Q1^T A2  (Q1 resident in D when D != null) ----
+  int stream_inner(int64_t c0, int64_t w1, int64_t w2, bool a2_src_q, const char* D, float* R12, void* R12op,
+                   char* ring, int64_t t, std::vector<cudaEvent_t>& ev_free) {
+    const int64_t h = c0 + w1;
+    const int64_t slot_cols = (D ? 0 : w1) + w2;
+    std::vector<cudaEvent_t> loaded(K);
+    for (int k = 0; k < K; ++k) loaded[k] = c->ev();
+    auto tl = tiles(t);
+    int64_t r0 = 0;
+    for (size_t i = 0; i < tl.size(); ++i) {
+      const int64_t tr = tl[i];
+      const int k = (int)(i % K);
+      char* slot = ring + (size_t)k * t * slot_cols * s;
+      char* sq = slot;
+      char* sa = slot + (D ? 0 : (size_t)t * w1 * s);
+      cudaStreamWaitEvent(sh, ev_free[k], 0);
+      if (!D) {
+        int rc = h2d(sq, t, Q, r0, tr, c0, w1);
+        if (rc < 0) return rc;
+      }
+      int rc = h2d(sa, t, hsrc(a2_src_q), r0, tr, h, w2);
+      if (rc < 0) return rc;
+      cudaEventRecord(loaded[k], sh);
+      cudaStreamWaitEvent(sc, loaded[k], 0);
+      cudaEvent_t a = seg_begin(sc);
+      const bool last = (i + 1 == tl.size());
+      rc = op_inner(c, prec, D ? D + r0 * s : sq, D ? m : t, sa, t, tr, w1, w2, R12, w1, last ? R12op : nullptr,
+                    w1, i > 0 ? 1 : 0, sc);
+      if (rc < 0) return rc;
+      seg_end(2, sc, a);
+      cudaEventRecord(ev_free[k], sc);
+      r0 += tr;
+    }
+    return RGSQR_OK;
+  }
+
+  // ---- streamed outer product  A2 <- A2 - Q1 R12 ----
+  // to_D: write A2' over Q1's rows in D (reuse rule 3) instead of downloading it.
+  int stream_outer(int64_t c0, int64_t w1, int64_t w2, bool a2_src_q, char* D, bool to_D, cudaEvent_t q1_out_done,
+                   const void* R12op, char* ring, int64_t t, std::vector<cudaEvent_t>& ev_free) {
+    const int64_t h = c0 + w1;
+    const int64_t slot_cols = (D ? 0 : w1) + w2;
+    std::vector<cudaEvent_t> loaded(K), done(K);
+    for (int k = 0; k < K; ++k) {
+      loaded[k] = c->ev();
+      done[k] = c->ev();
+    }
+    if (to_D && q1_out_done) cudaStreamWaitEvent(sc, q1_out_done, 0);
+    auto tl = tiles(t);
+    int64_t r0 = 0;
+    for (size_t i = 0; i < tl.size(); ++i) {
+      const int64_t tr = tl[i];
+      const int k = (int)(i % K);
+      char* slot = ring + (size_t)k * t * slot_cols * s;
+      char* sq = slot;
+      char* sa = slot + (D ? 0 : (size_t)t * w1 * s);
+      cudaStreamWaitEvent(sh, ev_free[k], 0);
+      if (!D) {
+        int rc = h2d(sq, t, Q, r0, tr, c0, w1);
+        if (rc < 0) return rc;
+      }
+      int rc = h2d(sa, t, hsrc(a2_src_q), r0, tr, h, w2);
+      if (rc < 0) return rc;
+      cudaEventRecord(loaded[k], sh);
+      cudaStreamWaitEvent(sc, loaded[k], 0);
+      cudaEvent_t a = seg_begin(sc);
+      rc = op_outer(c, prec, D ? D + r0 * s : sq, D ? m : t, R12op, w1, sa, t, tr, w1, w2, sc);
+      if (rc < 0) return rc;
+      if (to_D) {
+        RGSQR_CUDA(c, cudaMemcpy2DAsync(D + r0 * s, m * s, sa, t * s, tr * s, w2, cudaMemcpyDeviceToDevice, sc));
+        c->stats.d2d_bytes += tr * w2 * s;
+        seg_end(2, sc, a);
+        cudaEventRecord(ev_free[k], sc);
+      } else {
+        seg_end(2, sc, a);
+        cudaEventRecord(done[k], sc);
+        cudaStreamWaitEvent(sd, done[k], 0);
+        rc = d2h(Q, r0, tr, h, w2, sa, t);
+        if (rc < 0) return rc;
+        cudaEventRecord(ev_free[k], sd);
+      }
+      r0 += tr;
+    }
+    return RGSQR_OK;
+  }
+
+  // ---- one out-of-core node: left, inner, outer, right ----
+  // recursive = true: children are recursive nodes; false: blocked (left = panel,
+  // right handled by the caller's loop).
+  int ooc_node(int64_t c0, int64_t w1, int64_t w2, bool src_q, bool recursive) {
+    c->stats.n_ooc_nodes++;
+    const int64_t h = c0 + w1;
+    const size_t mark0 = c->arena.mark();
+    const size_t r12b = (size_t)w1 * w2 * 4 + 256, r12ob = (size_t)w1 * w2 * s + 256;
+    // ---- reuse plan (rules 1 and 3) ----
+    const size_t free0 = c->arena.free_bytes();
+    const size_t dB = (size_t)m * w1 * s + 256;
+    const size_t left_ws = incore_need(w1) - dB;
+    const size_t right_ws = incore_need(w2) - (size_t)m * w2 * s;
+    bool q1_res = reuse && dB + r12b + r12ob + left_ws + (size_t)K * 128 * w2 * s <= free0;
+    bool a2_to_d = q1_res && recursive && w2 <= w1 && dB + right_ws <= free0;
+    if (q1_res) {
+      char* D = static_cast<char*>(c->arena.alloc(dB));
+      float* R12 = static_cast<float*>(c->arena.alloc(r12b));
+      void* R12op = c->arena.alloc(r12ob);
+      // ring sized to leave room for the left child's in-core workspace
+      const size_t avail = c->arena.free_bytes() > left_ws + 4096 ? c->arena.free_bytes() - left_ws - 4096 : 0;
+      const int64_t t = pick_tile(avail, w2);
+      if (!D || !R12 || !R12op || t < 128) {
+        c->arena.release(mark0);
+        q1_res = a2_to_d = false;
+      } else {
+        char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * w2 * s));
+        std::vector<cudaEvent_t> ev_free(K);
+        for (int k = 0; k < K; ++k) ev_free[k] = c->ev();
+        cudaEvent_t q1_done = nullptr;
+        int rc = incore_node(c0, w1, src_q, D, false, &q1_done);
+        if (rc < 0) return rc;
+        rc = stream_inner(c0, w1, w2, src_q, D, R12, R12op, ring, t, ev_free);
+        if (rc < 0) return rc;
+        wait(sd, sc);
+        rc = d2h_r(c0, h, w1, w2, R12, w1);
+        if (rc < 0) return rc;
+        cudaEvent_t r12_out = c->ev();
+        cudaEventRecord(r12_out, sd);
+        rc = stream_outer(c0, w1, w2, src_q, D, a2_to_d, q1_done, R12op, ring, t, ev_free);
+        if (rc < 0) return rc;
+        // R12 / ring memory is released below: make every stream wait for its last users
+        cudaStreamWaitEvent(sc, r12_out, 0);
+        join_all();
+        c->arena.release(mark0 + 0);
+        if (a2_to_d) {
+          // keep D (now holding A2', rows permuted by nothing: same row order) for the right child
+          char* D2 = static_cast<char*>(c->arena.alloc(dB));  // same address as D (LIFO)
+          (void)D2;
+          rc = incore_node(h, w2, true, D, true, nullptr);
+          if (rc < 0) return rc;
+          join_all();
+          c->arena.release(mark0);
+          return RGSQR_OK;
+        }
+        c->arena.release(mark0);
+        return recursive ? node(h, w2, true) : RGSQR_OK;
+      }
+    }
+    // ---- no reuse: Q1 tiles are re-read from the host ----
+    int rc = recursive ? node(c0, w1, src_q) : panel(c0, w1, src_q);
+    if (rc < 0) return rc;
+    join_all();
+    float* R12 = static_cast<float*>(c->arena.alloc(r12b));
+    void* R12op = c->arena.alloc(r12ob);
+    if (!R12 || !R12op) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: no space for R12");
+    const int64_t t = pick_tile(c->arena.free_bytes() > 4096 ? c->arena.free_bytes() - 4096 : 0, w1 + w2);
+    if (t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: ring does not fit the budget");
+    char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
+    std::vector<cudaEvent_t> ev_free(K);
+    for (int k = 0; k < K; ++k) ev_free[k] = c->ev();
+    rc = stream_inner(c0, w1, w2, src_q, nullptr, R12, R12op, ring, t, ev_free);
+    if (rc < 0) return rc;
+    wait(sd, sc);
+    rc = d2h_r(c0, h, w1, w2, R12, w1);
+    if (rc < 0) return rc;
+    rc = stream_outer(c0, w1, w2, src_q, nullptr, false, nullptr, R12op, ring, t, ev_free);
+    if (rc < 0) return rc;
+    join_all();
+    c->arena.release(mark0);
+    return recursive ? node(h, w2, true) : RGSQR_OK;
+  }
+
+  int panel(int64_t c0, int64_t w, bool src_q) {
+    const size_t mark = c->arena.mark();
+    char* D = static_cast<char*>(c->arena.alloc((size_t)m * w * s));
+    if (!D || c->arena.free_bytes() + 0 < incore_need(w) - (size_t)m * w * s)
+      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "panel of " + std::to_string(w) + " columns does not fit");
+    int rc = incore_node(c0, w, src_q, D, false, nullptr);
+    if (rc < 0) return rc;
+    join_all();
+    c->arena.release(mark);
+    return RGSQR_OK;
+  }
+
+  // recursive algorithm (Eq. 2)
+  int node(int64_t c0, int64_t w, bool src_q) {
+    if (incore_need(w) <= c->arena.free_bytes()) return panel(c0, w, src_q);
+    const int64_t w1 = split_width(w, std::max(1, leaf_width_for(c, m)));
+    if (w1 == 0) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "budget cannot hold one leaf panel");
+    return ooc_node(c0, w1, w - w1, src_q, true);
+  }
+
+  // blocked algorithm: panels of width b, trailing update streamed
+  int blocked(int64_t b) {
+    for (int64_t c0 = 0; c0 < n; c0 += b) {
+      const int64_t w1 = std::min(b, n - c0), w2 = n - c0 - w1;
+      int rc = (w2 == 0) ? panel(c0, w1, c0 > 0) : ooc_node(c0, w1, w2, c0 > 0, false);
+      if (rc < 0) return rc;
+    }
+    return RGSQR_OK;
+  }
+};
+
+}  // namespace
+
+int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* Q, float* R, int prec,
+                size_t budget) {
+  int rc = validate(c, A, lda, m, n, Q, prec);
+  if (rc < 0) return rc;
+  if (!R && c->rank == 0) return fail(c, RGSQR_ERR_INVALID_ARG, "null R_out");
+  if (c->nranks > 1) return fail(c, RGSQR_ERR_UNSUPPORTED, "row-sharded multi-GPU factorization not built yet");
+  reset_stats(c);
+  c->segs.clear();
+  c->event_next = 0;
+  const int s = elem_bytes(prec);
+
+  // ---- page-lock caller buffers (timed separately) ----
+  auto tp0 = std::chrono::steady_clock::now();
+  std::vector<void*> registered;
+  auto pin = [&](const void* p, size_t bytes) -> int {
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+      cudaGetLastError();
+      at.type = cudaMemoryTypeUnregistered;
+    }
+    if (at.type == cudaMemoryTypeUnregistered) {
+      for (void* q : registered)
+        if (q == p) return RGSQR_OK;
+      if (cudaHostRegister(const_cast<void*>(p), bytes, cudaHostRegisterPortable) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, RGSQR_ERR_HOST_MEM, "cudaHostRegister failed");
+      }
+      registered.push_back(const_cast<void*>(p));
+    }
+    return RGSQR_OK;
+  };
+  const size_t abytes = ((size_t)lda * (n - 1) + m) * s;
+  if ((rc = pin(A, abytes)) < 0 || (rc = pin(Q, abytes)) < 0 || (R && (rc = pin(R, (size_t)n * n * 4)) < 0)) {
+    for (void* p : registered) cudaHostUnregister(p);
+    return rc;
+  }
+  auto tp1 = std::chrono::steady_clock::now();
+
+  // ---- device arena = the budget ----
+  const size_t persistent = (size_t)2 * (LEAF_MAX_W + 2) * 1024 * 4 + 512;
+  size_t cap = resolve_budget(c, budget);
+  cap = cap > persistent ? cap - persistent : 0;
+  auto t0 = std::chrono::steady_clock::now();
+  rc = ensure_arena(c, cap);
+  if (rc < 0) {
+    for (void* p : registered) cudaHostUnregister(p);
+    return rc;
+  }
+  Exec x{c, prec, s, static_cast<const char*>(A), static_cast<char*>(Q), lda, m, n, R,
+         c->compute(), c->st_h2d, c->st_d2h, (int)c->opt.ring_depth, c->opt.tile_rows_min,
+         c->opt.tile_rows_max, c->opt.reuse != 0};
+  if (c->opt.serialize) x.sh = x.sd = x.sc;
+  // make the copy streams start after prior work of the compute stream
+  x.join_all();
+  RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), x.sc));
+  std::thread zero;
+  if (R)
+    zero = std::thread([R, n] {
+      for (int64_t j = 0; j + 1 < n; ++j) std::memset(R + j * n + j + 1, 0, (size_t)(n - j - 1) * 4);
+    });
+  rc = c->opt.algo == 1 ? x.blocked(std::min<int64_t>(c->opt.block_cols, n)) : x.node(0, n, false);
+  int brk = INT_MAX;
+  if (rc >= 0) {
+    x.join_all();
+    cudaMemcpyAsync(&brk, c->d_breakdown, sizeof(int), cudaMemcpyDeviceToHost, x.sc);
+  }
+  cudaError_t e1 = cudaStreamSynchronize(x.sc);
+  cudaError_t e2 = cudaStreamSynchronize(c->st_h2d);
+  cudaError_t e3 = cudaStreamSynchronize(c->st_d2h);
+  if (zero.joinable()) zero.join();
+  auto t1 = std::chrono::steady_clock::now();
+  for (void* p : registered) cudaHostUnregister(p);
+  if (rc < 0) return rc;
+  if (e1 != cudaSuccess || e2 != cudaSuccess || e3 != cudaSuccess)
+    return fail(c, RGSQR_ERR_CUDA, std::string("stream error: ") +
+                                       cudaGetErrorString(e1 != cudaSuccess ? e1 : (e2 != cudaSuccess ? e2 : e3)));
+  // ---- stats ----
+  auto& st = c->stats;
+  st.pin_ms = std::chrono::duration<double, std::milli>(tp1 - tp0).count();
+  st.wall_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+  for (auto& sg : c->segs) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, sg.a, sg.b);
+    (sg.kind == 0 ? st.h2d_busy_ms : sg.kind == 1 ? st.d2h_busy_ms : st.compute_busy_ms) += ms;
+  }
+  const double sum = st.h2d_busy_ms + st.d2h_busy_ms + st.compute_busy_ms;
+  const double mx = std::max({st.h2d_busy_ms, st.d2h_busy_ms, st.compute_busy_ms});
+  st.overlap_ratio = sum - mx > 1e-9 ? std::min(1.0, std::max(0.0, (sum - st.wall_ms) / (sum - mx))) : 0.0;
+  st.arena_bytes = (int64_t)c->arena.size;
+  st.arena_high_water = (int64_t)c->arena.high;
+  st.flops = (int64_t)(2.0 * m * (double)n * n);
+  st.first_breakdown_col = (brk == 0x7f7f7f7f || brk == INT_MAX) ? -1 : brk;
+  return st.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;
+}
+
+}  // namespace rgsqr

@@ -1,0 +1,303 @@
+// ops.cu -- host launchers of the hot-path operations and the in-core recursion (Eq. 2).
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <climits>
+#include <mutex>
+
+#include "engine.h"
+
+namespace rgsqr {
+
+int elem_bytes(int precision) { return (precision == RGSQR_FP16 || precision == RGSQR_BF16) ? 2 : 4; }
+
+int fail(Ctx* c, int status, const std::string& msg) {
+  if (c) c->last_error = msg;
+  return status;
+}
+
+cudaEvent_t Ctx::ev() {
+  if (event_next == event_pool.size()) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    event_pool.push_back(e);
+  }
+  return event_pool[event_next++];
+}
+
+// ---------------------------------------------------------------------------------
+// TMA descriptors (driver entry point fetched through the runtime; no -lcuda)
+// ---------------------------------------------------------------------------------
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &p, 12000, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+bool encode_tmap_2d(CUtensorMap* map, int precision, const void* base, uint64_t inner, uint64_t outer,
+                    uint64_t outer_stride_bytes, uint32_t box_inner, uint32_t box_outer, std::string* err,
+                    bool atom32) {
+  auto enc = get_encode();
+  if (!enc) {
+    *err = "cuTensorMapEncodeTiled unavailable";
+    return false;
+  }
+  CUtensorMapDataType dt = precision == RGSQR_FP16   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                           : precision == RGSQR_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                                     : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {outer_stride_bytes};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(map, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   atom32 ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    *err = "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ") dims=" + std::to_string(inner) + "x" +
+           std::to_string(outer) + " stride=" + std::to_string(outer_stride_bytes);
+    return false;
+  }
+  return true;
+}
+
+static int pick_bn(int64_t N) { return N >= 256 ? 256 : (N > 64 ? 128 : 64); }
+
+template <typename T>
+static int op_inner_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
+                      int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate,
+                      cudaStream_t st) {
+  const int s = (int)sizeof(T);
+  const int BK = gemm_block_k(s);
+  const int bn = pick_bn(w2);
+  CUtensorMap ma, mb;
+  std::string err;
+  if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, BK, 128, &err) ||
+      !encode_tmap_2d(&mb, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, BK, bn, &err))
+    return fail(c, RGSQR_ERR_INVALID_ARG, "inner: " + err);
+  GemmParams p{};
+  p.M = w1;
+  p.N = w2;
+  p.K = m;
+  p.kb_total = (m + BK - 1) / BK;
+  const int64_t tiles = ((w1 + 127) / 128) * ((w2 + bn - 1) / bn);
+  int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : (c->num_sms + tiles - 1) / tiles);
+  splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.kb_total / 4));
+  const size_t cap = std::min<size_t>((size_t)64 << 20, c->arena.free_bytes());
+  while (splits > 1 && (size_t)splits * w1 * w2 * 4 + 256 > cap) --splits;
+  p.kb_per_split = (p.kb_total + splits - 1) / splits;
+  splits = (p.kb_total + p.kb_per_split - 1) / p.kb_per_split;
+  if (p.kb_total == 0) {
+    p.kb_per_split = 1;
+    splits = 1;
+  }
+  size_t mark = c->arena.mark();
+  if (splits > 1) {
+    float* P = static_cast<float*>(c->arena.alloc((size_t)splits * w1 * w2 * sizeof(float)));
+    if (!P) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner: no arena space for split-K partials");
+    p.P = P;
+    p.ldp = w1;
+    p.split_stride = w1 * w2;
+    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, (int)splits, st));
+    RGSQR_CUDA(c, launch_splitk_reduce<T>(P, w1 * w2, w1, (int)splits, R12, ldr, accumulate,
+                                          static_cast<T*>(R12op), ldop, w1, w2, st));
+    c->stats.n_other_launches++;
+  } else {
+    p.C = R12;
+    p.ldc = ldr;
+    p.accumulate = accumulate;
+    p.Cop = R12op;
+    p.ldop = ldop;
+    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, 1, st));
+  }
+  c->arena.release(mark);
+  c->stats.n_tn_launches++;
+  return RGSQR_OK;
+}
+
+template <typename T>
+static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2,
+                      int64_t lda, int64_t m, int64_t w1, int64_t w2, cudaStream_t st) {
+  const int s = (int)sizeof(T);
+  const int BK = gemm_block_k(s);
+  const int EPB = 128 / s;
+  const int bn = pick_bn(w2);
+  CUtensorMap ma, mb;
+  std::string err;
+  if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4) ||
+      !encode_tmap_2d(&mb, prec, R12op, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err))
+    return fail(c, RGSQR_ERR_INVALID_ARG, "outer: " + err);
+  GemmParams p{};
+  p.M = m;
+  p.N = w2;
+  p.K = w1;
+  p.kb_total = (w1 + BK - 1) / BK;
+  p.kb_per_split = p.kb_total;
+  p.A2 = A2;
+  p.lda2 = lda;
+  RGSQR_CUDA(c, launch_gemm<T>(true, bn, ma, mb, p, 1, st));
+  c->stats.n_nn_launches++;
+  return RGSQR_OK;
+}
+
+int op_inner(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m, int64_t w1,
+             int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate, cudaStream_t st) {
+  switch (prec) {
+    case RGSQR_FP16:
+      return op_inner_t<__half>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+    case RGSQR_BF16:
+      return op_inner_t<__nv_bfloat16>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+    case RGSQR_TF32:
+      return op_inner_t<float>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+  }
+  return fail(c, RGSQR_ERR_UNSUPPORTED, "inner: precision not supported");
+}
+
+int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2, int64_t lda,
+             int64_t m, int64_t w1, int64_t w2, cudaStream_t st) {
+  switch (prec) {
+    case RGSQR_FP16: return op_outer_t<__half>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
+    case RGSQR_BF16: return op_outer_t<__nv_bfloat16>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
+    case RGSQR_TF32: return op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
+  }
+  return fail(c, RGSQR_ERR_UNSUPPORTED, "outer: precision not supported");
+}
+
+static void leaf_geometry(Ctx* c, int64_t m, int* grid, int* rp) {
+  int G = c->opt.leaf_ctas > 0 ? (int)c->opt.leaf_ctas : c->num_sms;
+  G = (int)std::max<int64_t>(1, std::min<int64_t>(G, (m + 31) / 32));
+  int64_t r = (m + G - 1) / G;
+  r = (r + 3) & ~int64_t(3);
+  *grid = G;
+  *rp = (int)r;
+}
+
+int leaf_width_for(Ctx* c, int64_t m) {
+  int G, rp;
+  leaf_geometry(c, m, &G, &rp);
+  int64_t wmax = (int64_t)LEAF_SMEM_BUDGET / ((int64_t)rp * 4);
+  int64_t w = std::min<int64_t>({c->opt.leaf_width, (int64_t)LEAF_MAX_W, wmax});
+  if (w >= 8) w &= ~int64_t(7);
+  return (int)w;
+}
+
+int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float* R11, int64_t ldr,
+            int64_t col_offset, cudaStream_t st) {
+  int G, rp;
+  leaf_geometry(c, m, &G, &rp);
+  if (w < 1 || w > LEAF_MAX_W || (size_t)w * rp * 4 > LEAF_SMEM_BUDGET)
+    return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: panel " + std::to_string(m) + "x" + std::to_string(w) +
+                                              " does not fit on chip");
+  LeafParams p{};
+  p.P = P;
+  p.ldp = ldp;
+  p.m = m;
+  p.w = (int)w;
+  p.rows_per_cta = rp;
+  p.R = R11;
+  p.ldr = ldr;
+  p.partials = c->d_partials;
+  p.counter = c->d_counter;
+  p.breakdown = c->d_breakdown;
+  p.col_offset = col_offset;
+  cudaError_t e;
+  switch (prec) {
+    case RGSQR_FP16: e = launch_leaf<__half>(p, G, st); break;
+    case RGSQR_BF16: e = launch_leaf<__nv_bfloat16>(p, G, st); break;
+    case RGSQR_TF32: e = launch_leaf<float>(p, G, st); break;
+    default: return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: precision not supported");
+  }
+  if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("leaf launch: ") + cudaGetErrorString(e));
+  c->stats.n_leaf_launches++;
+  return RGSQR_OK;
+}
+
+// ---------------------------------------------------------------------------------
+// in-core recursion (Eq. 2) on a device-resident m x n matrix
+// ---------------------------------------------------------------------------------
+int64_t split_width(int64_t w, int64_t leaf) {
+  if (w <= leaf) return 0;
+  int64_t h = (w + 1) / 2;
+  int64_t align = w >= 256 ? 64 : 8;
+  int64_t w1 = (h + align - 1) / align * align;
+  if (w1 >= w) w1 = h;
+  return w1;
+}
+
+size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n) {
+  const int64_t leaf = leaf_width_for(c, m);
+  const int64_t w1 = split_width(n, leaf);
+  size_t b = 0;
+  if (w1 > 0) b += (size_t)w1 * (n - w1) * elem_bytes(prec) + 1024;  // R12 operand copy
+  // split-K partials: op_inner adapts its split factor to what is free; reserve a
+  // quarter of the node's matrix bytes, clamped to [1, 16] MiB
+  const size_t node_bytes = (size_t)m * n * elem_bytes(prec);
+  b += std::min<size_t>((size_t)16 << 20, std::max<size_t>((size_t)1 << 20, node_bytes / 4)) + 4096;
+  (void)c;
+  return b;
+}
+
+struct IncoreCtx {
+  Ctx* c;
+  int prec;
+  char* A;
+  int64_t lda, m, s;
+  float* R;
+  int64_t ldr;
+  int64_t leaf;
+  void* r12op;
+  int64_t col_offset;
+  cudaStream_t st;
+  IncoreHooks* hooks;
+};
+
+static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
+  const int64_t w1 = split_width(w, k.leaf);
+  if (w1 == 0) {
+    if (k.hooks && k.hooks->need) k.hooks->need(c0 + w);
+    int rc = op_leaf(k.c, k.prec, k.A + c0 * k.lda * k.s, k.lda, k.m, w, k.R + c0 + c0 * k.ldr, k.ldr,
+                     k.col_offset + c0, k.st);
+    if (rc == 0 && k.hooks && k.hooks->leaf_done) k.hooks->leaf_done(c0 + w);
+    return rc;
+  }
+  const int64_t w2 = w - w1, h = c0 + w1;
+  int rc = incore_rec(k, c0, w1);
+  if (rc < 0) return rc;
+  if (k.hooks && k.hooks->need) k.hooks->need(c0 + w);
+  const char* Q1 = k.A + c0 * k.lda * k.s;
+  char* A2 = k.A + h * k.lda * k.s;
+  rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, k.R + c0 + h * k.ldr, k.ldr, k.r12op, w1, 0,
+                k.st);
+  if (rc < 0) return rc;
+  rc = op_outer(k.c, k.prec, Q1, k.lda, k.r12op, w1, A2, k.lda, k.m, w1, w2, k.st);
+  if (rc < 0) return rc;
+  k.c->stats.n_incore_nodes++;
+  return incore_rec(k, h, w2);
+}
+
+int incore_factor(Ctx* c, int prec, void* A, int64_t lda, int64_t m, int64_t n, float* R, int64_t ldr,
+                  int64_t col_offset, cudaStream_t st, IncoreHooks* hooks) {
+  IncoreCtx k{c, prec, static_cast<char*>(A), lda, m, elem_bytes(prec), R, ldr, leaf_width_for(c, m), nullptr,
+              col_offset, st, hooks};
+  if (k.leaf < 1) return fail(c, RGSQR_ERR_UNSUPPORTED, "in-core: m too large for the on-chip leaf");
+  const int64_t w1 = split_width(n, k.leaf);
+  size_t mark = c->arena.mark();
+  if (w1 > 0) {
+    k.r12op = c->arena.alloc((size_t)w1 * (n - w1) * k.s);
+    if (!k.r12op) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core: no arena space for R12");
+  }
+  int rc = incore_rec(k, 0, n);
+  c->arena.release(mark);
+  return rc;
+}
+
+}  // namespace rgsqr

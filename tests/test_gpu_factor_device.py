@@ -1,0 +1,79 @@
+"""GPU parity of the device-resident recursive CGS (rgsqr_factor_device) against the oracle."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+import oracle  # noqa: E402
+import rgsqr_inputs as gi  # noqa: E402
+from tests.gpu_util import to_dev, from_dev  # noqa: E402
+
+TOL = {"fp16": 5e-3, "bf16": 5e-3, "tf32": 5e-3}
+STOR = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}
+
+
+@pytest.fixture(scope="module")
+def h():
+    from paper_conf_icpp_zhangw21_b200 import Handle
+    hd = Handle(0)
+    yield hd
+    hd.close()
+
+
+def run(h, A, storage, prec, m, n):
+    lda = (m + 7) // 8 * 8                       # lda * sizeof(elem) must be a multiple of 16 B
+    Ad = to_dev(A, storage)
+    if lda != m:
+        Ap = torch.zeros((n, lda), dtype=Ad.dtype, device="cuda")
+        Ap[:, :m] = Ad
+        Ad = Ap
+    R = torch.empty((n, n), dtype=torch.float32, device="cuda")
+    rc = h.factor_device(Ad, lda, m, n, Ad, R, precision=prec)
+    return rc, from_dev(Ad[:, :m]), R.cpu().numpy().T.astype(np.float64)
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+@pytest.mark.parametrize("m,n", [(4096, 256), (8192, 1000), (12345, 512)])
+def test_gaussian_vs_oracle(h, prec, m, n):
+    st = STOR[prec]
+    A = gi.gaussian(m, n, seed=1, dtype=st)
+    X = gi.to_float64(A, st)
+    rc, Q, R = run(h, A, st, prec, m, n)
+    assert rc == 0
+    ref = oracle.rgs(X, leaf=64)
+    assert oracle.is_upper_triangular(R)
+    be = oracle.backward_error(X, Q, R)
+    re = oracle.r_rel_error(R, ref.R)
+    emu = oracle.rgs_emulated(X, prec, leaf=64)
+    emu_re = oracle.r_rel_error(emu.R, ref.R)
+    assert be <= TOL[prec], be
+    assert re <= max(TOL[prec], 2 * emu_re), (re, emu_re)
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+@pytest.mark.parametrize("m,n", [(4096, 256), (65536, 512)])
+def test_exact_dyadic(h, prec, m, n):
+    """A = H[:, :n] R0: every intermediate is exact, so R == R0 and Q == H bitwise."""
+    st = STOR[prec]
+    A64, R0 = gi.dyadic_mixed(m, n, seed=3)
+    A = gi.to_storage(A64, st)
+    assert np.array_equal(gi.to_float64(A, st), A64)
+    rc, Q, R = run(h, A, st, prec, m, n)
+    np.testing.assert_array_equal(R, R0)
+    np.testing.assert_array_equal(Q, gi.hadamard(m, n))
+
+
+def test_diag_scaled(h):
+    A64, d = gi.diag_scaled(4096, 384, seed=1)
+    A = gi.to_storage(A64, "fp16")
+    rc, Q, R = run(h, A, "fp16", "fp16", 4096, 384)
+    np.testing.assert_array_equal(R, np.diag(d))
+
+
+def test_repeatable_bitwise(h):
+    A = gi.gaussian(8192, 512, seed=4, dtype="fp16")
+    _, Q1, R1 = run(h, A, "fp16", "fp16", 8192, 512)
+    _, Q2, R2 = run(h, A, "fp16", "fp16", 8192, 512)
+    np.testing.assert_array_equal(R1, R2)
+    np.testing.assert_array_equal(Q1, Q2)

@@ -1,0 +1,139 @@
+"""GPU parity of the host-resident (out-of-core) factorization rgsqr_factor against the
+oracle, across device budgets, reuse / serialize / blocked modes, plus the byte
+counters against the paper's data-movement model (oracle/model.py)."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+import oracle  # noqa: E402
+from oracle import model  # noqa: E402
+import rgsqr_inputs as gi  # noqa: E402
+
+MiB = 1 << 20
+STOR = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}
+
+
+@pytest.fixture()
+def h():
+    from paper_conf_icpp_zhangw21_b200 import Handle
+    hd = Handle(0)
+    yield hd
+    hd.close()
+
+
+def factor(h, A, prec, budget, **opts):
+    m, n = A.shape
+    for k, v in opts.items():
+        h.set_option(k, v)
+    Q = np.empty_like(A, order="F")
+    R = np.full((n, n), np.nan, dtype=np.float32, order="F")
+    rc = h.factor(A, m, m, n, Q, R, precision=prec, budget=budget)
+    return rc, Q, R, h.stats()
+
+
+@pytest.fixture(scope="module")
+def gauss():
+    A = gi.gaussian(16384, 1024, seed=7, dtype="fp16")
+    X = gi.to_float64(A, "fp16")
+    return A, X, oracle.rgs(X, leaf=64)
+
+
+@pytest.mark.parametrize("budget_mib,reuse", [(0, 1), (80, 1), (40, 1), (28, 1), (28, 0), (20, 0), (20, 1), (12, 1), (12, 0)])
+def test_ooc_gaussian_fp16(h, gauss, budget_mib, reuse):
+    A, X, ref = gauss
+    rc, Q, R, st = factor(h, A, "fp16", budget_mib * MiB, reuse=reuse)
+    assert rc == 0
+    Rg = R.astype(np.float64)
+    assert oracle.is_upper_triangular(Rg)
+    be = oracle.backward_error(X, gi.to_float64(Q, "fp16"), Rg)
+    re = oracle.r_rel_error(Rg, ref.R)
+    assert be < 5e-3 and re < 5e-3, (be, re, st)
+    if budget_mib:
+        assert st["arena_bytes"] <= budget_mib * MiB
+    if 0 < budget_mib < 44:            # the whole 32 MiB matrix + workspace needs ~44.5 MiB
+        assert st["n_ooc_nodes"] >= 1
+    assert st["h2d_matrix_bytes"] >= A.nbytes and st["d2h_matrix_bytes"] >= A.nbytes
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+@pytest.mark.parametrize("budget_mib,reuse,algo", [(12, 1, 0), (20, 0, 0), (40, 1, 1), (40, 0, 1)])
+def test_ooc_exact_dyadic(h, prec, budget_mib, reuse, algo):
+    """Exact-dyadic input: every intermediate is exact, so any tile plan / budget /
+    algorithm must return R == R0 and Q == H bitwise."""
+    m, n = 16384, 1024
+    A64, R0 = gi.dyadic_mixed(m, n, seed=5)
+    A = gi.to_storage(A64, STOR[prec])
+    budget = budget_mib * MiB * (2 if prec == "tf32" else 1)
+    rc, Q, R, st = factor(h, A, prec, budget, reuse=reuse, algo=algo, block_cols=256)
+    assert rc == 0
+    np.testing.assert_array_equal(R.astype(np.float64), R0)
+    np.testing.assert_array_equal(gi.to_float64(Q, STOR[prec]), gi.hadamard(m, n))
+
+
+def test_serialized_equals_overlapped_bitwise(h, gauss):
+    A = gauss[0]
+    _, Q1, R1, st1 = factor(h, A, "fp16", 28 * MiB, serialize=0)
+    _, Q2, R2, st2 = factor(h, A, "fp16", 28 * MiB, serialize=1)
+    np.testing.assert_array_equal(R1, R2)
+    np.testing.assert_array_equal(Q1, Q2)
+    assert st1["h2d_bytes"] == st2["h2d_bytes"]
+
+
+def test_in_place_q_aliases_a(h):
+    m, n = 8192, 512
+    A = gi.gaussian(m, n, seed=3, dtype="bf16")
+    X = gi.to_float64(A, "bf16")
+    R = np.zeros((n, n), dtype=np.float32, order="F")
+    rc = h.factor(A, m, m, n, A, R, precision="bf16", budget=12 * MiB)      # Q_out = A_host
+    assert rc == 0
+    assert oracle.backward_error(X, gi.to_float64(A, "bf16"), R.astype(np.float64)) < 5e-3
+
+
+def test_noreuse_bytes_match_recursive_model(h, gauss):
+    """Budget 20 MiB at 16384 x 1024 fp16: in-core nodes of 256 columns (8 MiB + workspace),
+    two OOC levels.  Without reuse the schedule moves exactly the model's words."""
+    A = gauss[0]
+    m, n = A.shape
+    _, _, _, st = factor(h, A, "fp16", 20 * MiB, reuse=0)
+    w = model.recursive_noreuse_split_words(m, n, 256)
+    assert st["h2d_matrix_bytes"] == 2 * w["h2d_matrix"]
+    assert st["d2h_matrix_bytes"] == 2 * w["d2h_matrix"]
+    assert st["d2h_r_bytes"] == 4 * w["d2h_r"]
+
+
+def test_noreuse_bytes_match_blocked_model(h, gauss):
+    A = gauss[0]
+    m, n = A.shape
+    _, _, _, st = factor(h, A, "fp16", 40 * MiB, reuse=0, algo=1, block_cols=256)
+    w = model.blocked_noreuse_split_words(m, n, 256)
+    assert st["h2d_matrix_bytes"] == 2 * w["h2d_matrix"]
+    assert st["d2h_matrix_bytes"] == 2 * w["d2h_matrix"]
+    assert st["d2h_r_bytes"] == 4 * w["d2h_r"]
+
+
+def test_reuse_moves_fewer_bytes_and_recursive_beats_blocked(h, gauss):
+    A = gauss[0]
+    _, _, _, s_reuse = factor(h, A, "fp16", 28 * MiB, reuse=1)
+    _, _, _, s_plain = factor(h, A, "fp16", 28 * MiB, reuse=0)
+    _, _, _, s_blk = factor(h, A, "fp16", 28 * MiB, reuse=0, algo=1, block_cols=128)
+    assert s_reuse["h2d_bytes"] < s_plain["h2d_bytes"]
+    assert s_plain["h2d_bytes"] < s_blk["h2d_bytes"]          # PAPER.md:155, Table 3
+
+
+def test_budget_too_small(h):
+    from paper_conf_icpp_zhangw21_b200 import RgsqrError
+    A = gi.gaussian(16384, 256, seed=1, dtype="fp16")
+    with pytest.raises(RgsqrError) as e:
+        factor(h, A, "fp16", 1 * MiB)
+    assert e.value.status == -2
+
+
+def test_zero_column_warning(h):
+    m, n = 8192, 256
+    A = gi.gaussian(m, n, seed=2, dtype="fp16")
+    A[:, 100] = 0
+    rc, Q, R, st = factor(h, A, "fp16", 4 * MiB)
+    assert rc == 1 and st["first_breakdown_col"] == 100
+    assert R[100, 100] == 0
