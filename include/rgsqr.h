@@ -74,7 +74,8 @@ enum rgsqr_option {
   RGSQR_OPT_SERIALIZE = 7,      /* 1 = one stream, no overlap (the paper's "Synchronous" rows) */
   RGSQR_OPT_REUSE = 8,          /* 1 = QR-level data reuse, default 1 */
   RGSQR_OPT_LEAF_CTAS = 9,      /* CTAs of the leaf kernel (0 = automatic) */
-  RGSQR_OPT_SPLITK = 10         /* force split-K factor of the TN product (0 = automatic) */
+  RGSQR_OPT_SPLITK = 10,        /* force split-K factor of the TN product (0 = automatic) */
+  RGSQR_OPT_PROFILE = 11        /* 1 = time every kernel with CUDA events (rgsqr_stats.kern_*) */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */
@@ -101,6 +102,16 @@ typedef struct rgsqr_stats {
   int64_t n_incore_nodes;
   int64_t first_breakdown_col;  /* -1 if none */
   int64_t flops;                /* 2 m n^2 (BASELINE.json metric convention) */
+  /* Per-kernel-class accounting, filled only when RGSQR_OPT_PROFILE = 1 (CUDA events
+   * around every launch).  Index: 0 leaf CGS, 1 inner product (TN + split-K reduce),
+   * 2 outer product (NN), 3 other.  flops / bytes are ALGORITHMIC:
+   *   leaf  (m x w):        2 m w^2 flop;          (2 m w) s + 4 w^2 bytes
+   *   inner (w1, m, w2):    2 m w1 w2 flop;        m (w1 + w2) s + 4 w1 w2 bytes
+   *   outer (m, w1, w2):    2 m w1 w2 flop;        m w1 s + w1 w2 s + 2 m w2 s bytes */
+  double  kern_ms[4];
+  int64_t kern_launches[4];
+  double  kern_flops[4];
+  double  kern_bytes[4];
 } rgsqr_stats;
 
 /* ---- lifetime -------------------------------------------------------------------- */

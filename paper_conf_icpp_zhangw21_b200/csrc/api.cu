@@ -68,6 +68,7 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   if (rc < 0) return rc;
   if (!R) return fail(c, RGSQR_ERR_INVALID_ARG, "null R");
   reset_stats(c);
+  c->begin_call();
   auto t0 = std::chrono::steady_clock::now();
   const size_t ws = incore_workspace_bytes(c, prec, m, n);
   const size_t cap = resolve_budget(c, budget);
@@ -91,6 +92,7 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   c->stats.arena_high_water = (int64_t)c->arena.high;
   c->stats.flops = (int64_t)(2.0 * m * (double)n * n);
   c->stats.first_breakdown_col = brk == 0x7f7f7f7f || brk == INT_MAX ? -1 : brk;
+  c->collect_kernel_stats();
   return c->stats.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;
 }
 
@@ -310,6 +312,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_REUSE: return &o.reuse;
     case RGSQR_OPT_LEAF_CTAS: return &o.leaf_ctas;
     case RGSQR_OPT_SPLITK: return &o.splitk;
+    case RGSQR_OPT_PROFILE: return &o.profile;
   }
   return nullptr;
 }

@@ -25,6 +25,13 @@ struct Options {
   int64_t reuse = 1;
   int64_t leaf_ctas = 0;
   int64_t splitk = 0;
+  int64_t profile = 0;
+};
+
+struct KernSeg {
+  int kind;                  // 0 leaf, 1 inner, 2 outer, 3 other
+  cudaEvent_t a, b;
+  double flops, bytes;
 };
 
 // Bump allocator over one cudaMalloc of at most the budget; LIFO release by mark.
@@ -65,15 +72,36 @@ struct Ctx {
   // small persistent device buffers (leaf barrier/partials, breakdown flag)
   float* d_partials = nullptr;
   unsigned int* d_counter = nullptr;
+  unsigned int leaf_epoch = 0;
   int* d_breakdown = nullptr;
   void* nccl_comm = nullptr;
   std::vector<TimedSeg> segs;
+  std::vector<KernSeg> ksegs;
   std::vector<cudaEvent_t> event_pool;
   size_t event_next = 0;
   bool timing = false;
 
   cudaStream_t compute() const { return st_user ? st_user : st_own; }
   cudaEvent_t ev();
+  // per-launch profiling (RGSQR_OPT_PROFILE)
+  cudaEvent_t kbegin(cudaStream_t st) {
+    if (!opt.profile) return nullptr;
+    cudaEvent_t e = ev();
+    cudaEventRecord(e, st);
+    return e;
+  }
+  void kend(int kind, cudaStream_t st, cudaEvent_t a, double flops, double bytes) {
+    if (!a) return;
+    cudaEvent_t b = ev();
+    cudaEventRecord(b, st);
+    ksegs.push_back({kind, a, b, flops, bytes});
+  }
+  void begin_call() {           // reset per-call accounting
+    segs.clear();
+    ksegs.clear();
+    event_next = 0;
+  }
+  void collect_kernel_stats();  // after a synchronize
 };
 
 // status helpers
@@ -88,7 +116,7 @@ int fail(Ctx* c, int status, const std::string& msg);
 int elem_bytes(int precision);
 bool encode_tmap_2d(CUtensorMap* map, int precision, const void* base, uint64_t inner, uint64_t outer,
                     uint64_t outer_stride_bytes, uint32_t box_inner, uint32_t box_outer, std::string* err,
-                    bool atom32 = false);
+                    int swz = 0);  // 0 SWIZZLE_128B, 1 SWIZZLE_128B_ATOM_32B, 2 none
 
 // ---- ops (device pointers, on stream st) ----
 int op_inner(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,

@@ -121,13 +121,34 @@ __global__ void __launch_bounds__(128, 1)
   __syncwarp();
 
   // ---------------- epilogue: all four warps ----------------
-  if (nkb > 0) ptx::mbar_wait(tfull, 0);
-  ptx::tc_fence_after();
+  // Thread (warp w, lane l) owns output row i = m0 + 32w + l; per 32-column chunk it
+  // reads its TMEM lane, and (NN / accumulating TN) the old values of its row, which
+  // are loaded one chunk ahead with predicated, branch-free loads so that the 32 loads
+  // of a chunk are in flight together (the first chunk before the accumulator is ready).
   const int lane = threadIdx.x & 31;
   const int64_t i = m0 + warp * 32 + lane;
   const bool row_ok = i < p.M;
+  const bool needs_old = kNN || (p.P == nullptr && p.accumulate);
+  float old[32], nxt[32];
+  auto load_chunk = [&](int cc, float (&dst)[32]) {
+    const int64_t nb = n0 + cc * 32;
+#pragma unroll
+    for (int j = 0; j < 32; ++j) {
+      const int64_t n = nb + j;
+      const bool ok = row_ok && n < p.N;
+      if constexpr (kNN)
+        dst[j] = ok ? Elem<T>::load(__ldcs(reinterpret_cast<const T*>(p.A2) + i + n * p.lda2)) : 0.0f;
+      else
+        dst[j] = ok ? __ldcs(p.C + i + n * p.ldc) : 0.0f;
+    }
+  };
+  if (needs_old) load_chunk(0, old);
+  if (nkb > 0) ptx::mbar_wait(tfull, 0);
+  ptx::tc_fence_after();
 #pragma unroll 1
   for (int cc = 0; cc < BN / 32; ++cc) {
+    if (n0 + cc * 32 >= p.N) break;  // warp-uniform
+    if (needs_old && cc + 1 < BN / 32) load_chunk(cc + 1, nxt);
     uint32_t v[32];
     if (nkb > 0) {
       ptx::tmem_ld_32x32b_x32(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(cc * 32), v);
@@ -136,26 +157,27 @@ __global__ void __launch_bounds__(128, 1)
 #pragma unroll
       for (int j = 0; j < 32; ++j) v[j] = 0u;
     }
-    if (!row_ok) continue;
     const int64_t nb = n0 + cc * 32;
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
       const int64_t n = nb + j;
-      if (n >= p.N) break;
+      const bool ok = row_ok && n < p.N;
       const float x = __uint_as_float(v[j]);
       if constexpr (kNN) {
-        T* a = reinterpret_cast<T*>(p.A2) + i + n * p.lda2;
-        *a = Elem<T>::store(Elem<T>::load(*a) - x);
+        if (ok) reinterpret_cast<T*>(p.A2)[i + n * p.lda2] = Elem<T>::store(old[j] - x);
       } else {
         if (p.P != nullptr) {
-          p.P[blockIdx.z * p.split_stride + i + n * p.ldp] = x;
+          if (ok) p.P[blockIdx.z * p.split_stride + i + n * p.ldp] = x;
         } else {
-          float* c = p.C + i + n * p.ldc;
-          const float y = p.accumulate ? *c + x : x;
-          *c = y;
-          if (p.Cop != nullptr) reinterpret_cast<T*>(p.Cop)[i + n * p.ldop] = Elem<T>::store(y);
+          const float y = p.accumulate ? old[j] + x : x;
+          if (ok) p.C[i + n * p.ldc] = y;
+          if (ok && p.Cop != nullptr) reinterpret_cast<T*>(p.Cop)[i + n * p.ldop] = Elem<T>::store(y);
         }
       }
+    }
+    if (needs_old) {
+#pragma unroll
+      for (int j = 0; j < 32; ++j) old[j] = nxt[j];
     }
   }
   ptx::tc_fence_before();
@@ -182,6 +204,219 @@ __global__ void splitk_reduce_kernel(const float* __restrict__ P, int64_t split_
   C[i + n * ldc] = acc;
   if (Cop != nullptr) Cop[i + n * ldop] = Elem<T>::store(acc);
 }
+
+// ---------------------------------------------------------------------------------
+// Persistent outer-product kernel  A2 <- A2 - Q1 R12.
+//
+// One CTA per SM loops over 128 x BN output tiles (tile = tm * tiles_n + tn, so
+// consecutive tiles of a CTA share Q1 rows in L2).  Warp roles (256 threads):
+//   warp 0      TMA producer of the Q1 / R12 k-blocks (STAGES-deep ring)
+//   warp 1      MMA issuer (tcgen05.mma, fp32 accumulator in TMEM, TWO accumulator
+//               buffers so the epilogue of tile j overlaps the MMAs of tile j+1)
+//   warp 2      TMEM allocator + TMA loader of the OLD A2 tile into a shared-memory C tile
+//   warps 4..7  epilogue: TMEM -> registers, C = C - acc in shared memory, rounded RN to
+//               the storage type, TMA store of the tile (one write of A2' per element)
+// ---------------------------------------------------------------------------------
+template <typename T, int BN>
+struct NNCfg {
+  static constexpr int BM = 128;
+  static constexpr int EPB = 128 / (int)sizeof(T);
+  static constexpr int BK = EPB;
+  static constexpr int UK = 32 / (int)sizeof(T);
+  static constexpr int A_BYTES = BM * 128;
+  static constexpr int B_BYTES = BN * 128;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int CBOX_N = 64;                                 // columns per C TMA box
+  static constexpr int C_BYTES = BM * BN * (int)sizeof(T);
+  static constexpr int STAGES_RAW = (220 * 1024 - C_BYTES - 2048) / STAGE_BYTES;
+  static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + C_BYTES + 1024 + 512;
+  static constexpr uint32_t TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
+  static constexpr uint32_t IDESC = ptx::idesc_f32acc(Elem<T>::kUmmaFormat, 1u, 0u, BM, BN);
+  static_assert(STAGES >= 2, "NN tile does not fit shared memory");
+  static_assert(2 * BN <= 512, "two accumulators must fit TMEM");
+};
+
+template <typename T, int BN>
+__global__ void __launch_bounds__(256, 1)
+    nn_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+              const __grid_constant__ CUtensorMap mapC, const NNParams p) {
+  using C = NNCfg<T, BN>;
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = ptx::smem_u32(smem_raw);
+  uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
+  T* Cs = reinterpret_cast<T*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES + C::C_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;   // [2]
+  uint64_t* tempty = tfull + 2;          // [2]
+  uint64_t* cfull = tempty + 2;
+  uint64_t* cempty = cfull + 1;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(cempty + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int num_tiles = p.tiles_m * p.tiles_n;
+  const int nkb = (int)p.kb_total;
+
+  if (warp == 0 && ptx::elect_one()) {
+    ptx::tma_prefetch_desc(&mapA);
+    ptx::tma_prefetch_desc(&mapB);
+    ptx::tma_prefetch_desc(&mapC);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      ptx::mbar_init(&tfull[b], 1);
+      ptx::mbar_init(&tempty[b], 4);
+    }
+    ptx::mbar_init(cfull, 1);
+    ptx::mbar_init(cempty, 1);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 2) ptx::tmem_alloc<C::TMEM_COLS>(tslot);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0) {
+    if (ptx::elect_one()) {
+      int it = 0;
+      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+        const int32_t m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * BN;
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const int s = it % C::STAGES;
+          ptx::mbar_wait(&empty[s], ((uint32_t)(it / C::STAGES) & 1u) ^ 1u);
+          uint8_t* sA = smem + s * C::STAGE_BYTES;
+          const int32_t k0 = kb * C::BK;
+          ptx::mbar_arrive_expect_tx(&full[s], C::STAGE_BYTES);
+#pragma unroll
+          for (int mb = 0; mb < C::BM / C::EPB; ++mb)
+            ptx::tma_load_2d(sA + mb * C::BK * 128, &mapA, &full[s], m0 + mb * C::EPB, k0);
+          ptx::tma_load_2d(sA + C::A_BYTES, &mapB, &full[s], k0, n0);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (ptx::elect_one()) {
+      int it = 0, lt = 0;
+      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++lt) {
+        const int b = lt & 1;
+        ptx::mbar_wait(&tempty[b], ((uint32_t)(lt >> 1) & 1u) ^ 1u);
+        ptx::tc_fence_after();
+        const uint32_t acc = tmem + (uint32_t)(b * BN);
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const int s = it % C::STAGES;
+          ptx::mbar_wait(&full[s], (uint32_t)(it / C::STAGES) & 1u);
+          ptx::tc_fence_after();
+          const uint32_t aBase = ptx::smem_u32(smem + s * C::STAGE_BYTES);
+          const uint32_t bBase = aBase + C::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < C::BK / C::UK; ++kk) {
+            uint64_t ad;
+            if constexpr (Elem<T>::kTF32)
+              ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 512, 1);
+            else
+              ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 1024);
+            const uint64_t bd = ptx::sdesc_sw128(bBase + kk * C::UK * (int)sizeof(T), 16, 1024);
+            ptx::umma<Elem<T>::kTF32>(acc, ad, bd, C::IDESC, (kb | kk) != 0 ? 1u : 0u);
+          }
+          ptx::umma_commit(&empty[s]);
+        }
+        ptx::umma_commit(&tfull[b]);
+      }
+    }
+  } else if (warp == 2) {
+    if (ptx::elect_one()) {
+      int lt = 0;
+      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++lt) {
+        const int32_t m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * BN;
+        ptx::mbar_wait(cempty, ((uint32_t)lt & 1u) ^ 1u);
+        ptx::mbar_arrive_expect_tx(cfull, C::C_BYTES);
+#pragma unroll
+        for (int cb = 0; cb < BN / C::CBOX_N; ++cb)
+          ptx::tma_load_2d(Cs + cb * C::CBOX_N * C::BM, &mapC, cfull, m0, n0 + cb * C::CBOX_N);
+      }
+    }
+  } else if (warp >= 4) {
+    const int ew = warp - 4;                 // == warp % 4: TMEM lanes [32 ew, 32 ew + 32)
+    const int r = ew * 32 + lane;            // row within the tile
+    int lt = 0;
+    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++lt) {
+      const int32_t m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * BN;
+      const int b = lt & 1;
+      ptx::mbar_wait(&tfull[b], (uint32_t)(lt >> 1) & 1u);
+      ptx::tc_fence_after();
+      ptx::mbar_wait(cfull, (uint32_t)lt & 1u);
+#pragma unroll 1
+      for (int cc = 0; cc < BN / 32; ++cc) {
+        uint32_t v[32];
+        ptx::tmem_ld_32x32b_x32(tmem + (uint32_t)(b * BN) + ((uint32_t)(ew * 32) << 16) + (uint32_t)(cc * 32), v);
+        ptx::tmem_ld_wait();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          T* cp = Cs + (cc * 32 + j) * C::BM + r;
+          *cp = Elem<T>::store(Elem<T>::load(*cp) - __uint_as_float(v[j]));
+        }
+      }
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&tempty[b]);
+      ptx::fence_proxy_async();              // generic smem writes -> visible to the TMA store
+      ptx::named_bar_sync(1, 128);
+      if (ew == 0 && lane == 0) {
+#pragma unroll
+        for (int cb = 0; cb < BN / C::CBOX_N; ++cb)
+          ptx::tma_store_2d(&mapC, Cs + cb * C::CBOX_N * C::BM, m0, n0 + cb * C::CBOX_N);
+        ptx::bulk_commit();
+        ptx::bulk_wait_read0();
+        ptx::mbar_arrive(cempty);
+      }
+    }
+    if (ew == 0 && lane == 0) ptx::bulk_wait0();
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<C::TMEM_COLS>(tmem);
+  }
+}
+
+template <typename T, int BN>
+static cudaError_t launch_nn_t(const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& mc,
+                               const NNParams& p, int grid, cudaStream_t st) {
+  using C = NNCfg<T, BN>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(nn_kernel<T, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  nn_kernel<T, BN><<<grid, 256, C::SMEM, st>>>(ma, mb, mc, p);
+  return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t launch_nn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& mc,
+                      const NNParams& p, int grid, cudaStream_t st) {
+  if constexpr (sizeof(T) == 4) {
+    if (bn >= 128) return launch_nn_t<T, 128>(ma, mb, mc, p, grid, st);
+    return launch_nn_t<T, 64>(ma, mb, mc, p, grid, st);
+  } else {
+    if (bn == 256) return launch_nn_t<T, 256>(ma, mb, mc, p, grid, st);
+    if (bn == 128) return launch_nn_t<T, 128>(ma, mb, mc, p, grid, st);
+    return launch_nn_t<T, 64>(ma, mb, mc, p, grid, st);
+  }
+}
+
+template cudaError_t launch_nn<__half>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&,
+                                       const NNParams&, int, cudaStream_t);
+template cudaError_t launch_nn<__nv_bfloat16>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&,
+                                              const NNParams&, int, cudaStream_t);
+template cudaError_t launch_nn<float>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&,
+                                      const NNParams&, int, cudaStream_t);
 
 // ---------------------------------------------------------------------------------
 // host-side launch helpers

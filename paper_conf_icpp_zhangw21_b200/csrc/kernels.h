@@ -7,7 +7,12 @@
 namespace rgsqr {
 
 constexpr int LEAF_MAX_W = 64;
+constexpr int LEAF_MAX_G = 160;       // leaf grid size cap (>= SM count)
+constexpr int LEAF_PARTS = 4;         // row quarters of the per-CTA partial sums
 constexpr size_t LEAF_SMEM_BUDGET = 200 * 1024;
+// smem column stride of the leaf panel slice: >= rows and == 4 (mod 32), so that the
+// float4 reads of 8 threads at the same row in 8 different columns hit 32 distinct banks
+__host__ __device__ inline int leaf_ld(int rows) { return ((rows + 31) / 32) * 32 + 4; }
 
 struct GemmParams {
   int64_t M, N, K;          // D[M x N] = sum_k A[M x K] B[N x K]^T (see gemm.cu)
@@ -27,6 +32,15 @@ struct GemmParams {
   int64_t lda2;
 };
 
+struct NNParams {
+  int tiles_m, tiles_n;     // 128-row x BN-column output tiles
+  int64_t kb_total;         // K blocks (K = w1)
+};
+
+template <typename T>
+cudaError_t launch_nn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& mc,
+                      const NNParams& p, int grid, cudaStream_t st);
+
 struct LeafParams {
   void* P;                  // panel m x w (ldp), overwritten by Q
   int64_t ldp;
@@ -35,8 +49,10 @@ struct LeafParams {
   int rows_per_cta;
   float* R;                 // w x w block of R (ldr)
   int64_t ldr;
-  float* partials;          // [2][LEAF_MAX_W+2][grid]
+  float* partials;          // [2][LEAF_MAX_W+2][grid] per-CTA partial sums
   unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
+  long long* dbg;           // optional [w][8] clock64 stamps of CTA 0
+  int vec_ok;               // P and ldp*sizeof(elem) 16-byte aligned: vector panel loads
   int* breakdown;           // device int, atomicMin of the first breakdown column
   int64_t col_offset;       // global index of the panel's first column
 };

@@ -15,155 +15,341 @@
 // i.e. the projection coefficient of the column just normalised is folded into the
 // norm's reduction (q_t^T a = (u_t^T a) / r_tt), so each column costs ONE grid-wide
 // reduction instead of two -- the same CGS quantities up to rounding order
-// (reading R19).  A round = per-warp partial dot products over the CTA's
-// rows, one partial vector per CTA to global memory, a grid barrier (release/acquire
-// counter), then every CTA sums the G partials in the same fixed order (deterministic,
-// no float atomics).
-#include <cooperative_groups.h>
-
+// (reading R19).
+//
+// Exchange per round: each CTA writes its partial vector (fp32) to global memory,
+// arrives on a counter (release) and spins on it (acquire); then every CTA loads the
+// G partials of each value (all loads of a warp issued together) and sums them in the
+// same fixed order (deterministic, no float atomics).  Measured alternatives
+// (scripts/barrier_bench.cu, RGSQR_LEAF_DEBUG stamps): per-word round tags avoid the
+// counter but flood L2 with spinning loads (4x slower gather).
 #include "dtype.cuh"
 #include "kernels.h"
 
 namespace rgsqr {
 
-static constexpr int LEAF_THREADS = 256;
+static constexpr int LEAF_THREADS = 512;
 static constexpr int LEAF_WARPS = LEAF_THREADS / 32;
+static constexpr int GEMV_PARTS = LEAF_THREADS / 32;   // row parts of the local GEMV
 
-__device__ __forceinline__ void grid_barrier(unsigned int* counter, unsigned int target) {
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    atomicAdd(counter, 1u);
-    unsigned int v;
-    do {
-      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(counter) : "memory");
-    } while (v < target);
-    __threadfence();
+// per-phase cycle stamps of CTA 0 (diagnostics; p.dbg == nullptr in production)
+#define DBG_STAMP(i)                                           \
+  if (p.dbg != nullptr && blockIdx.x == 0 && threadIdx.x == 0) \
+    p.dbg[(size_t)t * 8 + (i)] = clock64();
+
+// 16-byte vector load of consecutive storage elements widened to fp32.
+template <typename T>
+struct Vec;
+template <>
+struct Vec<__half> {
+  static constexpr int N = 8;
+  __device__ static void load(const __half* p, float* o) {
+    const uint4 u = *reinterpret_cast<const uint4*>(p);
+    const __half2* h = reinterpret_cast<const __half2*>(&u);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 f = __half22float2(h[i]);
+      o[2 * i] = f.x;
+      o[2 * i + 1] = f.y;
+    }
   }
-  __syncthreads();
+};
+template <>
+struct Vec<__nv_bfloat16> {
+  static constexpr int N = 8;
+  __device__ static void load(const __nv_bfloat16* p, float* o) {
+    const uint4 u = *reinterpret_cast<const uint4*>(p);
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 f = __bfloat1622float2(h[i]);
+      o[2 * i] = f.x;
+      o[2 * i + 1] = f.y;
+    }
+  }
+};
+template <>
+struct Vec<float> {
+  static constexpr int N = 4;
+  __device__ static void load(const float* p, float* o) {
+    const float4 u = *reinterpret_cast<const float4*>(p);
+    o[0] = u.x;
+    o[1] = u.y;
+    o[2] = u.z;
+    o[3] = u.w;
+  }
+};
+
+// column pair (x, y) whose dot product is value k of round t
+__device__ __forceinline__ void round_operands(int t, int w, int k, int& cx, int& cy) {
+  if (t == 0) {
+    if (k < w) { cx = k; cy = k; }                     // ||a_k||^2
+    else { cx = 0; cy = 1; }                           // a_0^T a_1
+  } else {
+    if (k == 0) { cx = t; cy = t; }                    // u_t^T u_t
+    else if (k == 1) { cx = t; cy = t + 1; }           // u_t^T a_{t+1}
+    else { cx = k - 2; cy = t + 1; }                   // q_i^T a_{t+1}
+  }
 }
 
 template <typename T>
 __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p) {
-  extern __shared__ float sp[];                     // [w][RP] column-major panel slice
+  extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
   __shared__ float tot[LEAF_MAX_W + 2];            // reduced round vector
   __shared__ float anorm2[LEAF_MAX_W];             // ||a_k||^2 (breakdown threshold)
-  __shared__ float coef[LEAF_MAX_W];               // r_{i,t+1}, i <= t
-  __shared__ float sc[2];                          // 1/r_tt, r_tt
+  __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];
 
   const int G = gridDim.x;
   const int g = blockIdx.x;
   const int w = p.w;
-  const int RP = p.rows_per_cta;
+  const int RP = p.rows_per_cta;                   // rows owned by this CTA (max), multiple of 8
+  const int LD = leaf_ld(RP);                      // smem column stride, == 4 (mod 32)
   const int64_t r0 = (int64_t)g * RP;
   const int64_t rem = p.m - r0;
   const int rows = rem <= 0 ? 0 : (rem < RP ? (int)rem : RP);
+  const int rows4 = (rows + 3) & ~3;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   T* P = reinterpret_cast<T*>(p.P);
 
-  // load the slice (coalesced along rows), exact widening to fp32
-  for (int j = 0; j < w; ++j)
-    for (int i = threadIdx.x; i < RP; i += LEAF_THREADS)
-      sp[j * RP + i] = i < rows ? Elem<T>::load(P[r0 + i + (int64_t)j * p.ldp]) : 0.0f;
+  // ---- load the slice: 16-byte vector loads (rows are 16-byte aligned), fp32 in smem ----
+  {
+    constexpr int V = Vec<T>::N;
+    const int nvec = p.vec_ok ? rows / V : 0;
+    for (int idx = threadIdx.x; idx < w * nvec; idx += LEAF_THREADS) {
+      const int j = idx / nvec, i = (idx - j * nvec) * V;
+      float f[V];
+      Vec<T>::load(P + r0 + i + (int64_t)j * p.ldp, f);
+#pragma unroll
+      for (int e = 0; e < V; e += 4)
+        *reinterpret_cast<float4*>(sp + j * LD + i + e) = make_float4(f[e], f[e + 1], f[e + 2], f[e + 3]);
+    }
+    const int span = LD - nvec * V;
+    for (int idx = threadIdx.x; idx < w * span; idx += LEAF_THREADS) {
+      const int j = idx / span, i = nvec * V + (idx - j * span);
+      sp[j * LD + i] = i < rows ? Elem<T>::load(P[r0 + i + (int64_t)j * p.ldp]) : 0.0f;
+    }
+  }
   __syncthreads();
 
   const float u_work = 5.9604645e-08f;             // 2^-24, fp32 accumulation
-  int bad_first = -1;
+  // Bulk GEMV mapping: thread (kq = lane, part = warp) handles values kq and kq + 32
+  // over row part `warp`.  8 consecutive kq read 8 different columns at the same row:
+  // with LD == 4 (mod 32) the float4 reads are conflict-free; a shared y is broadcast.
+  const int kq = lane;
+  const int nv4 = rows4 / 4;
+  const int per = (nv4 + GEMV_PARTS - 1) / GEMV_PARTS;
+  const int v_lo = min(nv4, warp * per), v_hi = min(nv4, v_lo + per);
+  // critical-dot mapping: warp = row part, lanes stride the part's rows
+  const int c_lo = v_lo * 4, c_hi = min(rows, v_hi * 4);
+
+  // dot(x-col, y-col) over this thread's float4 rows
+  auto dot4 = [&](int cx, int cy) {
+    const float4* x = reinterpret_cast<const float4*>(sp + cx * LD);
+    const float4* y = reinterpret_cast<const float4*>(sp + cy * LD);
+    float s0 = 0.f, s1 = 0.f;
+    for (int i = v_lo; i < v_hi; ++i) {
+      const float4 a = x[i], b = y[i];
+      s0 = fmaf(a.x, b.x, s0);
+      s1 = fmaf(a.y, b.y, s1);
+      s0 = fmaf(a.z, b.z, s0);
+      s1 = fmaf(a.w, b.w, s1);
+    }
+    return s0 + s1;
+  };
+  // warp-cooperative dots over the warp's row part (lanes stride rows, xor-trees):
+  // u^T u, u^T a, q^T a in one pass (u = column cu, a = column ca, q = column cq)
+  auto wdot3 = [&](int cu, int ca, int cq, bool three, float& suu, float& sua, float& sqa) {
+    const float* u = sp + cu * LD;
+    const float* a = sp + ca * LD;
+    const float* q = sp + cq * LD;
+    float s0 = 0.f, s1 = 0.f, s2 = 0.f;
+    for (int i = c_lo + lane; i < c_hi; i += 32) {
+      const float uv = u[i];
+      s0 = fmaf(uv, uv, s0);
+      if (three) {
+        const float av = a[i];
+        s1 = fmaf(uv, av, s1);
+        s2 = fmaf(q[i], av, s2);
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      s0 += __shfl_xor_sync(0xffffffffu, s0, o);
+      s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+      s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+    }
+    suu = s0;
+    sua = s1;
+    sqa = s2;
+  };
+  // publish the L values of part[][] as this CTA's partial vector of round t, arrive
+  auto publish_arrive = [&](int t, int L) {
+    __syncthreads();
+    float* buf = p.partials + (size_t)(t & 1) * (LEAF_MAX_W + 2) * G;
+    if (threadIdx.x < L) {
+      const int k = threadIdx.x;
+      float s = part[0][k];
+#pragma unroll
+      for (int q = 1; q < GEMV_PARTS; ++q) s += part[q][k];
+      buf[(size_t)k * G + g] = s;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0)  // release: orders this CTA's partial stores (bar.sync cumulativity)
+      asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.counter) : "memory");
+  };
+
+  // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ] ----
+  {
+    const int t = 0;
+    const int L = w + (w > 1 ? 1 : 0);
+    DBG_STAMP(0);
+    for (int k = kq; k < L; k += 32) {
+      int cx, cy;
+      round_operands(0, w, k, cx, cy);
+      part[warp][k] = dot4(cx, cy);
+    }
+    publish_arrive(0, L);
+  }
 
   for (int t = 0; t < w; ++t) {
-    // ---- 1. local partial sums of this round's vector ----
-    int L;
-    if (t == 0) L = w + (w > 1 ? 1 : 0);
-    else L = (t + 1 < w) ? t + 2 : 1;
-    for (int k = warp; k < L; k += LEAF_WARPS) {
-      const float* x;
-      const float* y;
-      if (t == 0) {
-        if (k < w) { x = sp + k * RP; y = x; }
-        else { x = sp; y = sp + RP; }                           // a_0^T a_1
-      } else {
-        if (k == 0) { x = sp + t * RP; y = x; }                 // u_t^T u_t
-        else if (k == 1) { x = sp + t * RP; y = sp + (t + 1) * RP; }  // u_t^T a_{t+1}
-        else { x = sp + (k - 2) * RP; y = sp + (t + 1) * RP; }  // q_i^T a_{t+1}
+    const int L = (t == 0) ? w + (w > 1 ? 1 : 0) : ((t + 1 < w) ? t + 2 : 1);
+    DBG_STAMP(1);
+    // ---- lookahead (overlaps the barrier): round t+1's q_i^T a_{t+2}, i <= t-1.
+    //      q_i (i <= t-1) are final and a_{t+2} is untouched until round t+1. ----
+    if (t + 2 < w && t >= 1) {
+      const int cnt = t;                               // i in [0, t-1]
+      const int ya = t + 2;
+      const bool ha = kq < cnt, hb = kq + 32 < cnt;
+      if (ha) {
+        const float4* y = reinterpret_cast<const float4*>(sp + ya * LD);
+        const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
+        const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
+        float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+        for (int i = v_lo; i < v_hi; ++i) {
+          const float4 yy = y[i], a = xa[i];
+          a0 = fmaf(a.x, yy.x, a0);
+          a1 = fmaf(a.y, yy.y, a1);
+          a0 = fmaf(a.z, yy.z, a0);
+          a1 = fmaf(a.w, yy.w, a1);
+          if (hb) {
+            const float4 b = xb[i];
+            b0 = fmaf(b.x, yy.x, b0);
+            b1 = fmaf(b.y, yy.y, b1);
+            b0 = fmaf(b.z, yy.z, b0);
+            b1 = fmaf(b.w, yy.w, b1);
+          }
+        }
+        part[warp][2 + kq] = a0 + a1;
+        if (hb) part[warp][2 + kq + 32] = b0 + b1;
       }
-      float s = 0.0f;
-      for (int i = lane; i < rows; i += 32) s = fmaf(x[i], y[i], s);
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-      if (lane == 0) p.partials[((int64_t)(t & 1) * (LEAF_MAX_W + 2) + k) * G + g] = s;
     }
-    // ---- 2. grid-wide exchange ----
-    grid_barrier(p.counter, (unsigned)((t + 1) * G));
-    // ---- 3. fixed-order reduction of the G partials (identical in every CTA) ----
-    for (int k = warp; k < L; k += LEAF_WARPS) {
-      const float* src = p.partials + ((int64_t)(t & 1) * (LEAF_MAX_W + 2) + k) * G;
-      float s = 0.0f;
-      for (int c = lane; c < G; c += 32) s += __ldcg(src + c);
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-      if (lane == 0) tot[k] = s;
-    }
-    __syncthreads();
-    // ---- 4. scalars (thread 0), R entries (CTA 0) ----
+    // ---- grid barrier of round t (arrived in publish_arrive) ----
     if (threadIdx.x == 0) {
-      float uu, ua;
-      if (t == 0) {
-        for (int k = 0; k < w; ++k) anorm2[k] = tot[k];
-        uu = tot[0];
-        ua = (w > 1) ? tot[w] : 0.0f;
-      } else {
-        uu = tot[0];
-        ua = (t + 1 < w) ? tot[1] : 0.0f;
-      }
-      float rtt = sqrtf(uu);
-      const float tau = (float)p.m * u_work * sqrtf(anorm2[t]);
-      const bool bad = !(rtt > tau) || !isfinite(rtt);
-      float inv = 0.0f;
-      if (bad) { rtt = 0.0f; if (bad_first < 0) bad_first = t; }
-      else inv = 1.0f / rtt;
-      sc[0] = inv;
-      sc[1] = rtt;
-      if (t + 1 < w) {
-        for (int i = 0; i < t; ++i) coef[i] = (t == 0) ? 0.0f : tot[2 + i];
-        coef[t] = ua * inv;
-      }
-      if (g == 0) {
-        p.R[t + (int64_t)t * p.ldr] = rtt;
-        if (t + 1 < w)
-          for (int i = 0; i <= t; ++i) p.R[i + (int64_t)(t + 1) * p.ldr] = coef[i];
+      const unsigned target = (unsigned)(t + 1) * (unsigned)G;
+      unsigned cv;
+      do {
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cv) : "l"(p.counter) : "memory");
+      } while (cv < target);
+    }
+    __syncthreads();
+    DBG_STAMP(2);
+    // ---- gather round t's G partials per value, fixed-order sum ----
+    {
+      constexpr int KPW = (LEAF_MAX_W + 2 + LEAF_WARPS - 1) / LEAF_WARPS;
+      constexpr int QMAX = (LEAF_MAX_G + 31) / 32;
+      const float* buf = p.partials + (size_t)(t & 1) * (LEAF_MAX_W + 2) * G;
+      float v[KPW][QMAX];
+#pragma unroll
+      for (int a = 0; a < KPW; ++a)
+#pragma unroll
+        for (int q = 0; q < QMAX; ++q) {
+          const int k = warp + a * LEAF_WARPS, c = lane + 32 * q;
+          v[a][q] = (k < L && c < G) ? __ldcg(buf + (size_t)k * G + c) : 0.0f;
+        }
+#pragma unroll
+      for (int a = 0; a < KPW; ++a) {
+        const int k = warp + a * LEAF_WARPS;
+        if (k >= L) break;                               // warp-uniform
+        float s = v[a][0];
+#pragma unroll
+        for (int q = 1; q < QMAX; ++q) s += v[a][q];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+        if (lane == 0) {
+          tot[k] = s;
+          if (t == 0 && k < w) anorm2[k] = s;
+        }
       }
     }
     __syncthreads();
-    // ---- 5. q_t = u_t / r_tt (store rounded), u_{t+1} = a_{t+1} - Q_{<=t} r_{:,t+1} ----
-    const float inv = sc[0];
-    float* ut = sp + t * RP;
+    DBG_STAMP(3);
+    // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{:,t+1} ----
+    const float uu = tot[0];
+    const float ua = (t == 0) ? ((w > 1) ? tot[w] : 0.0f) : ((t + 1 < w) ? tot[1] : 0.0f);
+    float rtt = sqrtf(uu);
+    const float tau = (float)p.m * u_work * sqrtf(anorm2[t]);
+    const bool bad = !(rtt > tau) || !isfinite(rtt);
+    const float inv = bad ? 0.0f : 1.0f / rtt;
+    if (bad) rtt = 0.0f;
+    const float ct = ua * inv;                        // r_{t,t+1}
+    const bool more = t + 1 < w;
+    if (g == 0) {
+      if (threadIdx.x == 0) {
+        p.R[t + (int64_t)t * p.ldr] = rtt;
+        if (bad) atomicMin(p.breakdown, (int)(p.col_offset + t));
+      }
+      if (more && threadIdx.x <= t)
+        p.R[threadIdx.x + (int64_t)(t + 1) * p.ldr] = threadIdx.x == t ? ct : tot[2 + threadIdx.x];
+      if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
+    }
+    // ---- q_t = u_t / r_tt (stored rounded), u_{t+1} = a_{t+1} - sum_{i<=t} q_i r_{i,t+1}
+    //      (sequential sum per row; rows are independent chains) ----
+    float* ut = sp + t * LD;
+    float* an = sp + (t + 1) * LD;
     for (int i = threadIdx.x; i < rows; i += LEAF_THREADS) {
       const float q = ut[i] * inv;
       ut[i] = q;
-      P[r0 + i + (int64_t)t * p.ldp] = Elem<T>::store(q);
-    }
-    __syncthreads();
-    if (t + 1 < w) {
-      float* a = sp + (t + 1) * RP;
-      for (int i = threadIdx.x; i < rows; i += LEAF_THREADS) {
-        float u = a[i];
-        for (int k = 0; k <= t; ++k) u = fmaf(-sp[k * RP + i], coef[k], u);
-        a[i] = u;
+      if (more) {
+        float u = an[i];
+        int k = 0;
+        for (; k + 8 <= t; k += 8) {
+          float qq[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) qq[e] = sp[(k + e) * LD + i];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) u = fmaf(-qq[e], tot[2 + k + e], u);
+        }
+        for (; k < t; ++k) u = fmaf(-sp[k * LD + i], tot[2 + k], u);
+        an[i] = fmaf(-q, ct, u);
       }
     }
     __syncthreads();
-  }
-  if (g == 0 && threadIdx.x == 0) {
-    // zero the strict lower triangle of R11 and report breakdown
-    for (int j = 0; j < w; ++j)
-      for (int i = j + 1; i < w; ++i) p.R[i + (int64_t)j * p.ldr] = 0.0f;
-    if (bad_first >= 0) atomicMin(p.breakdown, (int)(p.col_offset + bad_first));
+    DBG_STAMP(4);
+    // ---- round t+1: the three dots that needed round t, then publish + arrive ----
+    if (more) {
+      const int t1 = t + 1;
+      const int L1 = (t1 + 1 < w) ? t1 + 2 : 1;
+      if (p.dbg != nullptr && blockIdx.x == 0 && threadIdx.x == 0) p.dbg[(size_t)t1 * 8] = clock64();
+      float s_uu, s_ua, s_qa;                            // u^T u, u^T a_{t+2}, q_t^T a_{t+2}
+      const bool three = t1 + 1 < w;
+      wdot3(t1, three ? t1 + 1 : t1, t, three, s_uu, s_ua, s_qa);
+      if (lane == 0) {
+        part[warp][0] = s_uu;
+        if (t1 + 1 < w) {
+          part[warp][1] = s_ua;
+          part[warp][2 + t] = s_qa;
+        }
+      }
+      publish_arrive(t1, L1);
+    }
+    // q_t to global after the arrival, so the release does not wait for these stores
+    for (int i = threadIdx.x; i < rows; i += LEAF_THREADS) P[r0 + i + (int64_t)t * p.ldp] = Elem<T>::store(ut[i]);
   }
 }
 
 template <typename T>
 cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
-  const size_t smem = (size_t)p.w * p.rows_per_cta * sizeof(float);
+  const size_t smem = (size_t)p.w * leaf_ld(p.rows_per_cta) * sizeof(float);
   static size_t attr_smem = 0;
   if (smem > attr_smem) {
     cudaError_t e = cudaFuncSetAttribute(leaf_cgs_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -400,8 +400,7 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   if (!R && c->rank == 0) return fail(c, RGSQR_ERR_INVALID_ARG, "null R_out");
   if (c->nranks > 1) return fail(c, RGSQR_ERR_UNSUPPORTED, "row-sharded multi-GPU factorization not built yet");
   reset_stats(c);
-  c->segs.clear();
-  c->event_next = 0;
+  c->begin_call();
   const int s = elem_bytes(prec);
 
   // ---- page-lock caller buffers (timed separately) ----
@@ -485,6 +484,7 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   st.arena_high_water = (int64_t)c->arena.high;
   st.flops = (int64_t)(2.0 * m * (double)n * n);
   st.first_breakdown_col = (brk == 0x7f7f7f7f || brk == INT_MAX) ? -1 : brk;
+  c->collect_kernel_stats();
   return st.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;
 }
 

@@ -18,6 +18,18 @@ int fail(Ctx* c, int status, const std::string& msg) {
   return status;
 }
 
+void Ctx::collect_kernel_stats() {
+  for (auto& k : ksegs) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, k.a, k.b);
+    stats.kern_ms[k.kind] += ms;
+    stats.kern_launches[k.kind] += 1;
+    stats.kern_flops[k.kind] += k.flops;
+    stats.kern_bytes[k.kind] += k.bytes;
+  }
+  ksegs.clear();
+}
+
 cudaEvent_t Ctx::ev() {
   if (event_next == event_pool.size()) {
     cudaEvent_t e;
@@ -46,7 +58,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 
 bool encode_tmap_2d(CUtensorMap* map, int precision, const void* base, uint64_t inner, uint64_t outer,
                     uint64_t outer_stride_bytes, uint32_t box_inner, uint32_t box_outer, std::string* err,
-                    bool atom32) {
+                    int swz) {
   auto enc = get_encode();
   if (!enc) {
     *err = "cuTensorMapEncodeTiled unavailable";
@@ -60,7 +72,10 @@ bool encode_tmap_2d(CUtensorMap* map, int precision, const void* base, uint64_t 
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = enc(map, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   atom32 ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   swz == 1   ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B
+                   : swz == 2 ? CU_TENSOR_MAP_SWIZZLE_NONE
+                              : CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     *err = "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ") dims=" + std::to_string(inner) + "x" +
@@ -101,6 +116,7 @@ static int op_inner_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
     splits = 1;
   }
   size_t mark = c->arena.mark();
+  cudaEvent_t kb = c->kbegin(st);
   if (splits > 1) {
     float* P = static_cast<float*>(c->arena.alloc((size_t)splits * w1 * w2 * sizeof(float)));
     if (!P) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner: no arena space for split-K partials");
@@ -119,6 +135,7 @@ static int op_inner_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
     p.ldop = ldop;
     RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, 1, st));
   }
+  c->kend(1, st, kb, 2.0 * m * w1 * w2, (double)m * (w1 + w2) * s + 4.0 * w1 * w2);
   c->arena.release(mark);
   c->stats.n_tn_launches++;
   return RGSQR_OK;
@@ -130,21 +147,22 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
   const int EPB = 128 / s;
-  const int bn = pick_bn(w2);
-  CUtensorMap ma, mb;
+  int bn = pick_bn(w2);
+  if (s == 4) bn = std::min(bn, 128);  // fp32 C tile must leave room for the k-ring
+  CUtensorMap ma, mb, mc;
   std::string err;
-  if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4) ||
-      !encode_tmap_2d(&mb, prec, R12op, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err))
+  if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
+      !encode_tmap_2d(&mb, prec, R12op, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err) ||
+      !encode_tmap_2d(&mc, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, 128, 64, &err, 2))
     return fail(c, RGSQR_ERR_INVALID_ARG, "outer: " + err);
-  GemmParams p{};
-  p.M = m;
-  p.N = w2;
-  p.K = w1;
+  NNParams p{};
+  p.tiles_m = (int)((m + 127) / 128);
+  p.tiles_n = (int)((w2 + bn - 1) / bn);
   p.kb_total = (w1 + BK - 1) / BK;
-  p.kb_per_split = p.kb_total;
-  p.A2 = A2;
-  p.lda2 = lda;
-  RGSQR_CUDA(c, launch_gemm<T>(true, bn, ma, mb, p, 1, st));
+  const int grid = (int)std::min<int64_t>((int64_t)p.tiles_m * p.tiles_n, c->num_sms);
+  cudaEvent_t kb = c->kbegin(st);
+  RGSQR_CUDA(c, launch_nn<T>(bn, ma, mb, mc, p, grid, st));
+  c->kend(2, st, kb, 2.0 * m * w1 * w2, (double)m * w1 * s + (double)w1 * w2 * s + 2.0 * m * w2 * s);
   c->stats.n_nn_launches++;
   return RGSQR_OK;
 }
@@ -174,9 +192,9 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
 
 static void leaf_geometry(Ctx* c, int64_t m, int* grid, int* rp) {
   int G = c->opt.leaf_ctas > 0 ? (int)c->opt.leaf_ctas : c->num_sms;
-  G = (int)std::max<int64_t>(1, std::min<int64_t>(G, (m + 31) / 32));
+  G = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)G, (int64_t)LEAF_MAX_G, (m + 31) / 32}));
   int64_t r = (m + G - 1) / G;
-  r = (r + 3) & ~int64_t(3);
+  r = (r + 7) & ~int64_t(7);  // 16-byte aligned row slices for the vector loads
   *grid = G;
   *rp = (int)r;
 }
@@ -184,7 +202,7 @@ static void leaf_geometry(Ctx* c, int64_t m, int* grid, int* rp) {
 int leaf_width_for(Ctx* c, int64_t m) {
   int G, rp;
   leaf_geometry(c, m, &G, &rp);
-  int64_t wmax = (int64_t)LEAF_SMEM_BUDGET / ((int64_t)rp * 4);
+  int64_t wmax = (int64_t)LEAF_SMEM_BUDGET / ((int64_t)leaf_ld(rp) * 4);
   int64_t w = std::min<int64_t>({c->opt.leaf_width, (int64_t)LEAF_MAX_W, wmax});
   if (w >= 8) w &= ~int64_t(7);
   return (int)w;
@@ -194,7 +212,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
             int64_t col_offset, cudaStream_t st) {
   int G, rp;
   leaf_geometry(c, m, &G, &rp);
-  if (w < 1 || w > LEAF_MAX_W || (size_t)w * rp * 4 > LEAF_SMEM_BUDGET)
+  if (w < 1 || w > LEAF_MAX_W || (size_t)w * leaf_ld(rp) * 4 > LEAF_SMEM_BUDGET)
     return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: panel " + std::to_string(m) + "x" + std::to_string(w) +
                                               " does not fit on chip");
   LeafParams p{};
@@ -206,10 +224,16 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   p.R = R11;
   p.ldr = ldr;
   p.partials = c->d_partials;
+  static const bool dbg = getenv("RGSQR_LEAF_DEBUG") != nullptr;
+  static long long* dbg_buf = nullptr;
   p.counter = c->d_counter;
+  p.vec_ok = ((ldp * elem_bytes(prec)) % 16 == 0) && (reinterpret_cast<uintptr_t>(P) % 16 == 0);
+  if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 8 * LEAF_MAX_W);
+  p.dbg = dbg ? dbg_buf : nullptr;
   p.breakdown = c->d_breakdown;
   p.col_offset = col_offset;
   cudaError_t e;
+  cudaEvent_t kb = c->kbegin(st);
   switch (prec) {
     case RGSQR_FP16: e = launch_leaf<__half>(p, G, st); break;
     case RGSQR_BF16: e = launch_leaf<__nv_bfloat16>(p, G, st); break;
@@ -217,6 +241,18 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
     default: return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: precision not supported");
   }
   if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("leaf launch: ") + cudaGetErrorString(e));
+  const int s = elem_bytes(prec);
+  c->kend(0, st, kb, 2.0 * m * w * w, 2.0 * m * w * s + 4.0 * w * w);
+  if (p.dbg) {
+    long long hb[8 * LEAF_MAX_W];
+    cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 8 * w, cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+    double ph[4] = {0, 0, 0, 0};
+    for (int t = 0; t < w; ++t)
+      for (int i = 0; i < 4; ++i) ph[i] += (double)(hb[t * 8 + i + 1] - hb[t * 8 + i]);
+    fprintf(stderr, "[leaf m=%lld w=%lld G=%d RP=%d] cycles/round: gemv %.0f barrier %.0f gather %.0f update %.0f\n",
+            (long long)m, (long long)w, G, rp, ph[0] / w, ph[1] / w, ph[2] / w, ph[3] / w);
+  }
   c->stats.n_leaf_launches++;
   return RGSQR_OK;
 }

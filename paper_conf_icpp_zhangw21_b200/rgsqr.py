@@ -22,7 +22,7 @@ STORAGE = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32", "tf32x3": "fp32"}
 
 OK, WARN_RANK_DEFICIENT = 0, 1
 OPTIONS = {"leaf_width": 1, "tile_rows_min": 2, "tile_rows_max": 3, "ring_depth": 4, "algo": 5,
-           "block_cols": 6, "serialize": 7, "reuse": 8, "leaf_ctas": 9, "splitk": 10}
+           "block_cols": 6, "serialize": 7, "reuse": 8, "leaf_ctas": 9, "splitk": 10, "profile": 11}
 
 EXPORTS = ["rgsqr_create", "rgsqr_get_unique_id", "rgsqr_create_dist", "rgsqr_destroy", "rgsqr_factor",
            "rgsqr_factor_device", "rgsqr_op_leaf", "rgsqr_op_inner", "rgsqr_op_outer", "rgsqr_set_stream",
@@ -38,10 +38,19 @@ class Stats(C.Structure):
                 ("arena_bytes", C.c_int64), ("arena_high_water", C.c_int64),
                 ("n_leaf_launches", C.c_int64), ("n_tn_launches", C.c_int64), ("n_nn_launches", C.c_int64),
                 ("n_other_launches", C.c_int64), ("n_ooc_nodes", C.c_int64), ("n_incore_nodes", C.c_int64),
-                ("first_breakdown_col", C.c_int64), ("flops", C.c_int64)]
+                ("first_breakdown_col", C.c_int64), ("flops", C.c_int64),
+                ("kern_ms", C.c_double * 4), ("kern_launches", C.c_int64 * 4),
+                ("kern_flops", C.c_double * 4), ("kern_bytes", C.c_double * 4)]
 
     def as_dict(self):
-        return {k: getattr(self, k) for k, _ in self._fields_}
+        out = {}
+        for k, _ in self._fields_:
+            v = getattr(self, k)
+            out[k] = list(v) if k.startswith("kern_") else v
+        return out
+
+
+KERNEL_CLASSES = ("leaf", "inner", "outer", "other")
 
 
 class RgsqrError(RuntimeError):

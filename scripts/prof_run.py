@@ -1,0 +1,40 @@
+"""One device-resident factorization of a bench workload, for ncu launch lists / captures.
+
+    python scripts/prof_run.py [--m 65536] [--n 8192] [--prec fp16] [--reps 1]
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import rgsqr_inputs as gi  # noqa: E402
+from paper_conf_icpp_zhangw21_b200 import Handle, build  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--m", type=int, default=65536)
+ap.add_argument("--n", type=int, default=8192)
+ap.add_argument("--prec", default="fp16")
+ap.add_argument("--reps", type=int, default=1)
+ap.add_argument("--host", action="store_true", help="use the host (out-of-core) path, 1 GiB budget")
+a = ap.parse_args()
+build.build()
+st = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}[a.prec]
+A = gi.gaussian(a.m, a.n, seed=2, dtype=st)
+h = Handle(0)
+if a.host:
+    Q = np.empty_like(A, order="F")
+    R = np.empty((a.n, a.n), dtype=np.float32, order="F")
+    for _ in range(a.reps):
+        h.factor(A, a.m, a.m, a.n, Q, R, precision=a.prec, budget=1 << 30)
+else:
+    Ad = torch.from_numpy(np.ascontiguousarray(A.T)).cuda()
+    Qd = torch.empty_like(Ad)
+    Rd = torch.empty((a.n, a.n), dtype=torch.float32, device="cuda")
+    for _ in range(a.reps):
+        h.factor_device(Ad, a.m, a.m, a.n, Qd, Rd, precision=a.prec, budget=1 << 30)
+torch.cuda.synchronize()
+print("stats", h.stats())
