@@ -144,7 +144,7 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaStreamCreateWithFlags(&c->st_h2d, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
-      cudaMalloc(&c->d_counter, 256) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess) {
+      cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess) {
     delete c;
     return RGSQR_ERR_CUDA;
   }

@@ -53,6 +53,9 @@ struct LeafParams {
   unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
   long long* dbg;           // optional [w][8] clock64 stamps of CTA 0
   int vec_ok;               // P and ldp*sizeof(elem) 16-byte aligned: vector panel loads
+  int xmode;                // 0: counter barrier + gather; 2: fixed-point red.add exchange
+  unsigned int epoch;       // launch counter
+  unsigned long long* xw;   // [2][LEAF_MAX_W+2] exchange words (zeroed by the launcher)
   int* breakdown;           // device int, atomicMin of the first breakdown column
   int64_t col_offset;       // global index of the panel's first column
 };

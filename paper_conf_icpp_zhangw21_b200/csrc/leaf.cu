@@ -32,6 +32,15 @@ static constexpr int LEAF_THREADS = 512;
 static constexpr int LEAF_WARPS = LEAF_THREADS / 32;
 static constexpr int GEMV_PARTS = LEAF_THREADS / 32;   // row parts of the local GEMV
 
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
 // per-phase cycle stamps of CTA 0 (diagnostics; p.dbg == nullptr in production)
 #define DBG_STAMP(i)                                           \
   if (p.dbg != nullptr && blockIdx.x == 0 && threadIdx.x == 0) \
@@ -98,6 +107,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   __shared__ float tot[LEAF_MAX_W + 2];            // reduced round vector
   __shared__ float anorm2[LEAF_MAX_W];             // ||a_k||^2 (breakdown threshold)
   __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];
+  __shared__ unsigned long long xprev[2][LEAF_MAX_W + 2];  // last seen exchange words
+  for (int i = threadIdx.x; i < 2 * (LEAF_MAX_W + 2); i += blockDim.x) (&xprev[0][0])[i] = 0ull;
 
   const int G = gridDim.x;
   const int g = blockIdx.x;
@@ -182,20 +193,50 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     sua = s1;
     sqa = s2;
   };
+  // round tags of the tagged exchange: unique per (launch, round)
+  // Fixed-point exchange (rounds t >= 1, xmode 2): value k of round t is scaled by 2^e
+  // with e chosen from a bound on |partial| (column norms of round 0), rounded to an
+  // integer |v| <= 2^46 and added with ONE red.add.u64 per CTA to word W[t&1][k] as
+  //     (1 << 56) + (v + 2^46)          -- top byte counts arrivals, low 56 bits sum
+  // Integer addition is associative, so the total is independent of arrival order
+  // (deterministic) and exact in fixed point; the word is never reset within a launch:
+  // readers take the difference with the value they saw two rounds earlier.
+  auto fx_exp = [&](int t, int k) -> int {
+    float b2;                                          // bound^2 on |partial|
+    if (k == 0) b2 = anorm2[t];
+    else if (k == 1) b2 = anorm2[t] * anorm2[t + 1];
+    else b2 = anorm2[t + 1];
+    const float bound = 4.0f * sqrtf(b2) + 1e-30f;
+    int ex;
+    frexpf(bound, &ex);                                // bound < 2^ex
+    return 46 - ex;
+  };
   // publish the L values of part[][] as this CTA's partial vector of round t, arrive
   auto publish_arrive = [&](int t, int L) {
     __syncthreads();
+    const bool fx = p.xmode == 2 && t > 0;
     float* buf = p.partials + (size_t)(t & 1) * (LEAF_MAX_W + 2) * G;
     if (threadIdx.x < L) {
       const int k = threadIdx.x;
       float s = part[0][k];
 #pragma unroll
       for (int q = 1; q < GEMV_PARTS; ++q) s += part[q][k];
-      buf[(size_t)k * G + g] = s;
+      if (fx) {
+        long long v = __double2ll_rn(ldexp((double)s, fx_exp(t, k)));
+        v = v > (1ll << 46) ? (1ll << 46) : (v < -(1ll << 46) ? -(1ll << 46) : v);
+        const unsigned long long add = (1ull << 56) + (unsigned long long)(v + (1ll << 46));
+        asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + (t & 1) * (LEAF_MAX_W + 2) + k),
+                     "l"(add)
+                     : "memory");
+      } else {
+        buf[(size_t)k * G + g] = s;
+      }
     }
-    __syncthreads();
-    if (threadIdx.x == 0)  // release: orders this CTA's partial stores (bar.sync cumulativity)
-      asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.counter) : "memory");
+    if (!fx) {
+      __syncthreads();
+      if (threadIdx.x == 0)  // release: orders this CTA's partial stores (bar.sync cumulativity)
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.counter) : "memory");
+    }
   };
 
   // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ] ----
@@ -243,18 +284,34 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         if (hb) part[warp][2 + kq + 32] = b0 + b1;
       }
     }
+    const bool fx = p.xmode == 2 && t > 0;
     // ---- grid barrier of round t (arrived in publish_arrive) ----
-    if (threadIdx.x == 0) {
-      const unsigned target = (unsigned)(t + 1) * (unsigned)G;
+    if (!fx && threadIdx.x == 0) {
       unsigned cv;
+      const unsigned target = (p.xmode == 2 ? 1u : (unsigned)(t + 1)) * (unsigned)G;
       do {
         asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cv) : "l"(p.counter) : "memory");
       } while (cv < target);
     }
     __syncthreads();
     DBG_STAMP(2);
-    // ---- gather round t's G partials per value, fixed-order sum ----
-    {
+    if (fx) {
+      // ---- fixed-point exchange: poll the L words until all G CTAs have added ----
+      if (threadIdx.x < L) {
+        const int k = threadIdx.x;
+        unsigned long long* wp = p.xw + (t & 1) * (LEAF_MAX_W + 2) + k;
+        const unsigned long long prev = xprev[t & 1][k];
+        unsigned long long now = ld_relaxed_u64(wp), d = now - prev;
+        while ((unsigned)(d >> 56) != (unsigned)G) {
+          now = ld_relaxed_u64(wp);
+          d = now - prev;
+        }
+        xprev[t & 1][k] = now;
+        const long long total = (long long)(d & ((1ull << 56) - 1)) - (long long)G * (1ll << 46);
+        tot[k] = (float)ldexp((double)total, -fx_exp(t, k));
+      }
+    } else {
+      // ---- gather round t's G partials per value, fixed-order sum ----
       constexpr int KPW = (LEAF_MAX_W + 2 + LEAF_WARPS - 1) / LEAF_WARPS;
       constexpr int QMAX = (LEAF_MAX_G + 31) / 32;
       const float* buf = p.partials + (size_t)(t & 1) * (LEAF_MAX_W + 2) * G;
@@ -358,6 +415,8 @@ cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
     attr_smem = smem;
   }
   cudaError_t e = cudaMemsetAsync(p.counter, 0, sizeof(unsigned int), st);
+  if (e != cudaSuccess) return e;
+  e = cudaMemsetAsync(p.xw, 0, sizeof(unsigned long long) * 2 * (LEAF_MAX_W + 2), st);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);

@@ -227,6 +227,10 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   static const bool dbg = getenv("RGSQR_LEAF_DEBUG") != nullptr;
   static long long* dbg_buf = nullptr;
   p.counter = c->d_counter;
+  static const int xmode = getenv("RGSQR_LEAF_XMODE") ? atoi(getenv("RGSQR_LEAF_XMODE")) : 2;
+  p.xmode = xmode;
+  p.epoch = ++c->leaf_epoch;
+  p.xw = reinterpret_cast<unsigned long long*>(c->d_counter + 64);  // 256-byte offset in the 4 KiB block
   p.vec_ok = ((ldp * elem_bytes(prec)) % 16 == 0) && (reinterpret_cast<uintptr_t>(P) % 16 == 0);
   if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 8 * LEAF_MAX_W);
   p.dbg = dbg ? dbg_buf : nullptr;
