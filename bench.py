@@ -349,7 +349,7 @@ def main():
     # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cols = 1024 if m >= 65536 else n
+        cols = 2048 if m >= 65536 else n          # ~10-20 s of fp64 CGS on the host cores
         v, dt = cpu_oracle_sample(A, st_name, cols)
         cpu = {"value": v, "unit": "TFLOPS", "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
                "sample": f"oracle O3 (fp64 recursive CGS, numpy/OpenBLAS) on {m}x{cols} (first {cols} columns "

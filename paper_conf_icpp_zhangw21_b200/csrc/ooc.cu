@@ -240,22 +240,32 @@ struct Exec {
     }
     if (to_D && q1_out_done) cudaStreamWaitEvent(sc, q1_out_done, 0);
     auto tl = tiles(t);
-    int64_t r0 = 0;
-    for (size_t i = 0; i < tl.size(); ++i) {
-      const int64_t tr = tl[i];
+    std::vector<int64_t> row0(tl.size());
+    for (size_t i = 0, r = 0; i < tl.size(); r += tl[i], ++i) row0[i] = (int64_t)r;
+    // Reuse: walk the tiles in REVERSE order, so the last K tiles of the
+    // inner pass -- still in their ring slots, unmodified -- are consumed first without
+    // being uploaded again.  Tile i always lives in slot i % K.
+    const size_t n = tl.size();
+    for (size_t j = 0; j < n; ++j) {
+      const size_t i = reuse ? n - 1 - j : j;
+      const int64_t tr = tl[i], r0 = row0[i];
       const int k = (int)(i % K);
       char* slot = ring + (size_t)k * t * slot_cols * s;
       char* sq = slot;
       char* sa = slot + (D ? 0 : (size_t)t * w1 * s);
-      cudaStreamWaitEvent(sh, ev_free[k], 0);
-      if (!D) {
-        int rc = h2d(sq, t, Q, r0, tr, c0, w1);
+      const bool resident = reuse && j < (size_t)K && i + K >= n;   // left in the slot by stream_inner
+      if (!resident) {
+        cudaStreamWaitEvent(sh, ev_free[k], 0);
+        if (!D) {
+          int rc = h2d(sq, t, Q, r0, tr, c0, w1);
+          if (rc < 0) return rc;
+        }
+        int rc = h2d(sa, t, hsrc(a2_src_q), r0, tr, h, w2);
         if (rc < 0) return rc;
+        cudaEventRecord(loaded[k], sh);
+        cudaStreamWaitEvent(sc, loaded[k], 0);
       }
-      int rc = h2d(sa, t, hsrc(a2_src_q), r0, tr, h, w2);
-      if (rc < 0) return rc;
-      cudaEventRecord(loaded[k], sh);
-      cudaStreamWaitEvent(sc, loaded[k], 0);
+      int rc;
       cudaEvent_t a = seg_begin(sc);
       rc = op_outer(c, prec, D ? D + r0 * s : sq, D ? m : t, R12op, w1, sa, t, tr, w1, w2, sc);
       if (rc < 0) return rc;
@@ -272,7 +282,6 @@ struct Exec {
         if (rc < 0) return rc;
         cudaEventRecord(ev_free[k], sd);
       }
-      r0 += tr;
     }
     return RGSQR_OK;
   }
