@@ -51,7 +51,8 @@ struct LeafParams {
   int64_t ldr;
   float* partials;          // [2][LEAF_MAX_W+2][grid] per-CTA partial sums
   unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
-  long long* dbg;           // optional [w][8] clock64 stamps of CTA 0
+  long long* dbg;           // optional [w][8] clock64 stamps of CTA dbg_cta
+  int dbg_cta;
   int vec_ok;               // P and ldp*sizeof(elem) 16-byte aligned: vector panel loads
   int xmode;                // 0: counter barrier + gather; 2: fixed-point red.add exchange
   unsigned int epoch;       // launch counter

@@ -41,9 +41,13 @@ __device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long
   return v;
 }
 
-// per-phase cycle stamps of CTA 0 (diagnostics; p.dbg == nullptr in production)
+// exact power of two as a double (|e| < 1000)
+__device__ __forceinline__ double pow2d(int e) { return __hiloint2double((1023 + e) << 20, 0); }
+
+// per-phase cycle stamps of CTA p.dbg_cta (diagnostics; p.dbg == nullptr in production)
+#define DBG_CTA p.dbg_cta
 #define DBG_STAMP(i)                                           \
-  if (p.dbg != nullptr && blockIdx.x == 0 && threadIdx.x == 0) \
+  if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) \
     p.dbg[(size_t)t * 8 + (i)] = clock64();
 
 // 16-byte vector load of consecutive storage elements widened to fp32.
@@ -89,6 +93,30 @@ struct Vec<float> {
   }
 };
 
+// store 4 consecutive rounded elements (8- or 16-byte aligned destination)
+template <typename T>
+__device__ __forceinline__ void store4(T* dst, float4 v);
+template <>
+__device__ __forceinline__ void store4<__half>(__half* dst, float4 v) {
+  __half2 a = __floats2half2_rn(v.x, v.y), b = __floats2half2_rn(v.z, v.w);
+  uint2 u;
+  u.x = *reinterpret_cast<unsigned*>(&a);
+  u.y = *reinterpret_cast<unsigned*>(&b);
+  *reinterpret_cast<uint2*>(dst) = u;
+}
+template <>
+__device__ __forceinline__ void store4<__nv_bfloat16>(__nv_bfloat16* dst, float4 v) {
+  __nv_bfloat162 a = __floats2bfloat162_rn(v.x, v.y), b = __floats2bfloat162_rn(v.z, v.w);
+  uint2 u;
+  u.x = *reinterpret_cast<unsigned*>(&a);
+  u.y = *reinterpret_cast<unsigned*>(&b);
+  *reinterpret_cast<uint2*>(dst) = u;
+}
+template <>
+__device__ __forceinline__ void store4<float>(float* dst, float4 v) {
+  *reinterpret_cast<float4*>(dst) = v;
+}
+
 // column pair (x, y) whose dot product is value k of round t
 __device__ __forceinline__ void round_operands(int t, int w, int k, int& cx, int& cy) {
   if (t == 0) {
@@ -108,6 +136,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   __shared__ float anorm2[LEAF_MAX_W];             // ||a_k||^2 (breakdown threshold)
   __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];
   __shared__ unsigned long long xprev[2][LEAF_MAX_W + 2];  // last seen exchange words
+  __shared__ __align__(16) float coef[LEAF_MAX_W + 4];      // r_{i,t+1}, i < t (aligned copy)
+  __shared__ int exS[LEAF_MAX_W];                           // 2||a_j|| < 2^exS[j]
+  __shared__ float tauc[LEAF_MAX_W];                        // breakdown thresholds
   for (int i = threadIdx.x; i < 2 * (LEAF_MAX_W + 2); i += blockDim.x) (&xprev[0][0])[i] = 0ull;
 
   const int G = gridDim.x;
@@ -202,27 +233,30 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   // (deterministic) and exact in fixed point; the word is never reset within a launch:
   // readers take the difference with the value they saw two rounds earlier.
   auto fx_exp = [&](int t, int k) -> int {
-    float b2;                                          // bound^2 on |partial|
-    if (k == 0) b2 = anorm2[t];
-    else if (k == 1) b2 = anorm2[t] * anorm2[t + 1];
-    else b2 = anorm2[t + 1];
-    const float bound = 4.0f * sqrtf(b2) + 1e-30f;
-    int ex;
-    frexpf(bound, &ex);                                // bound < 2^ex
-    return 46 - ex;
+    // |partial| <= bound with bound = 4 ||a_t||^2, 4 ||a_t|| ||a_{t+1}|| or 4 ||a_{t+1}||
+    // (u_t shrinks a_t, ||q_i|| <= 1); exS[j] = exponent with 2 ||a_j|| < 2^exS[j]
+    if (k == 0) return 46 - 2 * exS[t];
+    if (k == 1) return 46 - (exS[t] + exS[t + 1]);
+    return 46 - (exS[t + 1] + 1);
   };
   // publish the L values of part[][] as this CTA's partial vector of round t, arrive
   auto publish_arrive = [&](int t, int L) {
     __syncthreads();
     const bool fx = p.xmode == 2 && t > 0;
     float* buf = p.partials + (size_t)(t & 1) * (LEAF_MAX_W + 2) * G;
-    if (threadIdx.x < L) {
-      const int k = threadIdx.x;
-      float s = part[0][k];
+    // sum of the GEMV_PARTS row-part partials of value k: 4 threads per value, each
+    // adds a quarter of the parts, then a 2-level xor tree (fixed order)
+    const int k = threadIdx.x >> 2, jq = threadIdx.x & 3;
+    float s = 0.f;
+    if (k < L) {
 #pragma unroll
-      for (int q = 1; q < GEMV_PARTS; ++q) s += part[q][k];
+      for (int q = 0; q < GEMV_PARTS / 4; ++q) s += part[jq * (GEMV_PARTS / 4) + q][k];
+    }
+    s += __shfl_xor_sync(0xffffffffu, s, 1);
+    s += __shfl_xor_sync(0xffffffffu, s, 2);
+    if (k < L && jq == 0) {
       if (fx) {
-        long long v = __double2ll_rn(ldexp((double)s, fx_exp(t, k)));
+        long long v = __double2ll_rn((double)s * pow2d(fx_exp(t, k)));
         v = v > (1ll << 46) ? (1ll << 46) : (v < -(1ll << 46) ? -(1ll << 46) : v);
         const unsigned long long add = (1ull << 56) + (unsigned long long)(v + (1ll << 46));
         asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + (t & 1) * (LEAF_MAX_W + 2) + k),
@@ -296,7 +330,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     __syncthreads();
     DBG_STAMP(2);
     if (fx) {
-      // ---- fixed-point exchange: poll the L words until all G CTAs have added ----
+      // ---- fixed-point exchange: each value's word is polled by its thread until all G
+      //      CTAs have added (measured: a single-sentinel poll + extra barrier is slower) ----
       if (threadIdx.x < L) {
         const int k = threadIdx.x;
         unsigned long long* wp = p.xw + (t & 1) * (LEAF_MAX_W + 2) + k;
@@ -308,7 +343,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
         xprev[t & 1][k] = now;
         const long long total = (long long)(d & ((1ull << 56) - 1)) - (long long)G * (1ll << 46);
-        tot[k] = (float)ldexp((double)total, -fx_exp(t, k));
+        const float val = (float)((double)total * pow2d(-fx_exp(t, k)));
+        tot[k] = val;
+        if (k >= 2) coef[k - 2] = val;
       }
     } else {
       // ---- gather round t's G partials per value, fixed-order sum ----
@@ -334,7 +371,14 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
         if (lane == 0) {
           tot[k] = s;
-          if (t == 0 && k < w) anorm2[k] = s;
+          if (t > 0 && k >= 2) coef[k - 2] = s;
+          if (t == 0 && k < w) {
+            anorm2[k] = s;
+            int ex;
+            frexpf(2.0f * sqrtf(s), &ex);
+            exS[k] = ex;
+            tauc[k] = (float)p.m * u_work * sqrtf(s);
+          }
         }
       }
     }
@@ -344,12 +388,13 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     const float uu = tot[0];
     const float ua = (t == 0) ? ((w > 1) ? tot[w] : 0.0f) : ((t + 1 < w) ? tot[1] : 0.0f);
     float rtt = sqrtf(uu);
-    const float tau = (float)p.m * u_work * sqrtf(anorm2[t]);
+    const float tau = tauc[t];
     const bool bad = !(rtt > tau) || !isfinite(rtt);
     const float inv = bad ? 0.0f : 1.0f / rtt;
     if (bad) rtt = 0.0f;
     const float ct = ua * inv;                        // r_{t,t+1}
     const bool more = t + 1 < w;
+    if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t * 8 + 5] = clock64();
     if (g == 0) {
       if (threadIdx.x == 0) {
         p.R[t + (int64_t)t * p.ldr] = rtt;
@@ -363,21 +408,47 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     //      (sequential sum per row; rows are independent chains) ----
     float* ut = sp + t * LD;
     float* an = sp + (t + 1) * LD;
-    for (int i = threadIdx.x; i < rows; i += LEAF_THREADS) {
-      const float q = ut[i] * inv;
-      ut[i] = q;
-      if (more) {
-        float u = an[i];
-        int k = 0;
-        for (; k + 8 <= t; k += 8) {
-          float qq[8];
-#pragma unroll
-          for (int e = 0; e < 8; ++e) qq[e] = sp[(k + e) * LD + i];
-#pragma unroll
-          for (int e = 0; e < 8; ++e) u = fmaf(-qq[e], tot[2 + k + e], u);
+    // 4 rows per thread: float4 reads of the q columns and of the coefficients keep the
+    // update off the shared-memory instruction limit; q_t is stored to global here.
+    for (int v = threadIdx.x; v < nv4; v += LEAF_THREADS) {
+      float4 q4 = reinterpret_cast<float4*>(ut)[v];
+      q4.x *= inv; q4.y *= inv; q4.z *= inv; q4.w *= inv;
+      reinterpret_cast<float4*>(ut)[v] = q4;
+      {
+        const int i0 = 4 * v;
+        T* dst = P + r0 + i0 + (int64_t)t * p.ldp;
+        if (p.vec_ok && i0 + 4 <= rows) {
+          store4<T>(dst, q4);
+        } else {
+          const float qv[4] = {q4.x, q4.y, q4.z, q4.w};
+          for (int e = 0; e < 4 && i0 + e < rows; ++e) dst[e] = Elem<T>::store(qv[e]);
         }
-        for (; k < t; ++k) u = fmaf(-sp[k * LD + i], tot[2 + k], u);
-        an[i] = fmaf(-q, ct, u);
+      }
+      if (more) {
+        float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0;
+        int k = 0;
+        for (; k + 4 <= t; k += 4) {
+          const float4 c = reinterpret_cast<const float4*>(coef)[k >> 2];
+          const float4 x0 = reinterpret_cast<const float4*>(sp + (k + 0) * LD)[v];
+          const float4 x1 = reinterpret_cast<const float4*>(sp + (k + 1) * LD)[v];
+          const float4 x2 = reinterpret_cast<const float4*>(sp + (k + 2) * LD)[v];
+          const float4 x3 = reinterpret_cast<const float4*>(sp + (k + 3) * LD)[v];
+          a0.x = fmaf(x0.x, c.x, a0.x); a0.y = fmaf(x0.y, c.x, a0.y); a0.z = fmaf(x0.z, c.x, a0.z); a0.w = fmaf(x0.w, c.x, a0.w);
+          a1.x = fmaf(x1.x, c.y, a1.x); a1.y = fmaf(x1.y, c.y, a1.y); a1.z = fmaf(x1.z, c.y, a1.z); a1.w = fmaf(x1.w, c.y, a1.w);
+          a0.x = fmaf(x2.x, c.z, a0.x); a0.y = fmaf(x2.y, c.z, a0.y); a0.z = fmaf(x2.z, c.z, a0.z); a0.w = fmaf(x2.w, c.z, a0.w);
+          a1.x = fmaf(x3.x, c.w, a1.x); a1.y = fmaf(x3.y, c.w, a1.y); a1.z = fmaf(x3.z, c.w, a1.z); a1.w = fmaf(x3.w, c.w, a1.w);
+        }
+        for (; k < t; ++k) {
+          const float c = coef[k];
+          const float4 x = reinterpret_cast<const float4*>(sp + k * LD)[v];
+          a0.x = fmaf(x.x, c, a0.x); a0.y = fmaf(x.y, c, a0.y); a0.z = fmaf(x.z, c, a0.z); a0.w = fmaf(x.w, c, a0.w);
+        }
+        float4 av = reinterpret_cast<float4*>(an)[v];
+        av.x -= (a0.x + a1.x) + q4.x * ct;
+        av.y -= (a0.y + a1.y) + q4.y * ct;
+        av.z -= (a0.z + a1.z) + q4.z * ct;
+        av.w -= (a0.w + a1.w) + q4.w * ct;
+        reinterpret_cast<float4*>(an)[v] = av;
       }
     }
     __syncthreads();
@@ -386,10 +457,11 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     if (more) {
       const int t1 = t + 1;
       const int L1 = (t1 + 1 < w) ? t1 + 2 : 1;
-      if (p.dbg != nullptr && blockIdx.x == 0 && threadIdx.x == 0) p.dbg[(size_t)t1 * 8] = clock64();
+      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8] = clock64();
       float s_uu, s_ua, s_qa;                            // u^T u, u^T a_{t+2}, q_t^T a_{t+2}
       const bool three = t1 + 1 < w;
       wdot3(t1, three ? t1 + 1 : t1, t, three, s_uu, s_ua, s_qa);
+      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 6] = clock64();
       if (lane == 0) {
         part[warp][0] = s_uu;
         if (t1 + 1 < w) {
@@ -398,9 +470,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
       }
       publish_arrive(t1, L1);
+      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 7] = clock64();
     }
-    // q_t to global after the arrival, so the release does not wait for these stores
-    for (int i = threadIdx.x; i < rows; i += LEAF_THREADS) P[r0 + i + (int64_t)t * p.ldp] = Elem<T>::store(ut[i]);
   }
 }
 

@@ -234,6 +234,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   p.vec_ok = ((ldp * elem_bytes(prec)) % 16 == 0) && (reinterpret_cast<uintptr_t>(P) % 16 == 0);
   if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 8 * LEAF_MAX_W);
   p.dbg = dbg ? dbg_buf : nullptr;
+  p.dbg_cta = dbg ? atoi(getenv("RGSQR_LEAF_DEBUG")) : 0;
   p.breakdown = c->d_breakdown;
   p.col_offset = col_offset;
   cudaError_t e;
@@ -251,11 +252,21 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
     long long hb[8 * LEAF_MAX_W];
     cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 8 * w, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
-    double ph[4] = {0, 0, 0, 0};
-    for (int t = 0; t < w; ++t)
-      for (int i = 0; i < 4; ++i) ph[i] += (double)(hb[t * 8 + i + 1] - hb[t * 8 + i]);
-    fprintf(stderr, "[leaf m=%lld w=%lld G=%d RP=%d] cycles/round: gemv %.0f barrier %.0f gather %.0f update %.0f\n",
-            (long long)m, (long long)w, G, rp, ph[0] / w, ph[1] / w, ph[2] / w, ph[3] / w);
+    // stamps of round t: 0 critical start, 6 after critical dots, 7 after publish, 1 loop top,
+    // 2 after lookahead + barrier, 3 after exchange, 5 after scalars, 4 after update
+    const int order[8] = {0, 6, 7, 1, 2, 3, 5, 4};
+    const char* names[7] = {"crit", "publish", "qstore", "lookahead", "exchange", "scalars", "update"};
+    double ph[7] = {0};
+    int cnt = 0;
+    for (int t = 1; t + 1 < w; ++t, ++cnt)
+      for (int i = 0; i < 7; ++i) ph[i] += (double)(hb[t * 8 + order[i + 1]] - hb[t * 8 + order[i]]);
+    fprintf(stderr, "[leaf m=%lld w=%lld G=%d RP=%d] cycles/round:", (long long)m, (long long)w, G, rp);
+    double sum = 0;
+    for (int i = 0; i < 7; ++i) {
+      fprintf(stderr, " %s %.0f", names[i], ph[i] / std::max(1, cnt));
+      sum += ph[i];
+    }
+    fprintf(stderr, " | total %.0f\n", sum / std::max(1, cnt));
   }
   c->stats.n_leaf_launches++;
   return RGSQR_OK;
