@@ -450,14 +450,49 @@ cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMa
   return launch_gemm_t<T, false, 64>(ma, mb, p, splits, st);
 }
 
+// Many splits (small nodes): one warp per output element; lane l sums splits
+// l, l+32, ... in order, then a fixed xor tree -- deterministic, and the split loads of
+// a warp are issued together instead of as one long dependent chain.
+template <typename T>
+__global__ void splitk_reduce_warp_kernel(const float* __restrict__ P, int64_t split_stride, int64_t ldp,
+                                          int splits, float* C, int64_t ldc, int accumulate, T* Cop,
+                                          int64_t ldop, int64_t M, int64_t N) {
+  const int64_t idx = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (idx >= M * N) return;
+  const int64_t i = idx % M, n = idx / M;
+  float v[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const int s = lane + 32 * q;
+    v[q] = s < splits ? __ldcs(P + s * split_stride + i + n * ldp) : 0.0f;
+  }
+  float acc = v[0];
+#pragma unroll
+  for (int q = 1; q < 8; ++q) acc += v[q];
+  for (int s = lane + 256; s < splits; s += 32) acc += P[s * split_stride + i + n * ldp];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (lane == 0) {
+    if (accumulate) acc = C[i + n * ldc] + acc;
+    C[i + n * ldc] = acc;
+    if (Cop != nullptr) Cop[i + n * ldop] = Elem<T>::store(acc);
+  }
+}
+
 template <typename T>
 cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t ldp, int splits,
                                  float* C, int64_t ldc, int accumulate, T* Cop, int64_t ldop,
                                  int64_t M, int64_t N, cudaStream_t st) {
   const int64_t total = M * N;
   const int threads = 256;
-  splitk_reduce_kernel<T><<<(unsigned)((total + threads - 1) / threads), threads, 0, st>>>(
-      P, split_stride, ldp, splits, C, ldc, accumulate, Cop, ldop, M, N);
+  if (splits >= 16) {
+    splitk_reduce_warp_kernel<T><<<(unsigned)((total * 32 + threads - 1) / threads), threads, 0, st>>>(
+        P, split_stride, ldp, splits, C, ldc, accumulate, Cop, ldop, M, N);
+  } else {
+    splitk_reduce_kernel<T><<<(unsigned)((total + threads - 1) / threads), threads, 0, st>>>(
+        P, split_stride, ldp, splits, C, ldc, accumulate, Cop, ldop, M, N);
+  }
   return cudaGetLastError();
 }
 

@@ -132,9 +132,12 @@ struct Exec {
   }
 
   // ---- in-core node: upload (unless resident), factor, stream Q and R out ----
-  int incore_node(int64_t c0, int64_t w, bool src_q, char* D, bool resident, cudaEvent_t* q_done) {
+  // Rs_ext: caller-owned R block (kept alive by the caller, so no stream has to wait for
+  // its download here); nullptr = allocate it from the arena and fence its reuse.
+  int incore_node(int64_t c0, int64_t w, bool src_q, char* D, bool resident, cudaEvent_t* q_done,
+                  float* Rs_ext = nullptr) {
     const size_t mark = c->arena.mark();
-    float* Rs = static_cast<float*>(c->arena.alloc((size_t)w * w * 4));
+    float* Rs = Rs_ext ? Rs_ext : static_cast<float*>(c->arena.alloc((size_t)w * w * 4));
     if (!Rs) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core node: no space for R block");
     RGSQR_CUDA(c, cudaMemsetAsync(Rs, 0, (size_t)w * w * 4, sc));
     const int64_t leaf = std::max(1, leaf_width_for(c, m));
@@ -184,9 +187,11 @@ struct Exec {
     cudaEvent_t done = c->ev();
     cudaEventRecord(done, sd);
     if (q_done) *q_done = done;
-    // the R block lives in the arena: nobody may reuse it before its download finished
-    cudaStreamWaitEvent(sc, done, 0);
-    cudaStreamWaitEvent(sh, done, 0);
+    if (!Rs_ext) {
+      // the R block lives in released arena space: nobody may reuse it before its download
+      cudaStreamWaitEvent(sc, done, 0);
+      cudaStreamWaitEvent(sh, done, 0);
+    }
     c->arena.release(mark);
     return RGSQR_OK;
   }
@@ -305,10 +310,15 @@ struct Exec {
       char* D = static_cast<char*>(c->arena.alloc(dB));
       float* R12 = static_cast<float*>(c->arena.alloc(r12b));
       void* R12op = c->arena.alloc(r12ob);
+      // the left child's R block lives below the ring for the whole node, so neither the
+      // uploads of the inner pass nor its kernels wait for that block's download
+      const size_t rsb = (size_t)w1 * w1 * 4;
+      float* Rs1 = static_cast<float*>(c->arena.alloc(rsb));
       // ring sized to leave room for the left child's in-core workspace
-      const size_t avail = c->arena.free_bytes() > left_ws + 4096 ? c->arena.free_bytes() - left_ws - 4096 : 0;
+      const size_t ws_left = left_ws > rsb ? left_ws - rsb : 0;
+      const size_t avail = c->arena.free_bytes() > ws_left + 4096 ? c->arena.free_bytes() - ws_left - 4096 : 0;
       const int64_t t = pick_tile(avail, w2);
-      if (!D || !R12 || !R12op || t < 128) {
+      if (!D || !R12 || !R12op || !Rs1 || t < 128) {
         c->arena.release(mark0);
         q1_res = a2_to_d = false;
       } else {
@@ -316,7 +326,7 @@ struct Exec {
         std::vector<cudaEvent_t> ev_free(K);
         for (int k = 0; k < K; ++k) ev_free[k] = c->ev();
         cudaEvent_t q1_done = nullptr;
-        int rc = incore_node(c0, w1, src_q, D, false, &q1_done);
+        int rc = incore_node(c0, w1, src_q, D, false, &q1_done, Rs1);
         if (rc < 0) return rc;
         rc = stream_inner(c0, w1, w2, src_q, D, R12, R12op, ring, t, ev_free);
         if (rc < 0) return rc;
@@ -455,6 +465,8 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   if (c->opt.serialize) x.sh = x.sd = x.sc;
   // make the copy streams start after prior work of the compute stream
   x.join_all();
+  cudaEvent_t t_ref = c->ev();
+  cudaEventRecord(t_ref, x.sc);
   RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), x.sc));
   std::thread zero;
   if (R)
@@ -481,6 +493,20 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   auto& st = c->stats;
   st.pin_ms = std::chrono::duration<double, std::milli>(tp1 - tp0).count();
   st.wall_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+  // optional per-stream timeline (the paper's Figs. 8/10/13 as CSV): RGSQR_TIMELINE=path
+  if (const char* tl = getenv("RGSQR_TIMELINE")) {
+    if (FILE* f = fopen(tl, "w")) {
+      fprintf(f, "stream,start_ms,end_ms\n");
+      const char* nm[3] = {"h2d", "d2h", "compute"};
+      for (auto& sg : c->segs) {
+        float a = 0, b = 0;
+        cudaEventElapsedTime(&a, t_ref, sg.a);
+        cudaEventElapsedTime(&b, t_ref, sg.b);
+        fprintf(f, "%s,%.4f,%.4f\n", nm[sg.kind], a, b);
+      }
+      fclose(f);
+    }
+  }
   for (auto& sg : c->segs) {
     float ms = 0;
     cudaEventElapsedTime(&ms, sg.a, sg.b);
