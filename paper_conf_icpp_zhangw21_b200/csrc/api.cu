@@ -69,6 +69,8 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   if (!R) return fail(c, RGSQR_ERR_INVALID_ARG, "null R");
   reset_stats(c);
   c->begin_call();
+  rc = sync_shape(c, m, &budget);
+  if (rc < 0) return rc;
   auto t0 = std::chrono::steady_clock::now();
   const size_t ws = incore_workspace_bytes(c, prec, m, n);
   const size_t cap = resolve_budget(c, budget);
@@ -91,6 +93,7 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   c->stats.arena_bytes = (int64_t)c->arena.size;
   c->stats.arena_high_water = (int64_t)c->arena.high;
   c->stats.flops = (int64_t)(2.0 * m * (double)n * n);
+  if (brk == -2) return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
   c->stats.first_breakdown_col = brk == 0x7f7f7f7f || brk == INT_MAX ? -1 : brk;
   c->collect_kernel_stats();
   return c->stats.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;
@@ -105,9 +108,14 @@ namespace {
 struct NcclApi {
   void* lib = nullptr;
   int (*getUniqueId)(void*) = nullptr;
-  int (*commInitRank)(void**, int, const void*, int) = nullptr;
+  // ncclCommInitRank takes the 128-byte ncclUniqueId BY VALUE
+  struct UniqueId {
+    char internal[128];
+  };
+  int (*commInitRank)(void**, int, UniqueId, int) = nullptr;
   int (*commDestroy)(void*) = nullptr;
   int (*allReduce)(const void*, void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  int (*allGather)(const void*, void*, size_t, int, void*, cudaStream_t) = nullptr;
   bool load() {
     if (lib) return true;
     const char* names[] = {"libnccl.so.2", "libnccl.so"};
@@ -117,11 +125,13 @@ struct NcclApi {
     }
     if (!lib) return false;
     getUniqueId = reinterpret_cast<int (*)(void*)>(dlsym(lib, "ncclGetUniqueId"));
-    commInitRank = reinterpret_cast<int (*)(void**, int, const void*, int)>(dlsym(lib, "ncclCommInitRank"));
+    commInitRank = reinterpret_cast<int (*)(void**, int, UniqueId, int)>(dlsym(lib, "ncclCommInitRank"));
     commDestroy = reinterpret_cast<int (*)(void*)>(dlsym(lib, "ncclCommDestroy"));
     allReduce = reinterpret_cast<int (*)(const void*, void*, size_t, int, int, void*, cudaStream_t)>(
         dlsym(lib, "ncclAllReduce"));
-    return getUniqueId && commInitRank && commDestroy && allReduce;
+    allGather = reinterpret_cast<int (*)(const void*, void*, size_t, int, void*, cudaStream_t)>(
+        dlsym(lib, "ncclAllGather"));
+    return getUniqueId && commInitRank && commDestroy && allReduce && allGather;
   }
 };
 NcclApi g_nccl;
@@ -144,7 +154,14 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaStreamCreateWithFlags(&c->st_h2d, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
-      cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess) {
+      cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess ||
+      cudaMalloc(&c->d_xw, sizeof(unsigned long long) * 2 * (LEAF_MAX_W + 2)) != cudaSuccess ||
+      cudaMalloc(&c->d_xprev, sizeof(unsigned long long) * 2 * (LEAF_MAX_W + 2)) != cudaSuccess ||
+      cudaMalloc(&c->d_peers, sizeof(void*) * 64) != cudaSuccess ||
+      cudaMalloc(&c->d_r0buf, sizeof(float) * (LEAF_MAX_W + 2)) != cudaSuccess ||
+      cudaMemset(c->d_xw, 0, sizeof(unsigned long long) * 2 * (LEAF_MAX_W + 2)) != cudaSuccess ||
+      cudaMemset(c->d_xprev, 0, sizeof(unsigned long long) * 2 * (LEAF_MAX_W + 2)) != cudaSuccess ||
+      cudaMemcpy(c->d_peers, &c->d_xw, sizeof(void*), cudaMemcpyHostToDevice) != cudaSuccess) {
     delete c;
     return RGSQR_ERR_CUDA;
   }
@@ -155,6 +172,36 @@ int create_impl(rgsqr_handle* h, int device) {
 
 Ctx* C(rgsqr_handle h) { return reinterpret_cast<Ctx*>(h); }
 }  // namespace
+
+namespace rgsqr {
+// Every rank of a row-sharded factorization must take identical planning decisions: check
+// that the local row counts agree, use the smallest resolved budget, record the global m.
+int sync_shape(Ctx* c, int64_t m, size_t* budget) {
+  c->m_global = m;
+  if (!c->nccl_comm) return RGSQR_OK;
+  const size_t b = resolve_budget(c, *budget);
+  int64_t h[3] = {m, -m, -(int64_t)b};
+  int64_t* d = nullptr;
+  if (cudaMalloc(&d, sizeof(h)) != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, "cudaMalloc");
+  cudaMemcpy(d, h, sizeof(h), cudaMemcpyHostToDevice);
+  const int rc = g_nccl.allReduce(d, d, 3, NCCL_INT64, /*ncclMax*/ 2, c->nccl_comm, c->compute());
+  cudaMemcpyAsync(h, d, sizeof(h), cudaMemcpyDeviceToHost, c->compute());
+  cudaStreamSynchronize(c->compute());
+  cudaFree(d);
+  if (rc != 0) return fail(c, RGSQR_ERR_NCCL, "shape allreduce");
+  if (h[0] != -h[1]) return fail(c, RGSQR_ERR_INVALID_ARG, "row-sharded run needs the same local m on every rank");
+  *budget = (size_t)(-h[2]);
+  c->m_global = m * c->nranks;
+  return RGSQR_OK;
+}
+
+int nccl_allreduce(Ctx* c, void* buf, size_t count, int nccl_dtype, cudaStream_t st) {
+  if (!c->nccl_comm) return RGSQR_OK;  // single-GPU context: nothing to reduce
+  if (g_nccl.allReduce(buf, buf, count, nccl_dtype, /*ncclSum*/ 0, c->nccl_comm, st) != 0)
+    return fail(c, RGSQR_ERR_NCCL, "ncclAllReduce failed");
+  return RGSQR_OK;
+}
+}  // namespace rgsqr
 
 extern "C" {
 
@@ -189,11 +236,46 @@ int rgsqr_create_dist(rgsqr_handle* h, int device, int rank, int nranks, const u
   Ctx* c = C(*h);
   c->rank = rank;
   c->nranks = nranks;
+  // A distributed context always has an NCCL communicator (also for nranks == 1, which runs
+  // the row-sharded code paths on one GPU: round-0 allreduce, R12 allreduce, .sys exchange).
+  if (!g_nccl.load()) return fail(c, RGSQR_ERR_NCCL, "libnccl.so.2 not loadable");
+  NcclApi::UniqueId uid;
+  std::memcpy(uid.internal, id, sizeof(uid.internal));
+  if (g_nccl.commInitRank(&c->nccl_comm, nranks, uid, rank) != 0)
+    return fail(c, RGSQR_ERR_NCCL, "ncclCommInitRank failed");
+  // Map every rank's leaf exchange words (CUDA IPC handles exchanged with ncclAllGather),
+  // so the leaf kernel can red.add its partials into all GPUs' words over NVLink.
+  std::vector<unsigned long long*> peers(nranks, nullptr);
+  peers[rank] = c->d_xw;
   if (nranks > 1) {
-    if (!g_nccl.load()) return fail(c, RGSQR_ERR_NCCL, "libnccl.so.2 not loadable");
-    if (g_nccl.commInitRank(&c->nccl_comm, nranks, id, rank) != 0)
-      return fail(c, RGSQR_ERR_NCCL, "ncclCommInitRank failed");
+    cudaIpcMemHandle_t mine;
+    if (cudaIpcGetMemHandle(&mine, c->d_xw) != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, "cudaIpcGetMemHandle");
+    char* dbuf = nullptr;
+    const size_t hs = sizeof(cudaIpcMemHandle_t);
+    if (cudaMalloc(&dbuf, hs * (nranks + 1)) != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, "cudaMalloc");
+    cudaMemcpy(dbuf + hs * nranks, &mine, hs, cudaMemcpyHostToDevice);
+    if (g_nccl.allGather(dbuf + hs * nranks, dbuf, hs, /*ncclChar*/ 0, c->nccl_comm, c->st_own) != 0)
+      return fail(c, RGSQR_ERR_NCCL, "ncclAllGather of IPC handles");
+    std::vector<cudaIpcMemHandle_t> all(nranks);
+    cudaMemcpyAsync(all.data(), dbuf, hs * nranks, cudaMemcpyDeviceToHost, c->st_own);
+    cudaStreamSynchronize(c->st_own);
+    cudaFree(dbuf);
+    for (int j = 0; j < nranks; ++j) {
+      if (j == rank) continue;
+      void* ptr = nullptr;
+      if (cudaIpcOpenMemHandle(&ptr, all[j], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+        return fail(c, RGSQR_ERR_CUDA, "cudaIpcOpenMemHandle (peer " + std::to_string(j) + ")");
+      peers[j] = static_cast<unsigned long long*>(ptr);
+      c->ipc_opened.push_back(ptr);
+    }
   }
+  if (nranks > 64) return fail(c, RGSQR_ERR_UNSUPPORTED, "more than 64 ranks");
+  cudaMemcpy(c->d_peers, peers.data(), sizeof(void*) * nranks, cudaMemcpyHostToDevice);
+  // every rank has zeroed its words (create_impl) before anyone may add into them
+  float one = 0.f;
+  cudaMemcpy(c->d_r0buf, &one, sizeof(float), cudaMemcpyHostToDevice);
+  if (nccl_allreduce(c, c->d_r0buf, 1, NCCL_FLOAT32, c->st_own) < 0 || cudaStreamSynchronize(c->st_own) != cudaSuccess)
+    return fail(c, RGSQR_ERR_NCCL, "initial barrier");
   return RGSQR_OK;
 }
 
@@ -202,11 +284,16 @@ int rgsqr_destroy(rgsqr_handle h) {
   if (!c) return RGSQR_ERR_INVALID_ARG;
   cudaSetDevice(c->device);
   cudaDeviceSynchronize();
+  for (void* ptr : c->ipc_opened) cudaIpcCloseMemHandle(ptr);
   if (c->nccl_comm && g_nccl.commDestroy) g_nccl.commDestroy(c->nccl_comm);
   if (c->arena.base) cudaFree(c->arena.base);
   cudaFree(c->d_partials);
   cudaFree(c->d_counter);
   cudaFree(c->d_breakdown);
+  cudaFree(c->d_xw);
+  cudaFree(c->d_xprev);
+  cudaFree(c->d_peers);
+  cudaFree(c->d_r0buf);
   for (auto e : c->event_pool) cudaEventDestroy(e);
   cudaStreamDestroy(c->st_own);
   cudaStreamDestroy(c->st_h2d);
@@ -243,6 +330,7 @@ int rgsqr_op_leaf(rgsqr_handle h, void* P, int64_t ldp, int64_t m, int64_t w, fl
   int brk = INT_MAX;
   RGSQR_CUDA(c, cudaMemcpyAsync(&brk, c->d_breakdown, sizeof(int), cudaMemcpyDeviceToHost, st));
   RGSQR_CUDA(c, cudaStreamSynchronize(st));
+  if (brk == -2) return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
   if (breakdown) *breakdown = (brk == 0x7f7f7f7f) ? -1 : brk;
   return brk == 0x7f7f7f7f ? RGSQR_OK : RGSQR_WARN_RANK_DEFICIENT;
 }

@@ -75,6 +75,13 @@ struct Ctx {
   unsigned int leaf_epoch = 0;
   int* d_breakdown = nullptr;
   void* nccl_comm = nullptr;
+  // leaf fixed-point exchange (never reset; see leaf.cu)
+  unsigned long long* d_xw = nullptr;        // this GPU's words [2][LEAF_MAX_W+2]
+  unsigned long long* d_xprev = nullptr;     // last-seen words, persistent
+  unsigned long long** d_peers = nullptr;    // [nranks] every GPU's d_xw (IPC-mapped)
+  std::vector<void*> ipc_opened;             // peer mappings to close
+  float* d_r0buf = nullptr;                  // round-0 vector of a row-sharded leaf
+  int64_t m_global = 0;                      // total rows of the current factorization
   std::vector<TimedSeg> segs;
   std::vector<KernSeg> ksegs;
   std::vector<cudaEvent_t> event_pool;
@@ -119,9 +126,18 @@ bool encode_tmap_2d(CUtensorMap* map, int precision, const void* base, uint64_t 
                     int swz = 0);  // 0 SWIZZLE_128B, 1 SWIZZLE_128B_ATOM_32B, 2 none
 
 // ---- ops (device pointers, on stream st) ----
+// reduce_ranks: in a row-sharded run, sum the R12 partials of all ranks (NCCL) before the
+// operand copy is formed; the streamed inner product passes false per tile and reduces
+// once after its last tile (reduce_r12).
 int op_inner(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
              int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate,
-             cudaStream_t st);
+             cudaStream_t st, bool reduce_ranks = true);
+int reduce_r12(Ctx* c, int prec, float* R12, int64_t ldr, void* R12op, int64_t ldop, int64_t w1, int64_t w2,
+               cudaStream_t st);
+int sync_shape(Ctx* c, int64_t m, size_t* budget);
+// NCCL (loaded at run time); sum-allreduce in place on stream st
+int nccl_allreduce(Ctx* c, void* buf, size_t count, int nccl_dtype, cudaStream_t st);
+constexpr int NCCL_INT64 = 4, NCCL_FLOAT32 = 7, NCCL_FLOAT64 = 8;
 int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2,
              int64_t lda, int64_t m, int64_t w1, int64_t w2, cudaStream_t st);
 int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float* R11, int64_t ldr,

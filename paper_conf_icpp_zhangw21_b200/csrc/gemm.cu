@@ -498,6 +498,32 @@ cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t l
 
 int gemm_block_k(int elem_bytes) { return 128 / elem_bytes; }
 
+template <typename T>
+__global__ void copy_cast_kernel(const float* __restrict__ src, int64_t lds, float* dst_f, int64_t ldf, T* dst_op,
+                                 int64_t ldo, int64_t M, int64_t N) {
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= M * N) return;
+  const int64_t i = idx % M, j = idx / M;
+  const float v = src[i + j * lds];
+  if (dst_f) dst_f[i + j * ldf] = v;
+  if (dst_op) dst_op[i + j * ldo] = Elem<T>::store(v);
+}
+
+template <typename T>
+cudaError_t launch_copy_cast(const float* src, int64_t lds, float* dst_f, int64_t ldf, T* dst_op, int64_t ldo,
+                             int64_t M, int64_t N, cudaStream_t st) {
+  const int64_t total = M * N;
+  if (total == 0) return cudaSuccess;
+  copy_cast_kernel<T><<<(unsigned)((total + 255) / 256), 256, 0, st>>>(src, lds, dst_f, ldf, dst_op, ldo, M, N);
+  return cudaGetLastError();
+}
+template cudaError_t launch_copy_cast<__half>(const float*, int64_t, float*, int64_t, __half*, int64_t, int64_t,
+                                              int64_t, cudaStream_t);
+template cudaError_t launch_copy_cast<__nv_bfloat16>(const float*, int64_t, float*, int64_t, __nv_bfloat16*,
+                                                     int64_t, int64_t, int64_t, cudaStream_t);
+template cudaError_t launch_copy_cast<float>(const float*, int64_t, float*, int64_t, float*, int64_t, int64_t,
+                                             int64_t, cudaStream_t);
+
 template cudaError_t launch_gemm<__half>(bool, int, const CUtensorMap&, const CUtensorMap&,
                                          const GemmParams&, int, cudaStream_t);
 template cudaError_t launch_gemm<__nv_bfloat16>(bool, int, const CUtensorMap&, const CUtensorMap&,

@@ -56,7 +56,14 @@ struct LeafParams {
   int vec_ok;               // P and ldp*sizeof(elem) 16-byte aligned: vector panel loads
   int xmode;                // 0: counter barrier + gather; 2: fixed-point red.add exchange
   unsigned int epoch;       // launch counter
-  unsigned long long* xw;   // [2][LEAF_MAX_W+2] exchange words (zeroed by the launcher)
+  unsigned long long* xw;   // [2][LEAF_MAX_W+2] this GPU's exchange words (never reset)
+  unsigned long long* const* xw_peers;  // device array [nranks]: every GPU's xw (row-sharded run)
+  unsigned long long* xprev_g;          // [2][LEAF_MAX_W+2] last-seen words, persistent
+  int nranks;               // GPUs sharing the rows of the panel
+  int sys;                  // distributed context: red.add into every rank's words, .sys scope
+  int r0_mode;              // 0 round 0 in-kernel, 1 round-0-only (write r0buf), 2 round 0 given
+  float* r0buf;             // [LEAF_MAX_W+2] round-0 vector (modes 1, 2)
+  int64_t m_global;         // total rows (breakdown threshold)
   int* breakdown;           // device int, atomicMin of the first breakdown column
   int64_t col_offset;       // global index of the panel's first column
 };
@@ -74,8 +81,9 @@ cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t l
 template <typename T>
 cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st);
 
+// dst_f[i,j] = src[i,j] (optional) and dst_op[i,j] = RN(src[i,j]) (optional), M x N
 template <typename T>
-cudaError_t launch_cast(const float* src, int64_t lds, T* dst, int64_t ldd, int64_t M, int64_t N,
-                        cudaStream_t st);
+cudaError_t launch_copy_cast(const float* src, int64_t lds, float* dst_f, int64_t ldf, T* dst_op, int64_t ldo,
+                             int64_t M, int64_t N, cudaStream_t st);
 
 }  // namespace rgsqr

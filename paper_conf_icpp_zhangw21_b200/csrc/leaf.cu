@@ -40,6 +40,17 @@ __device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long
   asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ unsigned long long ld_word(const unsigned long long* p, int sys) {
+  if (!sys) return ld_relaxed_u64(p);
+  unsigned long long v;
+  asm volatile("ld.relaxed.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Fixed-point exchange word: bits [53,64) count arrivals (<= 2047 = ranks x CTAs),
+// bits [0,53) accumulate (v + 2^41) with |v| <= 2^41 per arrival (no carry into the count).
+static constexpr int FX_CNT_SHIFT = 53;
+static constexpr int FX_VBITS = 41;
 
 // exact power of two as a double (|e| < 1000)
 __device__ __forceinline__ double pow2d(int e) { return __hiloint2double((1023 + e) << 20, 0); }
@@ -139,7 +150,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   __shared__ __align__(16) float coef[LEAF_MAX_W + 4];      // r_{i,t+1}, i < t (aligned copy)
   __shared__ int exS[LEAF_MAX_W];                           // 2||a_j|| < 2^exS[j]
   __shared__ float tauc[LEAF_MAX_W];                        // breakdown thresholds
-  for (int i = threadIdx.x; i < 2 * (LEAF_MAX_W + 2); i += blockDim.x) (&xprev[0][0])[i] = 0ull;
+  // last-seen exchange words persist across launches (words are never reset, see fx_exp)
+  for (int i = threadIdx.x; i < 2 * (LEAF_MAX_W + 2); i += blockDim.x) (&xprev[0][0])[i] = p.xprev_g[i];
+  const unsigned fx_count = (unsigned)(p.nranks * gridDim.x);   // arrivals per word per round
 
   const int G = gridDim.x;
   const int g = blockIdx.x;
@@ -235,9 +248,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   auto fx_exp = [&](int t, int k) -> int {
     // |partial| <= bound with bound = 4 ||a_t||^2, 4 ||a_t|| ||a_{t+1}|| or 4 ||a_{t+1}||
     // (u_t shrinks a_t, ||q_i|| <= 1); exS[j] = exponent with 2 ||a_j|| < 2^exS[j]
-    if (k == 0) return 46 - 2 * exS[t];
-    if (k == 1) return 46 - (exS[t] + exS[t + 1]);
-    return 46 - (exS[t + 1] + 1);
+    if (k == 0) return FX_VBITS - 2 * exS[t];
+    if (k == 1) return FX_VBITS - (exS[t] + exS[t + 1]);
+    return FX_VBITS - (exS[t + 1] + 1);
   };
   // publish the L values of part[][] as this CTA's partial vector of round t, arrive
   auto publish_arrive = [&](int t, int L) {
@@ -257,11 +270,18 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     if (k < L && jq == 0) {
       if (fx) {
         long long v = __double2ll_rn((double)s * pow2d(fx_exp(t, k)));
-        v = v > (1ll << 46) ? (1ll << 46) : (v < -(1ll << 46) ? -(1ll << 46) : v);
-        const unsigned long long add = (1ull << 56) + (unsigned long long)(v + (1ll << 46));
-        asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + (t & 1) * (LEAF_MAX_W + 2) + k),
-                     "l"(add)
-                     : "memory");
+        const long long vb = 1ll << FX_VBITS;
+        v = v > vb ? vb : (v < -vb ? -vb : v);
+        const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
+        const size_t off = (size_t)(t & 1) * (LEAF_MAX_W + 2) + k;
+        if (!p.sys) {
+          asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + off), "l"(add) : "memory");
+        } else {
+          // row-sharded run: the same word on every GPU receives every CTA's partial
+          for (int j = 0; j < p.nranks; ++j)
+            asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(p.xw_peers[j] + off), "l"(add)
+                         : "memory");
+        }
       } else {
         buf[(size_t)k * G + g] = s;
       }
@@ -274,7 +294,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   };
 
   // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ] ----
-  {
+  // (r0_mode 2: the globally reduced round-0 vector is given in p.r0buf)
+  if (p.r0_mode != 2) {
     const int t = 0;
     const int L = w + (w > 1 ? 1 : 0);
     DBG_STAMP(0);
@@ -319,8 +340,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       }
     }
     const bool fx = p.xmode == 2 && t > 0;
+    const bool given = t == 0 && p.r0_mode == 2;
     // ---- grid barrier of round t (arrived in publish_arrive) ----
-    if (!fx && threadIdx.x == 0) {
+    if (!fx && !given && threadIdx.x == 0) {
       unsigned cv;
       const unsigned target = (p.xmode == 2 ? 1u : (unsigned)(t + 1)) * (unsigned)G;
       do {
@@ -336,16 +358,35 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         const int k = threadIdx.x;
         unsigned long long* wp = p.xw + (t & 1) * (LEAF_MAX_W + 2) + k;
         const unsigned long long prev = xprev[t & 1][k];
-        unsigned long long now = ld_relaxed_u64(wp), d = now - prev;
-        while ((unsigned)(d >> 56) != (unsigned)G) {
-          now = ld_relaxed_u64(wp);
+        unsigned long long now = ld_word(wp, p.sys), d = now - prev;
+        long long spins = 0;
+        while ((unsigned)(d >> FX_CNT_SHIFT) != fx_count) {
+          now = ld_word(wp, p.sys);
           d = now - prev;
+          if (++spins > (1ll << 27)) {            // ~seconds: a peer is missing -- fail, never hang
+            atomicExch(p.breakdown, -2);
+            break;
+          }
         }
         xprev[t & 1][k] = now;
-        const long long total = (long long)(d & ((1ull << 56) - 1)) - (long long)G * (1ll << 46);
+        const long long total =
+            (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)fx_count * (1ll << FX_VBITS);
         const float val = (float)((double)total * pow2d(-fx_exp(t, k)));
         tot[k] = val;
         if (k >= 2) coef[k - 2] = val;
+      }
+    } else if (given) {
+      if (threadIdx.x < L) {
+        const int k = threadIdx.x;
+        const float s = p.r0buf[k];
+        tot[k] = s;
+        if (k < w) {
+          anorm2[k] = s;
+          int ex;
+          frexpf(2.0f * sqrtf(s), &ex);
+          exS[k] = ex;
+          tauc[k] = (float)p.m_global * u_work * sqrtf(s);
+        }
       }
     } else {
       // ---- gather round t's G partials per value, fixed-order sum ----
@@ -377,13 +418,19 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
             int ex;
             frexpf(2.0f * sqrtf(s), &ex);
             exS[k] = ex;
-            tauc[k] = (float)p.m * u_work * sqrtf(s);
+            tauc[k] = (float)p.m_global * u_work * sqrtf(s);
           }
         }
       }
     }
     __syncthreads();
     DBG_STAMP(3);
+    if (t == 0 && p.r0_mode == 1) {
+      // round-0-only launch of a row-sharded run: hand the local vector to the host
+      // (which all-reduces it across GPUs) and stop
+      if (g == 0 && threadIdx.x < L) p.r0buf[threadIdx.x] = tot[threadIdx.x];
+      return;
+    }
     // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{:,t+1} ----
     const float uu = tot[0];
     const float ua = (t == 0) ? ((w > 1) ? tot[w] : 0.0f) : ((t + 1 < w) ? tot[1] : 0.0f);
@@ -473,6 +520,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 7] = clock64();
     }
   }
+  // every CTA ends with the same last-seen words; CTA 0 persists them for the next launch
+  if (g == 0)
+    for (int i = threadIdx.x; i < 2 * (LEAF_MAX_W + 2); i += blockDim.x) p.xprev_g[i] = (&xprev[0][0])[i];
 }
 
 template <typename T>
@@ -486,8 +536,6 @@ cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
     attr_smem = smem;
   }
   cudaError_t e = cudaMemsetAsync(p.counter, 0, sizeof(unsigned int), st);
-  if (e != cudaSuccess) return e;
-  e = cudaMemsetAsync(p.xw, 0, sizeof(unsigned long long) * 2 * (LEAF_MAX_W + 2), st);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);

@@ -222,9 +222,15 @@ struct Exec {
       cudaStreamWaitEvent(sc, loaded[k], 0);
       cudaEvent_t a = seg_begin(sc);
       const bool last = (i + 1 == tl.size());
-      rc = op_inner(c, prec, D ? D + r0 * s : sq, D ? m : t, sa, t, tr, w1, w2, R12, w1, last ? R12op : nullptr,
-                    w1, i > 0 ? 1 : 0, sc);
+      // distributed: accumulate the LOCAL partial over all tiles, reduce across ranks once
+      const bool dist = c->nccl_comm != nullptr;
+      rc = op_inner(c, prec, D ? D + r0 * s : sq, D ? m : t, sa, t, tr, w1, w2, R12, w1,
+                    (last && !dist) ? R12op : nullptr, w1, i > 0 ? 1 : 0, sc, /*reduce_ranks=*/false);
       if (rc < 0) return rc;
+      if (last && dist) {
+        rc = reduce_r12(c, prec, R12, w1, R12op, w1, w1, w2, sc);
+        if (rc < 0) return rc;
+      }
       seg_end(2, sc, a);
       cudaEventRecord(ev_free[k], sc);
       r0 += tr;
@@ -417,8 +423,9 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   int rc = validate(c, A, lda, m, n, Q, prec);
   if (rc < 0) return rc;
   if (!R && c->rank == 0) return fail(c, RGSQR_ERR_INVALID_ARG, "null R_out");
-  if (c->nranks > 1) return fail(c, RGSQR_ERR_UNSUPPORTED, "row-sharded multi-GPU factorization not built yet");
   reset_stats(c);
+  rc = sync_shape(c, m, &budget);
+  if (rc < 0) return rc;
   c->begin_call();
   const int s = elem_bytes(prec);
 
@@ -518,6 +525,7 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   st.arena_bytes = (int64_t)c->arena.size;
   st.arena_high_water = (int64_t)c->arena.high;
   st.flops = (int64_t)(2.0 * m * (double)n * n);
+  if (brk == -2) return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
   st.first_breakdown_col = (brk == 0x7f7f7f7f || brk == INT_MAX) ? -1 : brk;
   c->collect_kernel_stats();
   return st.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;

@@ -88,9 +88,37 @@ bool encode_tmap_2d(CUtensorMap* map, int precision, const void* base, uint64_t 
 static int pick_bn(int64_t N) { return N >= 256 ? 256 : (N > 64 ? 128 : 64); }
 
 template <typename T>
+static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
+                          int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
+                          int accumulate, cudaStream_t st);
+
+// Row-sharded run: R12 = sum over ranks of the local Q1^T A2.  The local
+// partial goes to a contiguous temporary, is summed with ncclAllReduce, and only then
+// copied into R and rounded into the operand copy (the outer product and Q stay row-local).
+template <typename T>
 static int op_inner_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
                       int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate,
-                      cudaStream_t st) {
+                      cudaStream_t st, bool reduce_ranks) {
+  if (!c->nccl_comm || !reduce_ranks)
+    return op_inner_local<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+  if (accumulate) return fail(c, RGSQR_ERR_UNSUPPORTED, "inner: accumulate with rank reduction");
+  const size_t mark = c->arena.mark();
+  float* tmp = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * sizeof(float)));
+  if (!tmp) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner: no arena space for the R12 reduction");
+  int rc = op_inner_local<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, tmp, w1, nullptr, 0, 0, st);
+  if (rc < 0) return rc;
+  rc = nccl_allreduce(c, tmp, (size_t)w1 * w2, NCCL_FLOAT32, st);
+  if (rc < 0) return rc;
+  RGSQR_CUDA(c, launch_copy_cast<T>(tmp, w1, R12, ldr, static_cast<T*>(R12op), ldop, w1, w2, st));
+  c->stats.n_other_launches++;
+  c->arena.release(mark);
+  return RGSQR_OK;
+}
+
+template <typename T>
+static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
+                          int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
+                          int accumulate, cudaStream_t st) {
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
   const int bn = pick_bn(w2);
@@ -168,16 +196,43 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
 }
 
 int op_inner(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m, int64_t w1,
-             int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate, cudaStream_t st) {
+             int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate, cudaStream_t st,
+             bool reduce_ranks) {
   switch (prec) {
     case RGSQR_FP16:
-      return op_inner_t<__half>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+      return op_inner_t<__half>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st,
+                                reduce_ranks);
     case RGSQR_BF16:
-      return op_inner_t<__nv_bfloat16>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+      return op_inner_t<__nv_bfloat16>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st,
+                                       reduce_ranks);
     case RGSQR_TF32:
-      return op_inner_t<float>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+      return op_inner_t<float>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st,
+                               reduce_ranks);
   }
   return fail(c, RGSQR_ERR_UNSUPPORTED, "inner: precision not supported");
+}
+
+int reduce_r12(Ctx* c, int prec, float* R12, int64_t ldr, void* R12op, int64_t ldop, int64_t w1, int64_t w2,
+               cudaStream_t st) {
+  if (ldr != w1) return fail(c, RGSQR_ERR_INVALID_ARG, "reduce_r12: R12 must be contiguous");
+  if (c->nccl_comm) {
+    int rc = nccl_allreduce(c, R12, (size_t)w1 * w2, NCCL_FLOAT32, st);
+    if (rc < 0) return rc;
+  }
+  cudaError_t e;
+  switch (prec) {
+    case RGSQR_FP16:
+      e = launch_copy_cast<__half>(R12, ldr, nullptr, 0, static_cast<__half*>(R12op), ldop, w1, w2, st);
+      break;
+    case RGSQR_BF16:
+      e = launch_copy_cast<__nv_bfloat16>(R12, ldr, nullptr, 0, static_cast<__nv_bfloat16*>(R12op), ldop, w1,
+                                          w2, st);
+      break;
+    default: e = launch_copy_cast<float>(R12, ldr, nullptr, 0, static_cast<float*>(R12op), ldop, w1, w2, st);
+  }
+  if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("reduce_r12: ") + cudaGetErrorString(e));
+  c->stats.n_other_launches++;
+  return RGSQR_OK;
 }
 
 int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2, int64_t lda,
@@ -230,20 +285,47 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   static const int xmode = getenv("RGSQR_LEAF_XMODE") ? atoi(getenv("RGSQR_LEAF_XMODE")) : 2;
   p.xmode = xmode;
   p.epoch = ++c->leaf_epoch;
-  p.xw = reinterpret_cast<unsigned long long*>(c->d_counter + 64);  // 256-byte offset in the 4 KiB block
+  p.xw = c->d_xw;
+  p.xw_peers = c->d_peers;
+  p.xprev_g = c->d_xprev;
+  p.nranks = c->nranks;
+  p.sys = c->nccl_comm != nullptr;
+  p.r0buf = c->d_r0buf;
+  p.m_global = c->m_global > 0 ? c->m_global : m;
   p.vec_ok = ((ldp * elem_bytes(prec)) % 16 == 0) && (reinterpret_cast<uintptr_t>(P) % 16 == 0);
   if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 8 * LEAF_MAX_W);
   p.dbg = dbg ? dbg_buf : nullptr;
   p.dbg_cta = dbg ? atoi(getenv("RGSQR_LEAF_DEBUG")) : 0;
   p.breakdown = c->d_breakdown;
   p.col_offset = col_offset;
+  if (c->nccl_comm && p.xmode != 2) return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: sharded runs need xmode 2");
+  auto launch = [&](const LeafParams& q) -> cudaError_t {
+    switch (prec) {
+      case RGSQR_FP16: return launch_leaf<__half>(q, G, st);
+      case RGSQR_BF16: return launch_leaf<__nv_bfloat16>(q, G, st);
+      case RGSQR_TF32: return launch_leaf<float>(q, G, st);
+    }
+    return cudaErrorInvalidValue;
+  };
+  if (prec != RGSQR_FP16 && prec != RGSQR_BF16 && prec != RGSQR_TF32)
+    return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: precision not supported");
   cudaError_t e;
   cudaEvent_t kb = c->kbegin(st);
-  switch (prec) {
-    case RGSQR_FP16: e = launch_leaf<__half>(p, G, st); break;
-    case RGSQR_BF16: e = launch_leaf<__nv_bfloat16>(p, G, st); break;
-    case RGSQR_TF32: e = launch_leaf<float>(p, G, st); break;
-    default: return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: precision not supported");
+  if (!c->nccl_comm) {
+    p.r0_mode = 0;
+    e = launch(p);
+  } else {
+    // row-sharded: round 0 (column norms -> fixed-point scales) is summed over GPUs by NCCL
+    // between a round-0-only launch and the main launch; later rounds reduce in-kernel
+    LeafParams p0 = p;
+    p0.r0_mode = 1;
+    e = launch(p0);
+    if (e == cudaSuccess) {
+      int rc = nccl_allreduce(c, c->d_r0buf, (size_t)w + 1, NCCL_FLOAT32, st);
+      if (rc < 0) return rc;
+      p.r0_mode = 2;
+      e = launch(p);
+    }
   }
   if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("leaf launch: ") + cudaGetErrorString(e));
   const int s = elem_bytes(prec);
@@ -289,6 +371,7 @@ size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n) {
   const int64_t w1 = split_width(n, leaf);
   size_t b = 0;
   if (w1 > 0) b += (size_t)w1 * (n - w1) * elem_bytes(prec) + 1024;  // R12 operand copy
+  if (w1 > 0 && c->nccl_comm) b += (size_t)w1 * (n - w1) * 4 + 1024;  // R12 rank-reduction buffer
   // split-K partials: op_inner adapts its split factor to what is free; reserve a
   // quarter of the node's matrix bytes, clamped to [1, 16] MiB
   const size_t node_bytes = (size_t)m * n * elem_bytes(prec);

@@ -118,7 +118,7 @@ class Handle:
     def __init__(self, device: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes | None = None):
         self.lib = load_library()
         h = C.c_void_p()
-        if nranks > 1:
+        if unique_id is not None:      # distributed context (also nranks == 1: same code paths)
             rc = self.lib.rgsqr_create_dist(C.byref(h), device, rank, nranks, unique_id)
         else:
             rc = self.lib.rgsqr_create(C.byref(h), device)
