@@ -53,7 +53,6 @@ int validate(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, const voi
   if (n < 1 || m < n) return fail(c, RGSQR_ERR_INVALID_ARG, "need 1 <= n <= m");
   if (lda < m) return fail(c, RGSQR_ERR_INVALID_ARG, "need lda >= m");
   if (prec < RGSQR_FP16 || prec > RGSQR_TF32X3) return fail(c, RGSQR_ERR_INVALID_ARG, "bad precision");
-  if (prec == RGSQR_TF32X3) return fail(c, RGSQR_ERR_UNSUPPORTED, "TF32X3 not implemented yet");
   const int s = elem_bytes(prec);
   if ((lda * s) % 16 != 0) return fail(c, RGSQR_ERR_INVALID_ARG, "lda*sizeof(elem) must be a multiple of 16");
   if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(Q)) & 15)

@@ -498,6 +498,26 @@ cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t l
 
 int gemm_block_k(int elem_bytes) { return 128 / elem_bytes; }
 
+// TF32X3 operand split: lo = x - trunc_tf32(x) (exact in fp32).  The hi part is the
+// original array: tcgen05 kind::tf32 reads only the top 19 bits of each fp32 word.
+__global__ void tf32_lo_kernel(const float* __restrict__ src, int64_t lds, float* __restrict__ dst, int64_t ldd,
+                               int64_t M, int64_t N) {
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= M * N) return;
+  const int64_t i = idx % M, j = idx / M;
+  const float x = src[i + j * lds];
+  const float hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
+  dst[i + j * ldd] = x - hi;
+}
+
+cudaError_t launch_tf32_lo(const float* src, int64_t lds, float* dst, int64_t ldd, int64_t M, int64_t N,
+                           cudaStream_t st) {
+  const int64_t total = M * N;
+  if (total == 0) return cudaSuccess;
+  tf32_lo_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(src, lds, dst, ldd, M, N);
+  return cudaGetLastError();
+}
+
 template <typename T>
 __global__ void copy_cast_kernel(const float* __restrict__ src, int64_t lds, float* dst_f, int64_t ldf, T* dst_op,
                                  int64_t ldo, int64_t M, int64_t N) {

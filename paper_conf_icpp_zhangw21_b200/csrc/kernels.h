@@ -81,6 +81,9 @@ cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t l
 template <typename T>
 cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st);
 
+// TF32X3: dst = src - trunc_tf32(src), M x N
+cudaError_t launch_tf32_lo(const float* src, int64_t lds, float* dst, int64_t ldd, int64_t M, int64_t N,
+                           cudaStream_t st);
 // dst_f[i,j] = src[i,j] (optional) and dst_op[i,j] = RN(src[i,j]) (optional), M x N
 template <typename T>
 cudaError_t launch_copy_cast(const float* src, int64_t lds, float* dst_f, int64_t ldf, T* dst_op, int64_t ldo,

@@ -124,6 +124,7 @@ struct Exec {
     return v;
   }
   int64_t pick_tile(size_t avail, int64_t cols_per_slot) const {
+    if (prec == RGSQR_TF32X3) avail /= 2;  // leave room for the per-tile lo operands
     int64_t t = (int64_t)(avail / ((size_t)K * cols_per_slot * s));
     t = std::min<int64_t>(t, tmax);
     t = std::min<int64_t>(t, (m + 127) / 128 * 128);

@@ -116,9 +116,37 @@ static int op_inner_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
 }
 
 template <typename T>
+static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
+                         int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
+                         int accumulate, cudaStream_t st);
+
+// TF32X3 (3-pass split tf32): Q1^T A2 ~= Q1h^T A2h + Q1h^T A2l + Q1l^T A2h, hi = the stored
+// fp32 words read as tf32 (truncated by the MMA), lo = x - trunc_tf32(x); the three
+// products accumulate into R12 in this fixed order.  Error ~ |Q1l||A2l| ~ 2^-22 relative.
+template <typename T>
 static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
                           int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
                           int accumulate, cudaStream_t st) {
+  if (prec != RGSQR_TF32X3)
+    return op_inner_once<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
+  const size_t mark = c->arena.mark();
+  float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
+  float* a_lo = static_cast<float*>(c->arena.alloc((size_t)m * w2 * 4));
+  if (!q_lo || !a_lo) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner (tf32x3): no space for the lo operands");
+  RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(Q1), ldq, q_lo, m, m, w1, st));
+  RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(A2), lda, a_lo, m, m, w2, st));
+  c->stats.n_other_launches += 2;
+  int rc = op_inner_once<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, nullptr, 0, accumulate, st);
+  if (rc == 0) rc = op_inner_once<T>(c, prec, Q1, ldq, a_lo, m, m, w1, w2, R12, ldr, nullptr, 0, 1, st);
+  if (rc == 0) rc = op_inner_once<T>(c, prec, q_lo, m, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, 1, st);
+  c->arena.release(mark);
+  return rc;
+}
+
+template <typename T>
+static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
+                         int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
+                         int accumulate, cudaStream_t st) {
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
   const int bn = pick_bn(w2);
@@ -206,6 +234,7 @@ int op_inner(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int6
       return op_inner_t<__nv_bfloat16>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st,
                                        reduce_ranks);
     case RGSQR_TF32:
+    case RGSQR_TF32X3:
       return op_inner_t<float>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st,
                                reduce_ranks);
   }
@@ -241,6 +270,21 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
     case RGSQR_FP16: return op_outer_t<__half>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
     case RGSQR_BF16: return op_outer_t<__nv_bfloat16>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
     case RGSQR_TF32: return op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
+    case RGSQR_TF32X3: {
+      // A2 <- ((A2 - Q1h R12h) - Q1h R12l) - Q1l R12h  (three in-place tf32 updates)
+      const size_t mark = c->arena.mark();
+      float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
+      float* r_lo = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
+      if (!q_lo || !r_lo) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "outer (tf32x3): no space for lo operands");
+      RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(Q1), ldq, q_lo, m, m, w1, st));
+      RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(R12op), ldr, r_lo, w1, w1, w2, st));
+      c->stats.n_other_launches += 2;
+      int rc = op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
+      if (rc == 0) rc = op_outer_t<float>(c, prec, Q1, ldq, r_lo, w1, A2, lda, m, w1, w2, st);
+      if (rc == 0) rc = op_outer_t<float>(c, prec, q_lo, m, R12op, ldr, A2, lda, m, w1, w2, st);
+      c->arena.release(mark);
+      return rc;
+    }
   }
   return fail(c, RGSQR_ERR_UNSUPPORTED, "outer: precision not supported");
 }
@@ -303,11 +347,12 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
     switch (prec) {
       case RGSQR_FP16: return launch_leaf<__half>(q, G, st);
       case RGSQR_BF16: return launch_leaf<__nv_bfloat16>(q, G, st);
-      case RGSQR_TF32: return launch_leaf<float>(q, G, st);
+      case RGSQR_TF32:
+      case RGSQR_TF32X3: return launch_leaf<float>(q, G, st);   // fp32 CUDA-core leaf either way
     }
     return cudaErrorInvalidValue;
   };
-  if (prec != RGSQR_FP16 && prec != RGSQR_BF16 && prec != RGSQR_TF32)
+  if (prec < RGSQR_FP16 || prec > RGSQR_TF32X3)
     return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: precision not supported");
   cudaError_t e;
   cudaEvent_t kb = c->kbegin(st);
@@ -372,6 +417,7 @@ size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n) {
   size_t b = 0;
   if (w1 > 0) b += (size_t)w1 * (n - w1) * elem_bytes(prec) + 1024;  // R12 operand copy
   if (w1 > 0 && c->nccl_comm) b += (size_t)w1 * (n - w1) * 4 + 1024;  // R12 rank-reduction buffer
+  if (prec == RGSQR_TF32X3) b += (size_t)m * n * 4 + 4096;              // lo operands of the top node
   // split-K partials: op_inner adapts its split factor to what is free; reserve a
   // quarter of the node's matrix bytes, clamped to [1, 16] MiB
   const size_t node_bytes = (size_t)m * n * elem_bytes(prec);

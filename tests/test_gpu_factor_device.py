@@ -77,3 +77,28 @@ def test_repeatable_bitwise(h):
     _, Q2, R2 = run(h, A, "fp16", "fp16", 8192, 512)
     np.testing.assert_array_equal(R1, R2)
     np.testing.assert_array_equal(Q1, Q2)
+
+
+@pytest.mark.parametrize("m,n", [(4096, 256), (8192, 512)])
+def test_tf32x3_meets_north_star_1e5(h, m, n):
+    """BASELINE.json: backward error and R error <= 1e-5 for the TF32 path; one-pass TF32
+    cannot reach it (R15), the 3-pass split mode must."""
+    A = gi.gaussian(m, n, seed=1, dtype="fp32")
+    X = gi.to_float64(A, "fp32")
+    rc, Q, R = run(h, A, "fp32", "tf32x3", m, n)
+    assert rc == 0
+    ref = oracle.rgs(X, leaf=64)
+    be = oracle.backward_error(X, Q, R)
+    re = oracle.r_rel_error(R, ref.R)
+    assert be <= 1e-5 and re <= 1e-5, (be, re)
+
+
+def test_tf32x3_usv_kappa_1e3(h):
+    m, n = 8192, 256
+    A64, _ = gi.usv(m, n, kappa=1e3, seed=3)
+    A = gi.to_storage(A64, "fp32")
+    X = gi.to_float64(A, "fp32")
+    rc, Q, R = run(h, A, "fp32", "tf32x3", m, n)
+    ref = oracle.gram_cholesky_r(X)
+    assert oracle.backward_error(X, Q, R) <= 1e-5
+    assert oracle.r_rel_error(R, ref) <= 1e-5

@@ -137,3 +137,14 @@ def test_zero_column_warning(h):
     rc, Q, R, st = factor(h, A, "fp16", 4 * MiB)
     assert rc == 1 and st["first_breakdown_col"] == 100
     assert R[100, 100] == 0
+
+
+def test_ooc_tf32x3(h):
+    m, n = 16384, 512
+    A = gi.gaussian(m, n, seed=9, dtype="fp32")
+    X = gi.to_float64(A, "fp32")
+    rc, Q, R, st = factor(h, A, "tf32x3", 40 * MiB)
+    assert rc == 0 and st["n_ooc_nodes"] >= 1
+    Rg = R.astype(np.float64)
+    assert oracle.backward_error(X, Q.astype(np.float64), Rg) <= 1e-5
+    assert oracle.r_rel_error(Rg, oracle.rgs(X, leaf=64).R) <= 1e-5
