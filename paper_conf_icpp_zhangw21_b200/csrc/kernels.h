@@ -53,6 +53,7 @@ struct LeafParams {
   unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
   long long* dbg;           // optional [w][8] clock64 stamps of CTA dbg_cta
   int dbg_cta;
+  int skip;                 // diagnostics only (RGSQR_LEAF_SKIP): 1 update, 2 lookahead, 4 critical dots
   int vec_ok;               // P and ldp*sizeof(elem) 16-byte aligned: vector panel loads
   int xmode;                // 0: counter barrier + gather; 2: fixed-point red.add exchange
   unsigned int epoch;       // launch counter

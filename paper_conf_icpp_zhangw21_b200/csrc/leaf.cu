@@ -312,7 +312,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     DBG_STAMP(1);
     // ---- lookahead (overlaps the barrier): round t+1's q_i^T a_{t+2}, i <= t-1.
     //      q_i (i <= t-1) are final and a_{t+2} is untouched until round t+1. ----
-    if (t + 2 < w && t >= 1) {
+    if (t + 2 < w && t >= 1 && !(p.skip & 2)) {
       const int cnt = t;                               // i in [0, t-1]
       const int ya = t + 2;
       const bool ha = kq < cnt, hb = kq + 32 < cnt;
@@ -457,7 +457,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     float* an = sp + (t + 1) * LD;
     // 4 rows per thread: float4 reads of the q columns and of the coefficients keep the
     // update off the shared-memory instruction limit; q_t is stored to global here.
-    for (int v = threadIdx.x; v < nv4; v += LEAF_THREADS) {
+    for (int v = threadIdx.x; v < ((p.skip & 1) ? 0 : nv4); v += LEAF_THREADS) {
       float4 q4 = reinterpret_cast<float4*>(ut)[v];
       q4.x *= inv; q4.y *= inv; q4.z *= inv; q4.w *= inv;
       reinterpret_cast<float4*>(ut)[v] = q4;
@@ -507,7 +507,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8] = clock64();
       float s_uu, s_ua, s_qa;                            // u^T u, u^T a_{t+2}, q_t^T a_{t+2}
       const bool three = t1 + 1 < w;
-      wdot3(t1, three ? t1 + 1 : t1, t, three, s_uu, s_ua, s_qa);
+      if (p.skip & 4) { s_uu = 1.f; s_ua = s_qa = 0.f; }
+      else wdot3(t1, three ? t1 + 1 : t1, t, three, s_uu, s_ua, s_qa);
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 6] = clock64();
       if (lane == 0) {
         part[warp][0] = s_uu;

@@ -340,6 +340,8 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 8 * LEAF_MAX_W);
   p.dbg = dbg ? dbg_buf : nullptr;
   p.dbg_cta = dbg ? atoi(getenv("RGSQR_LEAF_DEBUG")) : 0;
+  static const int skip = getenv("RGSQR_LEAF_SKIP") ? atoi(getenv("RGSQR_LEAF_SKIP")) : 0;
+  p.skip = dbg ? skip : 0;
   p.breakdown = c->d_breakdown;
   p.col_offset = col_offset;
   if (c->nccl_comm && p.xmode != 2) return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: sharded runs need xmode 2");
