@@ -93,13 +93,23 @@ def gaussian(m: int, n: int, seed: int = 1, dtype: str = "fp32", row0: int = 0,
         raise ValueError("row0 must be a multiple of ROW_BLOCK")
     if out is None:
         out = np.empty((m, n), dtype=storage_numpy_dtype(dtype), order="F")
-    r = 0
-    while r < m:
+
+    def fill(r):
         b = (row0 + r) // ROW_BLOCK
         rows = min(ROW_BLOCK, m - r)
         blk = _block_rng(seed, b).standard_normal((n, ROW_BLOCK), dtype=np.float32)[:, :rows]
         out[r:r + rows, :] = f32_to_bf16_bits(blk.T) if dtype == "bf16" else blk.T
-        r += rows
+
+    starts = list(range(0, m, ROW_BLOCK))
+    if m * n >= (1 << 26) and len(starts) > 1:
+        # blocks are independent streams: fill them in parallel (numpy releases the GIL)
+        from concurrent.futures import ThreadPoolExecutor
+        import os
+        with ThreadPoolExecutor(max_workers=min(len(starts), len(os.sched_getaffinity(0)))) as ex:
+            list(ex.map(fill, starts))
+    else:
+        for r in starts:
+            fill(r)
     return out
 
 
