@@ -9,6 +9,10 @@ namespace rgsqr {
 constexpr int LEAF_MAX_W = 64;
 constexpr int LEAF_MAX_G = 160;       // leaf grid size cap (>= SM count)
 constexpr int LEAF_PARTS = 4;         // row quarters of the per-CTA partial sums
+// leaf exchange words: [2 parities][LEAF_MAX_W+2 values][LEAF_XW_COPIES]; CTA g adds into
+// copy g % LEAF_XW_COPIES, so no single L2 word receives more than ~G/4 atomics per round
+constexpr int LEAF_XW_COPIES = 4;
+constexpr int LEAF_XW_WORDS = 2 * (LEAF_MAX_W + 2) * LEAF_XW_COPIES;
 constexpr size_t LEAF_SMEM_BUDGET = 200 * 1024;
 // smem column stride of the leaf panel slice: >= rows and == 4 (mod 32), so that the
 // float4 reads of 8 threads at the same row in 8 different columns hit 32 distinct banks

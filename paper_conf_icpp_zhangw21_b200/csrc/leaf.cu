@@ -145,14 +145,13 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
   __shared__ float tot[LEAF_MAX_W + 2];            // reduced round vector
   __shared__ float anorm2[LEAF_MAX_W];             // ||a_k||^2 (breakdown threshold)
-  __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];
-  __shared__ unsigned long long xprev[2][LEAF_MAX_W + 2];  // last seen exchange words
-  __shared__ __align__(16) float coef[LEAF_MAX_W + 4];      // r_{i,t+1}, i < t (aligned copy)
+  __shared__ float part[2][GEMV_PARTS][LEAF_MAX_W + 2];     // by round parity
+  __shared__ unsigned long long xprev[LEAF_XW_WORDS];      // last seen exchange words
+  __shared__ __align__(16) float coef[2][LEAF_MAX_W + 4];   // r_{i,t+2}, i < t, by parity of t
   __shared__ int exS[LEAF_MAX_W];                           // 2||a_j|| < 2^exS[j]
   __shared__ float tauc[LEAF_MAX_W];                        // breakdown thresholds
   // last-seen exchange words persist across launches (words are never reset, see fx_exp)
-  for (int i = threadIdx.x; i < 2 * (LEAF_MAX_W + 2); i += blockDim.x) (&xprev[0][0])[i] = p.xprev_g[i];
-  const unsigned fx_count = (unsigned)(p.nranks * gridDim.x);   // arrivals per word per round
+  for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) xprev[i] = p.xprev_g[i];
 
   const int G = gridDim.x;
   const int g = blockIdx.x;
@@ -246,11 +245,12 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   // (deterministic) and exact in fixed point; the word is never reset within a launch:
   // readers take the difference with the value they saw two rounds earlier.
   auto fx_exp = [&](int t, int k) -> int {
-    // |partial| <= bound with bound = 4 ||a_t||^2, 4 ||a_t|| ||a_{t+1}|| or 4 ||a_{t+1}||
-    // (u_t shrinks a_t, ||q_i|| <= 1); exS[j] = exponent with 2 ||a_j|| < 2^exS[j]
+    // |partial| <= bound: 4||a_t||^2, 4||a_t|| ||a_{t+1}||, 4||a_{t+1}||, 4||a_{t+2}|| for value
+    // classes 0, 1, 2, 3+ (u_t shrinks a_t, ||q_i|| <= 1); 2||a_j|| < 2^exS[j]
     if (k == 0) return FX_VBITS - 2 * exS[t];
     if (k == 1) return FX_VBITS - (exS[t] + exS[t + 1]);
-    return FX_VBITS - (exS[t + 1] + 1);
+    if (k == 2) return FX_VBITS - (exS[t + 1] + 1);
+    return FX_VBITS - (exS[t + 2] + 1);
   };
   // publish the L values of part[][] as this CTA's partial vector of round t, arrive
   auto publish_arrive = [&](int t, int L) {
@@ -263,7 +263,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     float s = 0.f;
     if (k < L) {
 #pragma unroll
-      for (int q = 0; q < GEMV_PARTS / 4; ++q) s += part[jq * (GEMV_PARTS / 4) + q][k];
+      for (int q = 0; q < GEMV_PARTS / 4; ++q) s += part[t & 1][jq * (GEMV_PARTS / 4) + q][k];
     }
     s += __shfl_xor_sync(0xffffffffu, s, 1);
     s += __shfl_xor_sync(0xffffffffu, s, 2);
@@ -273,7 +273,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         const long long vb = 1ll << FX_VBITS;
         v = v > vb ? vb : (v < -vb ? -vb : v);
         const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
-        const size_t off = (size_t)(t & 1) * (LEAF_MAX_W + 2) + k;
+        const size_t off = ((size_t)(t & 1) * (LEAF_MAX_W + 2) + k) * LEAF_XW_COPIES + g % LEAF_XW_COPIES;
         if (!p.sys) {
           asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + off), "l"(add) : "memory");
         } else {
@@ -293,55 +293,67 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     }
   };
 
+  // Round layout (t >= 1), R19:  [0] u_t.u_t  [1] u_t.a_{t+1}  [2] q_{t-1}.a_{t+1}
+  // [3+i] q_i.a_{t+2} (i <= t-1).  The q_i.a_{t+2} values are published one round ahead, so
+  // after round t every CTA already knows r_{i,t+2} (i <= t-1) and can subtract those
+  // projections from a_{t+2} while round t+1's exchange is in flight; after that exchange
+  // only q_t and q_{t+1} remain to be subtracted (two columns on the critical path).
+  auto round_len = [&](int t) -> int {
+    if (t == 0) return w + (w > 1 ? 1 : 0);
+    if (t == w - 1) return 1;
+    if (t == w - 2) return 3;
+    return t + 3;
+  };
+  // col -= sum_{i < cnt} q_i * cf[i]   (4 rows per thread, fixed order of i within two sums)
+  auto project_out = [&](int col, int cnt, const float* cf) {
+    float* an = sp + col * LD;
+    for (int v = threadIdx.x; v < nv4; v += LEAF_THREADS) {
+      float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0;
+      int k = 0;
+      for (; k + 4 <= cnt; k += 4) {
+        const float4 c = reinterpret_cast<const float4*>(cf)[k >> 2];
+        const float4 x0 = reinterpret_cast<const float4*>(sp + (k + 0) * LD)[v];
+        const float4 x1 = reinterpret_cast<const float4*>(sp + (k + 1) * LD)[v];
+        const float4 x2 = reinterpret_cast<const float4*>(sp + (k + 2) * LD)[v];
+        const float4 x3 = reinterpret_cast<const float4*>(sp + (k + 3) * LD)[v];
+        a0.x = fmaf(x0.x, c.x, a0.x); a0.y = fmaf(x0.y, c.x, a0.y); a0.z = fmaf(x0.z, c.x, a0.z); a0.w = fmaf(x0.w, c.x, a0.w);
+        a1.x = fmaf(x1.x, c.y, a1.x); a1.y = fmaf(x1.y, c.y, a1.y); a1.z = fmaf(x1.z, c.y, a1.z); a1.w = fmaf(x1.w, c.y, a1.w);
+        a0.x = fmaf(x2.x, c.z, a0.x); a0.y = fmaf(x2.y, c.z, a0.y); a0.z = fmaf(x2.z, c.z, a0.z); a0.w = fmaf(x2.w, c.z, a0.w);
+        a1.x = fmaf(x3.x, c.w, a1.x); a1.y = fmaf(x3.y, c.w, a1.y); a1.z = fmaf(x3.z, c.w, a1.z); a1.w = fmaf(x3.w, c.w, a1.w);
+      }
+      for (; k < cnt; ++k) {
+        const float c = cf[k];
+        const float4 x = reinterpret_cast<const float4*>(sp + k * LD)[v];
+        a0.x = fmaf(x.x, c, a0.x); a0.y = fmaf(x.y, c, a0.y); a0.z = fmaf(x.z, c, a0.z); a0.w = fmaf(x.w, c, a0.w);
+      }
+      float4 av = reinterpret_cast<float4*>(an)[v];
+      av.x -= a0.x + a1.x;
+      av.y -= a0.y + a1.y;
+      av.z -= a0.z + a1.z;
+      av.w -= a0.w + a1.w;
+      reinterpret_cast<float4*>(an)[v] = av;
+    }
+  };
+
   // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ] ----
   // (r0_mode 2: the globally reduced round-0 vector is given in p.r0buf)
   if (p.r0_mode != 2) {
     const int t = 0;
-    const int L = w + (w > 1 ? 1 : 0);
+    const int L = round_len(0);
     DBG_STAMP(0);
     for (int k = kq; k < L; k += 32) {
       int cx, cy;
       round_operands(0, w, k, cx, cy);
-      part[warp][k] = dot4(cx, cy);
+      part[0][warp][k] = dot4(cx, cy);
     }
     publish_arrive(0, L);
   }
 
   for (int t = 0; t < w; ++t) {
-    const int L = (t == 0) ? w + (w > 1 ? 1 : 0) : ((t + 1 < w) ? t + 2 : 1);
-    DBG_STAMP(1);
-    // ---- lookahead (overlaps the barrier): round t+1's q_i^T a_{t+2}, i <= t-1.
-    //      q_i (i <= t-1) are final and a_{t+2} is untouched until round t+1. ----
-    if (t + 2 < w && t >= 1 && !(p.skip & 2)) {
-      const int cnt = t;                               // i in [0, t-1]
-      const int ya = t + 2;
-      const bool ha = kq < cnt, hb = kq + 32 < cnt;
-      if (ha) {
-        const float4* y = reinterpret_cast<const float4*>(sp + ya * LD);
-        const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
-        const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
-        float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
-        for (int i = v_lo; i < v_hi; ++i) {
-          const float4 yy = y[i], a = xa[i];
-          a0 = fmaf(a.x, yy.x, a0);
-          a1 = fmaf(a.y, yy.y, a1);
-          a0 = fmaf(a.z, yy.z, a0);
-          a1 = fmaf(a.w, yy.w, a1);
-          if (hb) {
-            const float4 b = xb[i];
-            b0 = fmaf(b.x, yy.x, b0);
-            b1 = fmaf(b.y, yy.y, b1);
-            b0 = fmaf(b.z, yy.z, b0);
-            b1 = fmaf(b.w, yy.w, b1);
-          }
-        }
-        part[warp][2 + kq] = a0 + a1;
-        if (hb) part[warp][2 + kq + 32] = b0 + b1;
-      }
-    }
+    const int L = round_len(t);
     const bool fx = p.xmode == 2 && t > 0;
     const bool given = t == 0 && p.r0_mode == 2;
-    // ---- grid barrier of round t (arrived in publish_arrive) ----
+    // ---- wait for round t (counter barrier for round 0 / xmode 0) ----
     if (!fx && !given && threadIdx.x == 0) {
       unsigned cv;
       const unsigned target = (p.xmode == 2 ? 1u : (unsigned)(t + 1)) * (unsigned)G;
@@ -350,17 +362,22 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       } while (cv < target);
     }
     __syncthreads();
-    DBG_STAMP(2);
     if (fx) {
-      // ---- fixed-point exchange: each value's word is polled by its thread until all G
-      //      CTAs have added (measured: a single-sentinel poll + extra barrier is slower) ----
-      if (threadIdx.x < L) {
-        const int k = threadIdx.x;
-        unsigned long long* wp = p.xw + (t & 1) * (LEAF_MAX_W + 2) + k;
-        const unsigned long long prev = xprev[t & 1][k];
+      // ---- fixed-point exchange: each value's word is polled by its thread until all
+      //      ranks x G CTAs have added ----
+      // LEAF_XW_COPIES threads per value, one word copy each; the copies' integer totals are
+      // summed with an xor tree (exact, so the order does not matter)
+      const int k = threadIdx.x / LEAF_XW_COPIES, hc = threadIdx.x % LEAF_XW_COPIES;
+      long long total = 0;
+      if (k < L) {
+        const int widx = ((t & 1) * (LEAF_MAX_W + 2) + k) * LEAF_XW_COPIES + hc;
+        const unsigned cnt_h =
+            (unsigned)p.nranks * (unsigned)(G / LEAF_XW_COPIES + (hc < G % LEAF_XW_COPIES ? 1 : 0));
+        const unsigned long long* wp = p.xw + widx;
+        const unsigned long long prev = xprev[widx];
         unsigned long long now = ld_word(wp, p.sys), d = now - prev;
         long long spins = 0;
-        while ((unsigned)(d >> FX_CNT_SHIFT) != fx_count) {
+        while ((unsigned)(d >> FX_CNT_SHIFT) != cnt_h) {
           now = ld_word(wp, p.sys);
           d = now - prev;
           if (++spins > (1ll << 27)) {            // ~seconds: a peer is missing -- fail, never hang
@@ -368,12 +385,15 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
             break;
           }
         }
-        xprev[t & 1][k] = now;
-        const long long total =
-            (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)fx_count * (1ll << FX_VBITS);
+        xprev[widx] = now;
+        total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt_h * (1ll << FX_VBITS);
+      }
+#pragma unroll
+      for (int o = 1; o < LEAF_XW_COPIES; o <<= 1) total += __shfl_xor_sync(0xffffffffu, total, o);
+      if (k < L && hc == 0) {
         const float val = (float)((double)total * pow2d(-fx_exp(t, k)));
         tot[k] = val;
-        if (k >= 2) coef[k - 2] = val;
+        if (k >= 3) coef[t & 1][k - 3] = val;
       }
     } else if (given) {
       if (threadIdx.x < L) {
@@ -412,7 +432,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
         if (lane == 0) {
           tot[k] = s;
-          if (t > 0 && k >= 2) coef[k - 2] = s;
+          if (t > 0 && k >= 3) coef[t & 1][k - 3] = s;
           if (t == 0 && k < w) {
             anorm2[k] = s;
             int ex;
@@ -424,106 +444,153 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       }
     }
     __syncthreads();
-    DBG_STAMP(3);
+    DBG_STAMP(2);
     if (t == 0 && p.r0_mode == 1) {
       // round-0-only launch of a row-sharded run: hand the local vector to the host
       // (which all-reduces it across GPUs) and stop
       if (g == 0 && threadIdx.x < L) p.r0buf[threadIdx.x] = tot[threadIdx.x];
       return;
     }
-    // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{:,t+1} ----
+    // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{t,t+1}, r_{t-1,t+1} ----
+    const bool more = t + 1 < w;
     const float uu = tot[0];
-    const float ua = (t == 0) ? ((w > 1) ? tot[w] : 0.0f) : ((t + 1 < w) ? tot[1] : 0.0f);
+    const float ua = (t == 0) ? ((w > 1) ? tot[w] : 0.0f) : (more ? tot[1] : 0.0f);
+    const float cq = (t >= 1 && more) ? tot[2] : 0.0f;   // r_{t-1,t+1} = q_{t-1}^T a_{t+1}
     float rtt = sqrtf(uu);
     const float tau = tauc[t];
     const bool bad = !(rtt > tau) || !isfinite(rtt);
     const float inv = bad ? 0.0f : 1.0f / rtt;
     if (bad) rtt = 0.0f;
-    const float ct = ua * inv;                        // r_{t,t+1}
-    const bool more = t + 1 < w;
-    if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t * 8 + 5] = clock64();
+    const float ct = ua * inv;                            // r_{t,t+1}
     if (g == 0) {
       if (threadIdx.x == 0) {
         p.R[t + (int64_t)t * p.ldr] = rtt;
         if (bad) atomicMin(p.breakdown, (int)(p.col_offset + t));
       }
-      if (more && threadIdx.x <= t)
-        p.R[threadIdx.x + (int64_t)(t + 1) * p.ldr] = threadIdx.x == t ? ct : tot[2 + threadIdx.x];
+      if (more && threadIdx.x <= t) {
+        const int i = threadIdx.x;
+        const float r = (i == t) ? ct : (i == t - 1) ? cq : coef[(t - 1) & 1][i];   // i <= t-2: round t-1
+        p.R[i + (int64_t)(t + 1) * p.ldr] = r;
+      }
       if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
     }
-    // ---- q_t = u_t / r_tt (stored rounded), u_{t+1} = a_{t+1} - sum_{i<=t} q_i r_{i,t+1}
-    //      (sequential sum per row; rows are independent chains) ----
-    float* ut = sp + t * LD;
-    float* an = sp + (t + 1) * LD;
-    // 4 rows per thread: float4 reads of the q columns and of the coefficients keep the
-    // update off the shared-memory instruction limit; q_t is stored to global here.
-    for (int v = threadIdx.x; v < ((p.skip & 1) ? 0 : nv4); v += LEAF_THREADS) {
-      float4 q4 = reinterpret_cast<float4*>(ut)[v];
-      q4.x *= inv; q4.y *= inv; q4.z *= inv; q4.w *= inv;
-      reinterpret_cast<float4*>(ut)[v] = q4;
-      {
-        const int i0 = 4 * v;
-        T* dst = P + r0 + i0 + (int64_t)t * p.ldp;
-        if (p.vec_ok && i0 + 4 <= rows) {
-          store4<T>(dst, q4);
-        } else {
-          const float qv[4] = {q4.x, q4.y, q4.z, q4.w};
-          for (int e = 0; e < 4 && i0 + e < rows; ++e) dst[e] = Elem<T>::store(qv[e]);
+    DBG_STAMP(5);
+    // ---- q_t = u_t / r_tt (stored rounded); u_{t+1} = w_{t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1}
+    //      where w_{t+1} = a_{t+1} - sum_{i<=t-2} q_i r_{i,t+1} was formed during round t ----
+    {
+      float* ut = sp + t * LD;
+      float* an = sp + (t + 1) * LD;
+      const float* qp = sp + (t >= 1 ? t - 1 : 0) * LD;
+      for (int v = threadIdx.x; v < ((p.skip & 1) ? 0 : nv4); v += LEAF_THREADS) {
+        float4 q4 = reinterpret_cast<float4*>(ut)[v];
+        q4.x *= inv; q4.y *= inv; q4.z *= inv; q4.w *= inv;
+        reinterpret_cast<float4*>(ut)[v] = q4;
+        {
+          const int i0 = 4 * v;
+          T* dst = P + r0 + i0 + (int64_t)t * p.ldp;
+          if (p.vec_ok && i0 + 4 <= rows) {
+            store4<T>(dst, q4);
+          } else {
+            const float qv[4] = {q4.x, q4.y, q4.z, q4.w};
+            for (int e = 0; e < 4 && i0 + e < rows; ++e) dst[e] = Elem<T>::store(qv[e]);
+          }
         }
-      }
-      if (more) {
-        float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0;
-        int k = 0;
-        for (; k + 4 <= t; k += 4) {
-          const float4 c = reinterpret_cast<const float4*>(coef)[k >> 2];
-          const float4 x0 = reinterpret_cast<const float4*>(sp + (k + 0) * LD)[v];
-          const float4 x1 = reinterpret_cast<const float4*>(sp + (k + 1) * LD)[v];
-          const float4 x2 = reinterpret_cast<const float4*>(sp + (k + 2) * LD)[v];
-          const float4 x3 = reinterpret_cast<const float4*>(sp + (k + 3) * LD)[v];
-          a0.x = fmaf(x0.x, c.x, a0.x); a0.y = fmaf(x0.y, c.x, a0.y); a0.z = fmaf(x0.z, c.x, a0.z); a0.w = fmaf(x0.w, c.x, a0.w);
-          a1.x = fmaf(x1.x, c.y, a1.x); a1.y = fmaf(x1.y, c.y, a1.y); a1.z = fmaf(x1.z, c.y, a1.z); a1.w = fmaf(x1.w, c.y, a1.w);
-          a0.x = fmaf(x2.x, c.z, a0.x); a0.y = fmaf(x2.y, c.z, a0.y); a0.z = fmaf(x2.z, c.z, a0.z); a0.w = fmaf(x2.w, c.z, a0.w);
-          a1.x = fmaf(x3.x, c.w, a1.x); a1.y = fmaf(x3.y, c.w, a1.y); a1.z = fmaf(x3.z, c.w, a1.z); a1.w = fmaf(x3.w, c.w, a1.w);
+        if (more) {
+          float4 av = reinterpret_cast<float4*>(an)[v];
+          if (t >= 1) {
+            const float4 qm = reinterpret_cast<const float4*>(qp)[v];
+            av.x = fmaf(-qm.x, cq, av.x); av.y = fmaf(-qm.y, cq, av.y);
+            av.z = fmaf(-qm.z, cq, av.z); av.w = fmaf(-qm.w, cq, av.w);
+          }
+          av.x = fmaf(-q4.x, ct, av.x); av.y = fmaf(-q4.y, ct, av.y);
+          av.z = fmaf(-q4.z, ct, av.z); av.w = fmaf(-q4.w, ct, av.w);
+          reinterpret_cast<float4*>(an)[v] = av;
         }
-        for (; k < t; ++k) {
-          const float c = coef[k];
-          const float4 x = reinterpret_cast<const float4*>(sp + k * LD)[v];
-          a0.x = fmaf(x.x, c, a0.x); a0.y = fmaf(x.y, c, a0.y); a0.z = fmaf(x.z, c, a0.z); a0.w = fmaf(x.w, c, a0.w);
-        }
-        float4 av = reinterpret_cast<float4*>(an)[v];
-        av.x -= (a0.x + a1.x) + q4.x * ct;
-        av.y -= (a0.y + a1.y) + q4.y * ct;
-        av.z -= (a0.z + a1.z) + q4.z * ct;
-        av.w -= (a0.w + a1.w) + q4.w * ct;
-        reinterpret_cast<float4*>(an)[v] = av;
       }
     }
     __syncthreads();
     DBG_STAMP(4);
-    // ---- round t+1: the three dots that needed round t, then publish + arrive ----
-    if (more) {
+    if (!more) break;
+    // ---- round t+1: the dots that needed round t -- u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2},
+    //      q_t.a_{t+2}, q_t.a_{t+3} -- then publish + arrive ----
+    {
       const int t1 = t + 1;
-      const int L1 = (t1 + 1 < w) ? t1 + 2 : 1;
+      const int L1 = round_len(t1);
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8] = clock64();
-      float s_uu, s_ua, s_qa;                            // u^T u, u^T a_{t+2}, q_t^T a_{t+2}
-      const bool three = t1 + 1 < w;
-      if (p.skip & 4) { s_uu = 1.f; s_ua = s_qa = 0.f; }
-      else wdot3(t1, three ? t1 + 1 : t1, t, three, s_uu, s_ua, s_qa);
+      const bool h2 = t + 2 < w, h3 = t + 3 < w;
+      const float* u = sp + t1 * LD;
+      const float* qv = sp + t * LD;
+      const float* a2 = sp + (h2 ? t + 2 : t1) * LD;
+      const float* a3 = sp + (h3 ? t + 3 : t1) * LD;
+      float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+      if (!(p.skip & 4)) {
+        for (int i = c_lo + lane; i < c_hi; i += 32) {
+          const float uv = u[i];
+          s0 = fmaf(uv, uv, s0);
+          if (h2) {
+            const float av = a2[i], qq = qv[i];
+            s1 = fmaf(uv, av, s1);
+            s2 = fmaf(qq, av, s2);
+            if (h3) s3 = fmaf(qq, a3[i], s3);
+          }
+        }
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        s0 += __shfl_xor_sync(0xffffffffu, s0, o);
+        s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+        s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+        s3 += __shfl_xor_sync(0xffffffffu, s3, o);
+      }
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 6] = clock64();
       if (lane == 0) {
-        part[warp][0] = s_uu;
-        if (t1 + 1 < w) {
-          part[warp][1] = s_ua;
-          part[warp][2 + t] = s_qa;
+        float* pw = part[t1 & 1][warp];
+        pw[0] = s0;
+        if (h2) {
+          pw[1] = s1;
+          pw[2] = s2;
+          if (h3) pw[3 + t] = s3;                        // q_t.a_{t1+2}: index 3 + (t1 - 1)
         }
       }
       publish_arrive(t1, L1);
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 7] = clock64();
     }
+    // ---- while round t+1's exchange is in flight:
+    //      (a) lookahead for round t+2: q_i.a_{t+4}, i <= t  (index 3 + i)
+    //      (b) w_{t+2} = a_{t+2} - sum_{i <= t-1} q_i r_{i,t+2}  (coefficients from round t) ----
+    if (t + 4 < w && !(p.skip & 2)) {
+      const int cnt = t + 1;                              // i in [0, t]
+      const bool ha = kq < cnt, hb = kq + 32 < cnt;
+      if (ha) {
+        const float4* y = reinterpret_cast<const float4*>(sp + (t + 4) * LD);
+        const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
+        const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
+        float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+        for (int i = v_lo; i < v_hi; ++i) {
+          const float4 yy = y[i], a = xa[i];
+          a0 = fmaf(a.x, yy.x, a0);
+          a1 = fmaf(a.y, yy.y, a1);
+          a0 = fmaf(a.z, yy.z, a0);
+          a1 = fmaf(a.w, yy.w, a1);
+          if (hb) {
+            const float4 b = xb[i];
+            b0 = fmaf(b.x, yy.x, b0);
+            b1 = fmaf(b.y, yy.y, b1);
+            b0 = fmaf(b.z, yy.z, b0);
+            b1 = fmaf(b.w, yy.w, b1);
+          }
+        }
+        float* pw = part[t & 1][warp];                    // round t+2 has the parity of t
+        pw[3 + kq] = a0 + a1;
+        if (hb) pw[3 + kq + 32] = b0 + b1;
+      }
+    }
+    if (t + 2 < w && t >= 1) project_out(t + 2, t, coef[t & 1]);
+    if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)(t + 1) * 8 + 1] = clock64();
   }
   // every CTA ends with the same last-seen words; CTA 0 persists them for the next launch
   if (g == 0)
-    for (int i = threadIdx.x; i < 2 * (LEAF_MAX_W + 2); i += blockDim.x) p.xprev_g[i] = (&xprev[0][0])[i];
+    for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) p.xprev_g[i] = xprev[i];
 }
 
 template <typename T>

@@ -381,17 +381,17 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
     long long hb[8 * LEAF_MAX_W];
     cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 8 * w, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
-    // stamps of round t: 0 critical start, 6 after critical dots, 7 after publish, 1 loop top,
-    // 2 after lookahead + barrier, 3 after exchange, 5 after scalars, 4 after update
-    const int order[8] = {0, 6, 7, 1, 2, 3, 5, 4};
-    const char* names[7] = {"crit", "publish", "qstore", "lookahead", "exchange", "scalars", "update"};
-    double ph[7] = {0};
+    // stamps of round t: 0 critical start, 6 after critical dots, 7 after publish, 1 after the
+    // overlapped lookahead + precompute, 2 after the exchange, 5 after scalars, 4 after update
+    const int order[7] = {0, 6, 7, 1, 2, 5, 4};
+    const char* names[6] = {"crit", "publish", "overlap", "exchange", "scalars", "update"};
+    double ph[6] = {0};
     int cnt = 0;
     for (int t = 1; t + 1 < w; ++t, ++cnt)
-      for (int i = 0; i < 7; ++i) ph[i] += (double)(hb[t * 8 + order[i + 1]] - hb[t * 8 + order[i]]);
+      for (int i = 0; i < 6; ++i) ph[i] += (double)(hb[t * 8 + order[i + 1]] - hb[t * 8 + order[i]]);
     fprintf(stderr, "[leaf m=%lld w=%lld G=%d RP=%d] cycles/round:", (long long)m, (long long)w, G, rp);
     double sum = 0;
-    for (int i = 0; i < 7; ++i) {
+    for (int i = 0; i < 6; ++i) {
       fprintf(stderr, " %s %.0f", names[i], ph[i] / std::max(1, cnt));
       sum += ph[i];
     }
