@@ -154,11 +154,11 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
       cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess ||
-      cudaMalloc(&c->d_xw, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||
+      cudaMalloc(&c->d_xw, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
       cudaMalloc(&c->d_xprev, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||
       cudaMalloc(&c->d_peers, sizeof(void*) * 64) != cudaSuccess ||
       cudaMalloc(&c->d_r0buf, sizeof(float) * (LEAF_MAX_W + 2)) != cudaSuccess ||
-      cudaMemset(c->d_xw, 0, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||
+      cudaMemset(c->d_xw, 0, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
       cudaMemset(c->d_xprev, 0, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||
       cudaMemcpy(c->d_peers, &c->d_xw, sizeof(void*), cudaMemcpyHostToDevice) != cudaSuccess) {
     delete c;

@@ -9,10 +9,12 @@ namespace rgsqr {
 constexpr int LEAF_MAX_W = 64;
 constexpr int LEAF_MAX_G = 160;       // leaf grid size cap (>= SM count)
 constexpr int LEAF_PARTS = 4;         // row quarters of the per-CTA partial sums
-// leaf exchange words: [2 parities][LEAF_MAX_W+2 values][LEAF_XW_COPIES]; CTA g adds into
-// copy g % LEAF_XW_COPIES, so no single L2 word receives more than ~G/4 atomics per round
-constexpr int LEAF_XW_COPIES = 4;
-constexpr int LEAF_XW_WORDS = 2 * (LEAF_MAX_W + 2) * LEAF_XW_COPIES;
+// leaf exchange words: [LEAF_XW_SETS round sets][LEAF_MAX_W+2 values], word i at
+// xw[i * LEAF_XW_STRIDE] (one 256-byte line each: concurrent atomics and polls of different
+// values land in different L2 slices)
+constexpr int LEAF_XW_SETS = 4;
+constexpr int LEAF_XW_STRIDE = 32;
+constexpr int LEAF_XW_WORDS = LEAF_XW_SETS * (LEAF_MAX_W + 2);
 constexpr size_t LEAF_SMEM_BUDGET = 200 * 1024;
 // smem column stride of the leaf panel slice: >= rows and == 4 (mod 32), so that the
 // float4 reads of 8 threads at the same row in 8 different columns hit 32 distinct banks
@@ -57,13 +59,12 @@ struct LeafParams {
   unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
   long long* dbg;           // optional [w][8] clock64 stamps of CTA dbg_cta
   int dbg_cta;
-  int skip;                 // diagnostics only (RGSQR_LEAF_SKIP): 1 update, 2 lookahead, 4 critical dots
+  int skip;                 // diagnostics only (RGSQR_LEAF_SKIP): 2 lookahead dots, 4 projection
   int vec_ok;               // P and ldp*sizeof(elem) 16-byte aligned: vector panel loads
-  int xmode;                // 0: counter barrier + gather; 2: fixed-point red.add exchange
   unsigned int epoch;       // launch counter
-  unsigned long long* xw;   // [2][LEAF_MAX_W+2] this GPU's exchange words (never reset)
+  unsigned long long* xw;   // LEAF_XW_WORDS words (stride LEAF_XW_STRIDE), this GPU's, never reset
   unsigned long long* const* xw_peers;  // device array [nranks]: every GPU's xw (row-sharded run)
-  unsigned long long* xprev_g;          // [2][LEAF_MAX_W+2] last-seen words, persistent
+  unsigned long long* xprev_g;          // [LEAF_XW_WORDS] last-seen words, persistent
   int nranks;               // GPUs sharing the rows of the panel
   int sys;                  // distributed context: red.add into every rank's words, .sys scope
   int r0_mode;              // 0 round 0 in-kernel, 1 round-0-only (write r0buf), 2 round 0 given

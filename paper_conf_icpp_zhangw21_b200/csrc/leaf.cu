@@ -7,22 +7,24 @@
 // CGS needs reductions over all m rows; they are done in ROUNDS, one round per column:
 //
 //   round 0 : S = [ ||a_k||^2 (k < w),  a_0^T a_1 ]
-//   round t : S = [ u_t^T u_t,  u_t^T a_{t+1},  q_i^T a_{t+1} (i < t) ]
+//   round t : S = [ u_t^T u_t,  u_t^T a_{t+1},  q_{t-1}^T a_{t+1},  q_i^T a_{t+2} (i <= t-1) ]
 //   after round t (every CTA, identical scalars):
 //       r_tt = ||u_t||,  q_t = u_t / r_tt,  r_{t,t+1} = (u_t^T a_{t+1}) / r_tt,
-//       r_{i,t+1} = q_i^T a_{t+1} (i < t),  u_{t+1} = a_{t+1} - sum_{i<=t} q_i r_{i,t+1}.
+//       u_{t+1} = w_{t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1},
+//       w_{t+2} = a_{t+2} - sum_{i<=t-1} q_i r_{i,t+2}   (while round t+1 is in flight)
 //
 // i.e. the projection coefficient of the column just normalised is folded into the
 // norm's reduction (q_t^T a = (u_t^T a) / r_tt), so each column costs ONE grid-wide
 // reduction instead of two -- the same CGS quantities up to rounding order
 // (reading R19).
 //
-// Exchange per round: each CTA writes its partial vector (fp32) to global memory,
-// arrives on a counter (release) and spins on it (acquire); then every CTA loads the
-// G partials of each value (all loads of a warp issued together) and sums them in the
-// same fixed order (deterministic, no float atomics).  Measured alternatives
-// (scripts/barrier_bench.cu, RGSQR_LEAF_DEBUG stamps): per-word round tags avoid the
-// counter but flood L2 with spinning loads (4x slower gather).
+// Exchange (rounds >= 1): every CTA red.add's each of its partials, converted to an exact
+// fixed-point integer, into one 64-bit word per value that also counts arrivals; the
+// value's thread in every CTA polls the word until all CTAs have added.  Integer sums are
+// order-independent, so the result is deterministic.  Only the 4 values that depend on the
+// previous round sit on the critical path; the others (q_i^T a_{t+2}, i <= t-2) are added
+// two rounds early.  Round 0 uses a counter barrier + fixed-order gather of fp32 partials.
+// Measured alternatives: scripts/barrier_bench.cu, scripts/exchange_bench.cu.
 #include "dtype.cuh"
 #include "kernels.h"
 
@@ -128,24 +130,12 @@ __device__ __forceinline__ void store4<float>(float* dst, float4 v) {
   *reinterpret_cast<float4*>(dst) = v;
 }
 
-// column pair (x, y) whose dot product is value k of round t
-__device__ __forceinline__ void round_operands(int t, int w, int k, int& cx, int& cy) {
-  if (t == 0) {
-    if (k < w) { cx = k; cy = k; }                     // ||a_k||^2
-    else { cx = 0; cy = 1; }                           // a_0^T a_1
-  } else {
-    if (k == 0) { cx = t; cy = t; }                    // u_t^T u_t
-    else if (k == 1) { cx = t; cy = t + 1; }           // u_t^T a_{t+1}
-    else { cx = k - 2; cy = t + 1; }                   // q_i^T a_{t+1}
-  }
-}
-
 template <typename T>
 __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p) {
   extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
   __shared__ float tot[LEAF_MAX_W + 2];            // reduced round vector
-  __shared__ float anorm2[LEAF_MAX_W];             // ||a_k||^2 (breakdown threshold)
-  __shared__ float part[2][GEMV_PARTS][LEAF_MAX_W + 2];     // by round parity
+  __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];        // round 0 / lookahead partials
+  __shared__ float cpart[GEMV_PARTS][4];                    // critical-dot partials
   __shared__ unsigned long long xprev[LEAF_XW_WORDS];      // last seen exchange words
   __shared__ __align__(16) float coef[2][LEAF_MAX_W + 4];   // r_{i,t+2}, i < t, by parity of t
   __shared__ int exS[LEAF_MAX_W];                           // 2||a_j|| < 2^exS[j]
@@ -193,8 +183,6 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   const int nv4 = rows4 / 4;
   const int per = (nv4 + GEMV_PARTS - 1) / GEMV_PARTS;
   const int v_lo = min(nv4, warp * per), v_hi = min(nv4, v_lo + per);
-  // critical-dot mapping: warp = row part, lanes stride the part's rows
-  const int c_lo = v_lo * 4, c_hi = min(rows, v_hi * 4);
 
   // dot(x-col, y-col) over this thread's float4 rows
   auto dot4 = [&](int cx, int cy) {
@@ -210,40 +198,13 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     }
     return s0 + s1;
   };
-  // warp-cooperative dots over the warp's row part (lanes stride rows, xor-trees):
-  // u^T u, u^T a, q^T a in one pass (u = column cu, a = column ca, q = column cq)
-  auto wdot3 = [&](int cu, int ca, int cq, bool three, float& suu, float& sua, float& sqa) {
-    const float* u = sp + cu * LD;
-    const float* a = sp + ca * LD;
-    const float* q = sp + cq * LD;
-    float s0 = 0.f, s1 = 0.f, s2 = 0.f;
-    for (int i = c_lo + lane; i < c_hi; i += 32) {
-      const float uv = u[i];
-      s0 = fmaf(uv, uv, s0);
-      if (three) {
-        const float av = a[i];
-        s1 = fmaf(uv, av, s1);
-        s2 = fmaf(q[i], av, s2);
-      }
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      s0 += __shfl_xor_sync(0xffffffffu, s0, o);
-      s1 += __shfl_xor_sync(0xffffffffu, s1, o);
-      s2 += __shfl_xor_sync(0xffffffffu, s2, o);
-    }
-    suu = s0;
-    sua = s1;
-    sqa = s2;
-  };
-  // round tags of the tagged exchange: unique per (launch, round)
-  // Fixed-point exchange (rounds t >= 1, xmode 2): value k of round t is scaled by 2^e
-  // with e chosen from a bound on |partial| (column norms of round 0), rounded to an
-  // integer |v| <= 2^46 and added with ONE red.add.u64 per CTA to word W[t&1][k] as
-  //     (1 << 56) + (v + 2^46)          -- top byte counts arrivals, low 56 bits sum
+  // Fixed-point exchange (rounds t >= 1): value k of round t is scaled by 2^e with e chosen
+  // from a bound on |partial| (column norms of round 0), rounded to an integer |v| <= 2^41
+  // and added with ONE red.add.u64 per CTA to its word as
+  //     (1 << 53) + (v + 2^41)          -- bits [53,64) count arrivals, low 53 bits sum
   // Integer addition is associative, so the total is independent of arrival order
-  // (deterministic) and exact in fixed point; the word is never reset within a launch:
-  // readers take the difference with the value they saw two rounds earlier.
+  // (deterministic) and exact in fixed point; words are never reset: readers take the
+  // difference with the value they saw at the previous use of the word.
   auto fx_exp = [&](int t, int k) -> int {
     // |partial| <= bound: 4||a_t||^2, 4||a_t|| ||a_{t+1}||, 4||a_{t+1}||, 4||a_{t+2}|| for value
     // classes 0, 1, 2, 3+ (u_t shrinks a_t, ||q_i|| <= 1); 2||a_j|| < 2^exS[j]
@@ -252,52 +213,47 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     if (k == 2) return FX_VBITS - (exS[t + 1] + 1);
     return FX_VBITS - (exS[t + 2] + 1);
   };
-  // publish the L values of part[][] as this CTA's partial vector of round t, arrive
-  auto publish_arrive = [&](int t, int L) {
-    __syncthreads();
-    const bool fx = p.xmode == 2 && t > 0;
-    float* buf = p.partials + (size_t)(t & 1) * (LEAF_MAX_W + 2) * G;
-    // sum of the GEMV_PARTS row-part partials of value k: 4 threads per value, each
-    // adds a quarter of the parts, then a 2-level xor tree (fixed order)
+  // Words of round t: set t mod LEAF_XW_SETS (a round's words are reused only after every
+  // CTA has read them: the lookahead values of round t are added two rounds early), one
+  // 256-byte line per word so that concurrent atomics and polls land in different L2 slices.
+  auto xw_index = [&](int t, int k) -> int { return (t & (LEAF_XW_SETS - 1)) * (LEAF_MAX_W + 2) + k; };
+  auto fx_add = [&](int t, int k, float s) {
+    long long v = __double2ll_rn((double)s * pow2d(fx_exp(t, k)));
+    const long long vb = 1ll << FX_VBITS;
+    v = v > vb ? vb : (v < -vb ? -vb : v);
+    const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
+    const size_t off = (size_t)xw_index(t, k) * LEAF_XW_STRIDE;
+    if (!p.sys) {
+      asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + off), "l"(add) : "memory");
+    } else {
+      // row-sharded run: the same word on every GPU receives every CTA's partial
+      for (int j = 0; j < p.nranks; ++j)
+        asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(p.xw_peers[j] + off), "l"(add)
+                     : "memory");
+    }
+  };
+  // CTA total of values [0, n) of a [GEMV_PARTS][ld] partial buffer: 4 threads per value, each
+  // adds a quarter of the parts, then a 2-level xor tree (fixed order).  Called by all threads;
+  // the returned sum is valid on the thread with (threadIdx.x & 3) == 0 of value threadIdx.x >> 2.
+  auto cta_sum = [&](const float* buf, int ld, int n) -> float {
     const int k = threadIdx.x >> 2, jq = threadIdx.x & 3;
     float s = 0.f;
-    if (k < L) {
+    if (k < n) {
 #pragma unroll
-      for (int q = 0; q < GEMV_PARTS / 4; ++q) s += part[t & 1][jq * (GEMV_PARTS / 4) + q][k];
+      for (int q = 0; q < GEMV_PARTS / 4; ++q) s += buf[(jq * (GEMV_PARTS / 4) + q) * ld + k];
     }
     s += __shfl_xor_sync(0xffffffffu, s, 1);
     s += __shfl_xor_sync(0xffffffffu, s, 2);
-    if (k < L && jq == 0) {
-      if (fx) {
-        long long v = __double2ll_rn((double)s * pow2d(fx_exp(t, k)));
-        const long long vb = 1ll << FX_VBITS;
-        v = v > vb ? vb : (v < -vb ? -vb : v);
-        const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
-        const size_t off = ((size_t)(t & 1) * (LEAF_MAX_W + 2) + k) * LEAF_XW_COPIES + g % LEAF_XW_COPIES;
-        if (!p.sys) {
-          asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + off), "l"(add) : "memory");
-        } else {
-          // row-sharded run: the same word on every GPU receives every CTA's partial
-          for (int j = 0; j < p.nranks; ++j)
-            asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(p.xw_peers[j] + off), "l"(add)
-                         : "memory");
-        }
-      } else {
-        buf[(size_t)k * G + g] = s;
-      }
-    }
-    if (!fx) {
-      __syncthreads();
-      if (threadIdx.x == 0)  // release: orders this CTA's partial stores (bar.sync cumulativity)
-        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.counter) : "memory");
-    }
+    return s;
   };
 
   // Round layout (t >= 1), R19:  [0] u_t.u_t  [1] u_t.a_{t+1}  [2] q_{t-1}.a_{t+1}
-  // [3+i] q_i.a_{t+2} (i <= t-1).  The q_i.a_{t+2} values are published one round ahead, so
-  // after round t every CTA already knows r_{i,t+2} (i <= t-1) and can subtract those
-  // projections from a_{t+2} while round t+1's exchange is in flight; after that exchange
-  // only q_t and q_{t+1} remain to be subtracted (two columns on the critical path).
+  // [3+i] q_i.a_{t+2} (i <= t-1).  Values [3+i], i <= t-2 ("lookahead") only need q's known
+  // two rounds earlier: they are computed AND added to round t's words during round t-2's
+  // exchange.  Round t's critical values [0], [1], [2], [3+t-1] are formed in one pass over
+  // the rows right after round t-1's scalars.  After round t every CTA knows r_{i,t+2}
+  // (i <= t-1) and subtracts those projections from a_{t+2} while round t+1's exchange is in
+  // flight; after that exchange only q_t and q_{t+1} remain to be subtracted.
   auto round_len = [&](int t) -> int {
     if (t == 0) return w + (w > 1 ? 1 : 0);
     if (t == w - 1) return 1;
@@ -335,49 +291,84 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     }
   };
 
-  // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ] ----
+  // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ]: counter barrier + fixed-order gather
+  //      (its column norms fix the fixed-point scales of the later rounds) ----
   // (r0_mode 2: the globally reduced round-0 vector is given in p.r0buf)
   if (p.r0_mode != 2) {
-    const int t = 0;
     const int L = round_len(0);
-    DBG_STAMP(0);
     for (int k = kq; k < L; k += 32) {
-      int cx, cy;
-      round_operands(0, w, k, cx, cy);
-      part[0][warp][k] = dot4(cx, cy);
-    }
-    publish_arrive(0, L);
-  }
-
-  for (int t = 0; t < w; ++t) {
-    const int L = round_len(t);
-    const bool fx = p.xmode == 2 && t > 0;
-    const bool given = t == 0 && p.r0_mode == 2;
-    // ---- wait for round t (counter barrier for round 0 / xmode 0) ----
-    if (!fx && !given && threadIdx.x == 0) {
-      unsigned cv;
-      const unsigned target = (p.xmode == 2 ? 1u : (unsigned)(t + 1)) * (unsigned)G;
-      do {
-        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cv) : "l"(p.counter) : "memory");
-      } while (cv < target);
+      int cx = k < w ? k : 0, cy = k < w ? k : 1;
+      part[warp][k] = dot4(cx, cy);
     }
     __syncthreads();
-    if (fx) {
-      // ---- fixed-point exchange: each value's word is polled by its thread until all
-      //      ranks x G CTAs have added ----
-      // LEAF_XW_COPIES threads per value, one word copy each; the copies' integer totals are
-      // summed with an xor tree (exact, so the order does not matter)
-      const int k = threadIdx.x / LEAF_XW_COPIES, hc = threadIdx.x % LEAF_XW_COPIES;
-      long long total = 0;
-      if (k < L) {
-        const int widx = ((t & 1) * (LEAF_MAX_W + 2) + k) * LEAF_XW_COPIES + hc;
-        const unsigned cnt_h =
-            (unsigned)p.nranks * (unsigned)(G / LEAF_XW_COPIES + (hc < G % LEAF_XW_COPIES ? 1 : 0));
-        const unsigned long long* wp = p.xw + widx;
+    const float s = cta_sum(&part[0][0], LEAF_MAX_W + 2, L);
+    if ((threadIdx.x & 3) == 0 && (threadIdx.x >> 2) < L) p.partials[(size_t)(threadIdx.x >> 2) * G + g] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {  // release: orders this CTA's partial stores (bar.sync cumulativity)
+      asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.counter) : "memory");
+      unsigned cv;
+      do {
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cv) : "l"(p.counter) : "memory");
+      } while (cv < (unsigned)G);
+    }
+    __syncthreads();
+    constexpr int KPW = (LEAF_MAX_W + 2 + LEAF_WARPS - 1) / LEAF_WARPS;
+    constexpr int QMAX = (LEAF_MAX_G + 31) / 32;
+    float v[KPW][QMAX];
+#pragma unroll
+    for (int a = 0; a < KPW; ++a)
+#pragma unroll
+      for (int q = 0; q < QMAX; ++q) {
+        const int k = warp + a * LEAF_WARPS, c = lane + 32 * q;
+        v[a][q] = (k < L && c < G) ? __ldcg(p.partials + (size_t)k * G + c) : 0.0f;
+      }
+#pragma unroll
+    for (int a = 0; a < KPW; ++a) {
+      const int k = warp + a * LEAF_WARPS;
+      if (k >= L) break;                               // warp-uniform
+      float s2 = v[a][0];
+#pragma unroll
+      for (int q = 1; q < QMAX; ++q) s2 += v[a][q];
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+      if (lane == 0) tot[k] = s2;
+    }
+    if (p.r0_mode == 1) {
+      // round-0-only launch of a row-sharded run: hand the local vector to the host
+      // (which all-reduces it across GPUs) and stop
+      __syncthreads();
+      if (g == 0 && threadIdx.x < L) p.r0buf[threadIdx.x] = tot[threadIdx.x];
+      return;
+    }
+  } else if (threadIdx.x < round_len(0)) {
+    tot[threadIdx.x] = p.r0buf[threadIdx.x];
+  }
+  __syncthreads();
+  if (threadIdx.x < w) {
+    const int k = threadIdx.x;
+    const float s = tot[k];
+    int ex;
+    frexpf(2.0f * sqrtf(s), &ex);
+    exS[k] = ex;
+    tauc[k] = (float)p.m_global * u_work * sqrtf(s);
+  }
+  // (the __syncthreads at the top of the round loop publishes exS / tauc)
+
+  for (int t = 0; t < w; ++t) {
+    DBG_STAMP(0);
+    if (t > 0) {
+      // ---- round t's exchange: each value's word is polled by its thread until all
+      //      ranks x G CTAs have added (lookahead words are complete long before) ----
+      const int L = round_len(t);
+      if (threadIdx.x < L) {
+        const int k = threadIdx.x;
+        const int widx = xw_index(t, k);
+        const unsigned cnt = (unsigned)(p.nranks * G);
+        const unsigned long long* wp = p.xw + (size_t)widx * LEAF_XW_STRIDE;
         const unsigned long long prev = xprev[widx];
         unsigned long long now = ld_word(wp, p.sys), d = now - prev;
         long long spins = 0;
-        while ((unsigned)(d >> FX_CNT_SHIFT) != cnt_h) {
+        while ((unsigned)(d >> FX_CNT_SHIFT) != cnt) {
           now = ld_word(wp, p.sys);
           d = now - prev;
           if (++spins > (1ll << 27)) {            // ~seconds: a peer is missing -- fail, never hang
@@ -386,71 +377,14 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           }
         }
         xprev[widx] = now;
-        total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt_h * (1ll << FX_VBITS);
-      }
-#pragma unroll
-      for (int o = 1; o < LEAF_XW_COPIES; o <<= 1) total += __shfl_xor_sync(0xffffffffu, total, o);
-      if (k < L && hc == 0) {
+        const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
         const float val = (float)((double)total * pow2d(-fx_exp(t, k)));
         tot[k] = val;
         if (k >= 3) coef[t & 1][k - 3] = val;
       }
-    } else if (given) {
-      if (threadIdx.x < L) {
-        const int k = threadIdx.x;
-        const float s = p.r0buf[k];
-        tot[k] = s;
-        if (k < w) {
-          anorm2[k] = s;
-          int ex;
-          frexpf(2.0f * sqrtf(s), &ex);
-          exS[k] = ex;
-          tauc[k] = (float)p.m_global * u_work * sqrtf(s);
-        }
-      }
-    } else {
-      // ---- gather round t's G partials per value, fixed-order sum ----
-      constexpr int KPW = (LEAF_MAX_W + 2 + LEAF_WARPS - 1) / LEAF_WARPS;
-      constexpr int QMAX = (LEAF_MAX_G + 31) / 32;
-      const float* buf = p.partials + (size_t)(t & 1) * (LEAF_MAX_W + 2) * G;
-      float v[KPW][QMAX];
-#pragma unroll
-      for (int a = 0; a < KPW; ++a)
-#pragma unroll
-        for (int q = 0; q < QMAX; ++q) {
-          const int k = warp + a * LEAF_WARPS, c = lane + 32 * q;
-          v[a][q] = (k < L && c < G) ? __ldcg(buf + (size_t)k * G + c) : 0.0f;
-        }
-#pragma unroll
-      for (int a = 0; a < KPW; ++a) {
-        const int k = warp + a * LEAF_WARPS;
-        if (k >= L) break;                               // warp-uniform
-        float s = v[a][0];
-#pragma unroll
-        for (int q = 1; q < QMAX; ++q) s += v[a][q];
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-        if (lane == 0) {
-          tot[k] = s;
-          if (t > 0 && k >= 3) coef[t & 1][k - 3] = s;
-          if (t == 0 && k < w) {
-            anorm2[k] = s;
-            int ex;
-            frexpf(2.0f * sqrtf(s), &ex);
-            exS[k] = ex;
-            tauc[k] = (float)p.m_global * u_work * sqrtf(s);
-          }
-        }
-      }
     }
     __syncthreads();
-    DBG_STAMP(2);
-    if (t == 0 && p.r0_mode == 1) {
-      // round-0-only launch of a row-sharded run: hand the local vector to the host
-      // (which all-reduces it across GPUs) and stop
-      if (g == 0 && threadIdx.x < L) p.r0buf[threadIdx.x] = tot[threadIdx.x];
-      return;
-    }
+    DBG_STAMP(1);
     // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{t,t+1}, r_{t-1,t+1} ----
     const bool more = t + 1 < w;
     const float uu = tot[0];
@@ -474,94 +408,73 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       }
       if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
     }
-    DBG_STAMP(5);
-    // ---- q_t = u_t / r_tt (stored rounded); u_{t+1} = w_{t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1}
-    //      where w_{t+1} = a_{t+1} - sum_{i<=t-2} q_i r_{i,t+1} was formed during round t ----
+    DBG_STAMP(2);
+    // ---- one pass over the rows (thread = row):  q_t = u_t / r_tt (stored rounded),
+    //      u_{t+1} = w_{t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1}, where w_{t+1} = a_{t+1} -
+    //      sum_{i<=t-2} q_i r_{i,t+1} was formed during round t; and round t+1's critical
+    //      dots u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2}, q_t.a_{t+2}, q_t.a_{t+3} ----
+    const bool h2 = t + 2 < w, h3 = t + 3 < w;
     {
       float* ut = sp + t * LD;
-      float* an = sp + (t + 1) * LD;
+      float* an = sp + (more ? t + 1 : t) * LD;
       const float* qp = sp + (t >= 1 ? t - 1 : 0) * LD;
-      for (int v = threadIdx.x; v < ((p.skip & 1) ? 0 : nv4); v += LEAF_THREADS) {
-        float4 q4 = reinterpret_cast<float4*>(ut)[v];
-        q4.x *= inv; q4.y *= inv; q4.z *= inv; q4.w *= inv;
-        reinterpret_cast<float4*>(ut)[v] = q4;
-        {
-          const int i0 = 4 * v;
-          T* dst = P + r0 + i0 + (int64_t)t * p.ldp;
-          if (p.vec_ok && i0 + 4 <= rows) {
-            store4<T>(dst, q4);
-          } else {
-            const float qv[4] = {q4.x, q4.y, q4.z, q4.w};
-            for (int e = 0; e < 4 && i0 + e < rows; ++e) dst[e] = Elem<T>::store(qv[e]);
+      const float* a2 = sp + (h2 ? t + 2 : t) * LD;
+      const float* a3 = sp + (h3 ? t + 3 : t) * LD;
+      T* qdst = P + r0 + (int64_t)t * p.ldp;
+      float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+      for (int r = threadIdx.x; r < rows; r += LEAF_THREADS) {
+        const float q = ut[r] * inv;
+        ut[r] = q;
+        qdst[r] = Elem<T>::store(q);
+        if (more) {
+          float av = an[r];
+          if (t >= 1) av = fmaf(-qp[r], cq, av);
+          av = fmaf(-q, ct, av);
+          an[r] = av;
+          s0 = fmaf(av, av, s0);
+          if (h2) {
+            const float a2v = a2[r];
+            s1 = fmaf(av, a2v, s1);
+            s2 = fmaf(q, a2v, s2);
+            if (h3) s3 = fmaf(q, a3[r], s3);
           }
         }
-        if (more) {
-          float4 av = reinterpret_cast<float4*>(an)[v];
-          if (t >= 1) {
-            const float4 qm = reinterpret_cast<const float4*>(qp)[v];
-            av.x = fmaf(-qm.x, cq, av.x); av.y = fmaf(-qm.y, cq, av.y);
-            av.z = fmaf(-qm.z, cq, av.z); av.w = fmaf(-qm.w, cq, av.w);
-          }
-          av.x = fmaf(-q4.x, ct, av.x); av.y = fmaf(-q4.y, ct, av.y);
-          av.z = fmaf(-q4.z, ct, av.z); av.w = fmaf(-q4.w, ct, av.w);
-          reinterpret_cast<float4*>(an)[v] = av;
+      }
+      if (more) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+          s0 += __shfl_xor_sync(0xffffffffu, s0, o);
+          s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+          s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+          s3 += __shfl_xor_sync(0xffffffffu, s3, o);
+        }
+        if (lane == 0) {
+          cpart[warp][0] = s0;
+          cpart[warp][1] = s1;
+          cpart[warp][2] = s2;
+          cpart[warp][3] = s3;
         }
       }
     }
     __syncthreads();
-    DBG_STAMP(4);
+    DBG_STAMP(3);
     if (!more) break;
-    // ---- round t+1: the dots that needed round t -- u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2},
-    //      q_t.a_{t+2}, q_t.a_{t+3} -- then publish + arrive ----
+    // ---- publish round t+1's critical values: [0], [1], [2] and [3 + t] ----
     {
-      const int t1 = t + 1;
-      const int L1 = round_len(t1);
-      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8] = clock64();
-      const bool h2 = t + 2 < w, h3 = t + 3 < w;
-      const float* u = sp + t1 * LD;
-      const float* qv = sp + t * LD;
-      const float* a2 = sp + (h2 ? t + 2 : t1) * LD;
-      const float* a3 = sp + (h3 ? t + 3 : t1) * LD;
-      float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
-      if (!(p.skip & 4)) {
-        for (int i = c_lo + lane; i < c_hi; i += 32) {
-          const float uv = u[i];
-          s0 = fmaf(uv, uv, s0);
-          if (h2) {
-            const float av = a2[i], qq = qv[i];
-            s1 = fmaf(uv, av, s1);
-            s2 = fmaf(qq, av, s2);
-            if (h3) s3 = fmaf(qq, a3[i], s3);
-          }
-        }
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        s0 += __shfl_xor_sync(0xffffffffu, s0, o);
-        s1 += __shfl_xor_sync(0xffffffffu, s1, o);
-        s2 += __shfl_xor_sync(0xffffffffu, s2, o);
-        s3 += __shfl_xor_sync(0xffffffffu, s3, o);
-      }
-      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 6] = clock64();
-      if (lane == 0) {
-        float* pw = part[t1 & 1][warp];
-        pw[0] = s0;
-        if (h2) {
-          pw[1] = s1;
-          pw[2] = s2;
-          if (h3) pw[3 + t] = s3;                        // q_t.a_{t1+2}: index 3 + (t1 - 1)
-        }
-      }
-      publish_arrive(t1, L1);
-      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)t1 * 8 + 7] = clock64();
+      const int n = !h2 ? 1 : (!h3 ? 3 : 4);
+      const float s = cta_sum(&cpart[0][0], 4, n);
+      const int c = threadIdx.x >> 2;
+      if ((threadIdx.x & 3) == 0 && c < n) fx_add(t + 1, c < 3 ? c : 3 + t, s);
     }
+    DBG_STAMP(4);
     // ---- while round t+1's exchange is in flight:
-    //      (a) lookahead for round t+2: q_i.a_{t+4}, i <= t  (index 3 + i)
+    //      (a) round t+2's lookahead values q_i.a_{t+4}, i <= t (index 3 + i), computed and
+    //          added to round t+2's words now;
     //      (b) w_{t+2} = a_{t+2} - sum_{i <= t-1} q_i r_{i,t+2}  (coefficients from round t) ----
-    if (t + 4 < w && !(p.skip & 2)) {
+    if (t + 4 < w) {
       const int cnt = t + 1;                              // i in [0, t]
       const bool ha = kq < cnt, hb = kq + 32 < cnt;
-      if (ha) {
+      if (ha && !(p.skip & 2)) {
         const float4* y = reinterpret_cast<const float4*>(sp + (t + 4) * LD);
         const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
         const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
@@ -580,13 +493,17 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
             b1 = fmaf(b.w, yy.w, b1);
           }
         }
-        float* pw = part[t & 1][warp];                    // round t+2 has the parity of t
-        pw[3 + kq] = a0 + a1;
-        if (hb) pw[3 + kq + 32] = b0 + b1;
+        part[warp][kq] = a0 + a1;
+        if (hb) part[warp][kq + 32] = b0 + b1;
       }
+      __syncthreads();
+      const float s = cta_sum(&part[0][0], LEAF_MAX_W + 2, cnt);
+      const int i = threadIdx.x >> 2;
+      if ((threadIdx.x & 3) == 0 && i < cnt) fx_add(t + 2, 3 + i, s);
     }
-    if (t + 2 < w && t >= 1) project_out(t + 2, t, coef[t & 1]);
-    if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)(t + 1) * 8 + 1] = clock64();
+    DBG_STAMP(5);
+    if (t + 2 < w && t >= 1 && !(p.skip & 4)) project_out(t + 2, t, coef[t & 1]);
+    DBG_STAMP(6);
   }
   // every CTA ends with the same last-seen words; CTA 0 persists them for the next launch
   if (g == 0)

@@ -326,8 +326,6 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   static const bool dbg = getenv("RGSQR_LEAF_DEBUG") != nullptr;
   static long long* dbg_buf = nullptr;
   p.counter = c->d_counter;
-  static const int xmode = getenv("RGSQR_LEAF_XMODE") ? atoi(getenv("RGSQR_LEAF_XMODE")) : 2;
-  p.xmode = xmode;
   p.epoch = ++c->leaf_epoch;
   p.xw = c->d_xw;
   p.xw_peers = c->d_peers;
@@ -344,7 +342,6 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   p.skip = dbg ? skip : 0;
   p.breakdown = c->d_breakdown;
   p.col_offset = col_offset;
-  if (c->nccl_comm && p.xmode != 2) return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: sharded runs need xmode 2");
   auto launch = [&](const LeafParams& q) -> cudaError_t {
     switch (prec) {
       case RGSQR_FP16: return launch_leaf<__half>(q, G, st);
@@ -381,10 +378,10 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
     long long hb[8 * LEAF_MAX_W];
     cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 8 * w, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
-    // stamps of round t: 0 critical start, 6 after critical dots, 7 after publish, 1 after the
-    // overlapped lookahead + precompute, 2 after the exchange, 5 after scalars, 4 after update
-    const int order[7] = {0, 6, 7, 1, 2, 5, 4};
-    const char* names[6] = {"crit", "publish", "overlap", "exchange", "scalars", "update"};
+    // stamps of iteration t: 0 start, 1 round t exchanged, 2 scalars, 3 row pass (q_t, u_{t+1},
+    // round t+1's critical dots), 4 critical values added, 5 lookahead dots added, 6 projection
+    const int order[7] = {0, 1, 2, 3, 4, 5, 6};
+    const char* names[6] = {"exchange", "scalars", "rowpass", "publish", "lookahead", "project"};
     double ph[6] = {0};
     int cnt = 0;
     for (int t = 1; t + 1 < w; ++t, ++cnt)
