@@ -10,7 +10,8 @@ arithmetic.
 Contents (each function cites the PAPER.md passage it follows):
 
 * ``cgs.py``    -- O1 column CGS (Eq. 1), O2 CGS2, O3 recursive CGS (Eq. 2),
-                   O4 blocked CGS (section 3.1.2), O5 precision-emulating recursive CGS.
+                   O4 blocked CGS (section 3.1.2), O5 precision-emulating recursive CGS,
+                   O6 recursive CGS2 (reorthogonalized).
 * ``checks.py`` -- backward error, orthogonality loss, triangularity, R error,
                    Gram-Cholesky reference R for large inputs.
 * ``model.py``  -- recursion shapes, flop count, the paper's data-movement models.
@@ -22,7 +23,7 @@ paper's printed shape / byte formulas (tests/golden/).  Parity status per
 function is listed in DESIGN.md section 4 ("parity unpinned" where applicable:
 O5 -- an emulation whose only pin is agreement with O3 in the fp64 limit).
 """
-from .cgs import cgs, cgs2, rgs, blocked_cgs, rgs_emulated, QRResult  # noqa: F401
+from .cgs import cgs, cgs2, rgs, rgs2, blocked_cgs, rgs_emulated, QRResult  # noqa: F401
 from .checks import (backward_error, orthogonality, r_rel_error, is_upper_triangular,  # noqa: F401
                      gram_cholesky_r)
 from . import model  # noqa: F401

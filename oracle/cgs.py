@@ -136,6 +136,45 @@ def blocked_cgs(X: np.ndarray, b: int) -> QRResult:
 
 
 # ---------------------------------------------------------------------------------
+# O6: recursive CGS2 -- Eq. (2) with every CGS step applied twice (SURVEY.md 8 f3,
+#     DESIGN.md reading R22)
+# ---------------------------------------------------------------------------------
+def rgs2(X: np.ndarray, leaf: int = 32) -> QRResult:
+    """O6. The recursion of Eq. (2) with reorthogonalization ("CGS2",
+    the stable relative of CGS):
+      node:  R12 = Q1^T A2;  A2 -= Q1 R12;  S = Q1^T A2;  A2 -= Q1 S;  R12 += S
+      leaf:  [Q', R'] = CGS(panel) (Eq. 1);  [Q, S] = CGS(Q');  R = S R'
+    In exact arithmetic S = 0 at the nodes and S = I at the leaves, so O6 = O3."""
+    X = np.array(X, dtype=np.float64, order="F", copy=True)
+    n = X.shape[1]
+    R = np.zeros((n, n), order="F")
+    brk = [-1]
+
+    def rec(c0: int, c1: int):
+        w = c1 - c0
+        if w <= leaf:
+            first = cgs(X[:, c0:c1])                  # Q' R'
+            second = cgs(first.Q)                     # Q' = Q S
+            X[:, c0:c1] = second.Q
+            R[c0:c1, c0:c1] = second.R @ first.R      # R = S R'
+            b = first.breakdown if first.breakdown >= 0 else second.breakdown
+            if b >= 0 and brk[0] < 0:
+                brk[0] = c0 + b
+            return
+        h = c0 + w // 2
+        rec(c0, h)
+        R12 = X[:, c0:h].T @ X[:, h:c1]               # first projection
+        X[:, h:c1] -= X[:, c0:h] @ R12
+        S = X[:, c0:h].T @ X[:, h:c1]                 # reorthogonalization
+        X[:, h:c1] -= X[:, c0:h] @ S
+        R[c0:h, h:c1] = R12 + S
+        rec(h, c1)
+
+    rec(0, n)
+    return QRResult(X, R, brk[0])
+
+
+# ---------------------------------------------------------------------------------
 # O5: precision-emulating recursive CGS (predicts the algorithmic error level)
 # ---------------------------------------------------------------------------------
 def _round_bf16(x: np.ndarray) -> np.ndarray:
@@ -178,27 +217,43 @@ def _mm(A, B, mode):
     return A @ B                                      # 16-bit operands are exact in fp32
 
 
-def rgs_emulated(X: np.ndarray, mode: str, leaf: int = 32) -> QRResult:
+def rgs_emulated(X: np.ndarray, mode: str, leaf: int = 32, reorth: bool = False) -> QRResult:
     """O5. O3 with the GPU's storage/operand rounding emulated (R5, R8,
     R9): Q and A2' stored in the storage format, R12 rounded to it as an MMA
     operand, fp32 accumulation, leaf CGS in fp32.  An error-level predictor,
-    not a bitwise model (summation order differs from the GPU)."""
+    not a bitwise model (summation order differs from the GPU).  reorth=True
+    emulates O6 (CGS2) the same way."""
     Xs = _store(np.asarray(X, dtype=np.float32), mode).copy(order="F")
     m, n = Xs.shape
     R = np.zeros((n, n), dtype=np.float64)
 
-    def leaf_cgs(c0, c1):
-        P = Xs[:, c0:c1].astype(np.float32)
+    def panel_cgs(P):
+        P = P.astype(np.float32)
         Q = np.zeros_like(P)
-        for j in range(c1 - c0):
+        Rp = np.zeros((P.shape[1], P.shape[1]), dtype=np.float64)
+        for j in range(P.shape[1]):
             a = P[:, j]
             r = Q[:, :j].T @ a
             u = a - Q[:, :j] @ r
             rjj = np.float32(np.sqrt(np.float32(u @ u)))
             Q[:, j] = _store(u / rjj, mode)
-            R[c0:c0 + j, c0 + j] = r
-            R[c0 + j, c0 + j] = rjj
+            Rp[:j, j] = r
+            Rp[j, j] = rjj
+        return Q, Rp
+
+    def leaf_cgs(c0, c1):
+        Q, Rp = panel_cgs(Xs[:, c0:c1])
+        if reorth:
+            Q, S = panel_cgs(Q)
+            Rp = (S.astype(np.float32) @ Rp.astype(np.float32)).astype(np.float64)
+        R[c0:c1, c0:c1] = Rp
         Xs[:, c0:c1] = Q
+
+    def project(c0, h, c1):
+        R12 = _mm(Xs[:, c0:h].T, Xs[:, h:c1], mode)
+        R12op = _store(R12, mode)
+        Xs[:, h:c1] = _store(Xs[:, h:c1] - _mm(Xs[:, c0:h], R12op, mode), mode)
+        return R12
 
     def rec(c0, c1):
         w = c1 - c0
@@ -207,10 +262,10 @@ def rgs_emulated(X: np.ndarray, mode: str, leaf: int = 32) -> QRResult:
             return
         h = c0 + w // 2
         rec(c0, h)
-        R12 = _mm(Xs[:, c0:h].T, Xs[:, h:c1], mode)
+        R12 = project(c0, h, c1)
+        if reorth:
+            R12 = (R12 + project(c0, h, c1)).astype(np.float32)
         R[c0:h, h:c1] = R12
-        R12op = _store(R12, mode)
-        Xs[:, h:c1] = _store(Xs[:, h:c1] - _mm(Xs[:, c0:h], R12op, mode), mode)
         rec(h, c1)
 
     rec(0, n)

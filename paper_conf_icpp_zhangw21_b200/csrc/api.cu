@@ -400,6 +400,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_LEAF_CTAS: return &o.leaf_ctas;
     case RGSQR_OPT_SPLITK: return &o.splitk;
     case RGSQR_OPT_PROFILE: return &o.profile;
+    case RGSQR_OPT_REORTH: return &o.reorth;
   }
   return nullptr;
 }
@@ -415,6 +416,7 @@ int rgsqr_set_option(rgsqr_handle h, int key, int64_t value) {
     case RGSQR_OPT_TILE_ROWS_MAX: if (value < 128 || value % 128) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_RING_DEPTH: if (value < 2 || value > 16) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_ALGO: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_REORTH: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_BLOCK_COLS: if (value < 8) return RGSQR_ERR_INVALID_ARG; break;
     default: if (value < 0) return RGSQR_ERR_INVALID_ARG;
   }

@@ -26,6 +26,7 @@ struct Options {
   int64_t leaf_ctas = 0;
   int64_t splitk = 0;
   int64_t profile = 0;
+  int64_t reorth = 0;        // CGS2 (RGSQR_OPT_REORTH)
 };
 
 struct KernSeg {

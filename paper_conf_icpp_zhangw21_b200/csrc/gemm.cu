@@ -544,6 +544,29 @@ template cudaError_t launch_copy_cast<__nv_bfloat16>(const float*, int64_t, floa
 template cudaError_t launch_copy_cast<float>(const float*, int64_t, float*, int64_t, float*, int64_t, int64_t,
                                              int64_t, cudaStream_t);
 
+// CGS2 leaf: R <- S R (both w x w upper triangular, column-major), one CTA, fixed-order sums.
+__global__ void trmm_upper_kernel(const float* __restrict__ S, int64_t lds, float* R, int64_t ldr, int w) {
+  __shared__ float sS[LEAF_MAX_W * LEAF_MAX_W], sR[LEAF_MAX_W * LEAF_MAX_W];
+  for (int idx = threadIdx.x; idx < w * w; idx += blockDim.x) {
+    const int i = idx % w, j = idx / w;
+    sS[idx] = S[i + j * lds];
+    sR[idx] = R[i + j * ldr];
+  }
+  __syncthreads();
+  for (int idx = threadIdx.x; idx < w * w; idx += blockDim.x) {
+    const int i = idx % w, j = idx / w;
+    float acc = 0.0f;
+    for (int k = i; k <= j; ++k) acc = fmaf(sS[i + k * w], sR[k + j * w], acc);
+    R[i + j * ldr] = i <= j ? acc : 0.0f;
+  }
+}
+
+cudaError_t launch_trmm_upper(const float* S, int64_t lds, float* R, int64_t ldr, int w, cudaStream_t st) {
+  if (w < 1 || w > LEAF_MAX_W) return cudaErrorInvalidValue;
+  trmm_upper_kernel<<<1, 512, 0, st>>>(S, lds, R, ldr, w);
+  return cudaGetLastError();
+}
+
 template cudaError_t launch_gemm<__half>(bool, int, const CUtensorMap&, const CUtensorMap&,
                                          const GemmParams&, int, cudaStream_t);
 template cudaError_t launch_gemm<__nv_bfloat16>(bool, int, const CUtensorMap&, const CUtensorMap&,

@@ -95,4 +95,8 @@ template <typename T>
 cudaError_t launch_copy_cast(const float* src, int64_t lds, float* dst_f, int64_t ldf, T* dst_op, int64_t ldo,
                              int64_t M, int64_t N, cudaStream_t st);
 
+// R <- S R for upper-triangular w x w blocks (w <= LEAF_MAX_W), column-major, in place in R:
+// the leaf's second CGS pass (CGS2) factors Q' = Q S, so A = Q' R' = Q (S R').
+cudaError_t launch_trmm_upper(const float* S, int64_t lds, float* R, int64_t ldr, int w, cudaStream_t st);
+
 }  // namespace rgsqr

@@ -54,6 +54,10 @@ __device__ __forceinline__ unsigned long long ld_word(const unsigned long long* 
 static constexpr int FX_CNT_SHIFT = 53;
 static constexpr int FX_VBITS = 41;
 
+// named barriers: the reducing warp waits for all threads, the others only arrive
+__device__ __forceinline__ void bar_sync_n(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+__device__ __forceinline__ void bar_arrive_n(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
 // exact power of two as a double (|e| < 1000)
 __device__ __forceinline__ double pow2d(int e) { return __hiloint2double((1023 + e) << 20, 0); }
 
@@ -133,11 +137,11 @@ __device__ __forceinline__ void store4<float>(float* dst, float4 v) {
 template <typename T>
 __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p) {
   extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
-  __shared__ float tot[LEAF_MAX_W + 2];            // reduced round vector
+  __shared__ float tot[2][LEAF_MAX_W + 2];         // reduced round vector, by parity of the round
   __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];        // round 0 / lookahead partials
   __shared__ float cpart[GEMV_PARTS][4];                    // critical-dot partials
   __shared__ unsigned long long xprev[LEAF_XW_WORDS];      // last seen exchange words
-  __shared__ __align__(16) float coef[2][LEAF_MAX_W + 4];   // r_{i,t+2}, i < t, by parity of t
+  __shared__ __align__(16) float coef[3][LEAF_MAX_W + 4];   // r_{i,t+2}, i < t, by t mod 3
   __shared__ int exS[LEAF_MAX_W];                           // 2||a_j|| < 2^exS[j]
   __shared__ float tauc[LEAF_MAX_W];                        // breakdown thresholds
   // last-seen exchange words persist across launches (words are never reset, see fx_exp)
@@ -232,6 +236,20 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
                      : "memory");
     }
   };
+  auto fx_add_scaled = [&](int t, int k, float s, double scale) {
+    long long v = __double2ll_rn((double)s * scale);
+    const long long vb = 1ll << FX_VBITS;
+    v = v > vb ? vb : (v < -vb ? -vb : v);
+    const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
+    const size_t off = (size_t)xw_index(t, k) * LEAF_XW_STRIDE;
+    if (!p.sys) {
+      asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + off), "l"(add) : "memory");
+    } else {
+      for (int j = 0; j < p.nranks; ++j)
+        asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(p.xw_peers[j] + off), "l"(add)
+                     : "memory");
+    }
+  };
   // CTA total of values [0, n) of a [GEMV_PARTS][ld] partial buffer: 4 threads per value, each
   // adds a quarter of the parts, then a 2-level xor tree (fixed order).  Called by all threads;
   // the returned sum is valid on the thread with (threadIdx.x & 3) == 0 of value threadIdx.x >> 2.
@@ -260,37 +278,6 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     if (t == w - 2) return 3;
     return t + 3;
   };
-  // col -= sum_{i < cnt} q_i * cf[i]   (4 rows per thread, fixed order of i within two sums)
-  auto project_out = [&](int col, int cnt, const float* cf) {
-    float* an = sp + col * LD;
-    for (int v = threadIdx.x; v < nv4; v += LEAF_THREADS) {
-      float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0;
-      int k = 0;
-      for (; k + 4 <= cnt; k += 4) {
-        const float4 c = reinterpret_cast<const float4*>(cf)[k >> 2];
-        const float4 x0 = reinterpret_cast<const float4*>(sp + (k + 0) * LD)[v];
-        const float4 x1 = reinterpret_cast<const float4*>(sp + (k + 1) * LD)[v];
-        const float4 x2 = reinterpret_cast<const float4*>(sp + (k + 2) * LD)[v];
-        const float4 x3 = reinterpret_cast<const float4*>(sp + (k + 3) * LD)[v];
-        a0.x = fmaf(x0.x, c.x, a0.x); a0.y = fmaf(x0.y, c.x, a0.y); a0.z = fmaf(x0.z, c.x, a0.z); a0.w = fmaf(x0.w, c.x, a0.w);
-        a1.x = fmaf(x1.x, c.y, a1.x); a1.y = fmaf(x1.y, c.y, a1.y); a1.z = fmaf(x1.z, c.y, a1.z); a1.w = fmaf(x1.w, c.y, a1.w);
-        a0.x = fmaf(x2.x, c.z, a0.x); a0.y = fmaf(x2.y, c.z, a0.y); a0.z = fmaf(x2.z, c.z, a0.z); a0.w = fmaf(x2.w, c.z, a0.w);
-        a1.x = fmaf(x3.x, c.w, a1.x); a1.y = fmaf(x3.y, c.w, a1.y); a1.z = fmaf(x3.z, c.w, a1.z); a1.w = fmaf(x3.w, c.w, a1.w);
-      }
-      for (; k < cnt; ++k) {
-        const float c = cf[k];
-        const float4 x = reinterpret_cast<const float4*>(sp + k * LD)[v];
-        a0.x = fmaf(x.x, c, a0.x); a0.y = fmaf(x.y, c, a0.y); a0.z = fmaf(x.z, c, a0.z); a0.w = fmaf(x.w, c, a0.w);
-      }
-      float4 av = reinterpret_cast<float4*>(an)[v];
-      av.x -= a0.x + a1.x;
-      av.y -= a0.y + a1.y;
-      av.z -= a0.z + a1.z;
-      av.w -= a0.w + a1.w;
-      reinterpret_cast<float4*>(an)[v] = av;
-    }
-  };
-
   // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ]: counter barrier + fixed-order gather
   //      (its column norms fix the fixed-point scales of the later rounds) ----
   // (r0_mode 2: the globally reduced round-0 vector is given in p.r0buf)
@@ -331,22 +318,22 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       for (int q = 1; q < QMAX; ++q) s2 += v[a][q];
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) s2 += __shfl_xor_sync(0xffffffffu, s2, o);
-      if (lane == 0) tot[k] = s2;
+      if (lane == 0) tot[0][k] = s2;
     }
     if (p.r0_mode == 1) {
       // round-0-only launch of a row-sharded run: hand the local vector to the host
       // (which all-reduces it across GPUs) and stop
       __syncthreads();
-      if (g == 0 && threadIdx.x < L) p.r0buf[threadIdx.x] = tot[threadIdx.x];
+      if (g == 0 && threadIdx.x < L) p.r0buf[threadIdx.x] = tot[0][threadIdx.x];
       return;
     }
   } else if (threadIdx.x < round_len(0)) {
-    tot[threadIdx.x] = p.r0buf[threadIdx.x];
+    tot[0][threadIdx.x] = p.r0buf[threadIdx.x];
   }
   __syncthreads();
   if (threadIdx.x < w) {
     const int k = threadIdx.x;
-    const float s = tot[k];
+    const float s = tot[0][k];
     int ex;
     frexpf(2.0f * sqrtf(s), &ex);
     exS[k] = ex;
@@ -354,6 +341,17 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   }
   // (the __syncthreads at the top of the round loop publishes exS / tauc)
 
+  // Warp roles inside a round (all warps own rows: thread-per-row in the row pass and the
+  // projection, warp-per-32-row-block in the lookahead GEMV, so every phase of warp v only
+  // touches the rows [32v + 512k, 32v + 512k + 32) it wrote itself and needs no CTA barrier):
+  //   CRIT_W reduces the critical partials (named barrier 1, the other warps only arrive)
+  //   LA_W   reduces the lookahead partials (named barrier 2)
+  // Only the exchange result is broadcast with a full barrier.  tot[] is double- and coef[]
+  // triple-buffered because a warp may run one round ahead of a slower one.
+  constexpr int CRIT_W = LEAF_WARPS - 1, LA_W = LEAF_WARPS - 2;
+  const int row_warps = rows >= LEAF_THREADS ? LEAF_WARPS : (rows + 31) / 32;   // warps owning rows
+  unsigned long long pre = 0;                      // prefetched exchange word (pollers)
+  bool have_pre = false;
   for (int t = 0; t < w; ++t) {
     DBG_STAMP(0);
     if (t > 0) {
@@ -366,7 +364,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         const unsigned cnt = (unsigned)(p.nranks * G);
         const unsigned long long* wp = p.xw + (size_t)widx * LEAF_XW_STRIDE;
         const unsigned long long prev = xprev[widx];
-        unsigned long long now = ld_word(wp, p.sys), d = now - prev;
+        unsigned long long now = have_pre ? pre : ld_word(wp, p.sys), d = now - prev;
         long long spins = 0;
         while ((unsigned)(d >> FX_CNT_SHIFT) != cnt) {
           now = ld_word(wp, p.sys);
@@ -379,17 +377,18 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         xprev[widx] = now;
         const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
         const float val = (float)((double)total * pow2d(-fx_exp(t, k)));
-        tot[k] = val;
-        if (k >= 3) coef[t & 1][k - 3] = val;
+        tot[t & 1][k] = val;
+        if (k >= 3) coef[t % 3][k - 3] = val;
       }
     }
     __syncthreads();
     DBG_STAMP(1);
     // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{t,t+1}, r_{t-1,t+1} ----
     const bool more = t + 1 < w;
-    const float uu = tot[0];
-    const float ua = (t == 0) ? ((w > 1) ? tot[w] : 0.0f) : (more ? tot[1] : 0.0f);
-    const float cq = (t >= 1 && more) ? tot[2] : 0.0f;   // r_{t-1,t+1} = q_{t-1}^T a_{t+1}
+    const float* tt = tot[t & 1];
+    const float uu = tt[0];
+    const float ua = (t == 0) ? ((w > 1) ? tt[w] : 0.0f) : (more ? tt[1] : 0.0f);
+    const float cq = (t >= 1 && more) ? tt[2] : 0.0f;    // r_{t-1,t+1} = q_{t-1}^T a_{t+1}
     float rtt = sqrtf(uu);
     const float tau = tauc[t];
     const bool bad = !(rtt > tau) || !isfinite(rtt);
@@ -403,17 +402,18 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       }
       if (more && threadIdx.x <= t) {
         const int i = threadIdx.x;
-        const float r = (i == t) ? ct : (i == t - 1) ? cq : coef[(t - 1) & 1][i];   // i <= t-2: round t-1
+        const float r = (i == t) ? ct : (i == t - 1) ? cq : coef[(t + 2) % 3][i];   // i <= t-2: round t-1
         p.R[i + (int64_t)(t + 1) * p.ldr] = r;
       }
       if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
     }
     DBG_STAMP(2);
-    // ---- one pass over the rows (thread = row):  q_t = u_t / r_tt (stored rounded),
+    // ---- one pass over this thread's rows:  q_t = u_t / r_tt (stored rounded),
     //      u_{t+1} = w_{t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1}, where w_{t+1} = a_{t+1} -
-    //      sum_{i<=t-2} q_i r_{i,t+1} was formed during round t; and round t+1's critical
+    //      sum_{i<=t-2} q_i r_{i,t+1} was formed during round t-1; and round t+1's critical
     //      dots u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2}, q_t.a_{t+2}, q_t.a_{t+3} ----
     const bool h2 = t + 2 < w, h3 = t + 3 < w;
+    float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
     {
       float* ut = sp + t * LD;
       float* an = sp + (more ? t + 1 : t) * LD;
@@ -421,88 +421,150 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       const float* a2 = sp + (h2 ? t + 2 : t) * LD;
       const float* a3 = sp + (h3 ? t + 3 : t) * LD;
       T* qdst = P + r0 + (int64_t)t * p.ldp;
-      float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
       for (int r = threadIdx.x; r < rows; r += LEAF_THREADS) {
-        const float q = ut[r] * inv;
+        // all loads first (the columns are distinct whenever their values are used)
+        const float uv = ut[r], av0 = an[r], qpv = qp[r], a2v = a2[r], a3v = a3[r];
+        const float q = uv * inv;
         ut[r] = q;
         qdst[r] = Elem<T>::store(q);
         if (more) {
-          float av = an[r];
-          if (t >= 1) av = fmaf(-qp[r], cq, av);
+          float av = av0;
+          if (t >= 1) av = fmaf(-qpv, cq, av);
           av = fmaf(-q, ct, av);
           an[r] = av;
           s0 = fmaf(av, av, s0);
           if (h2) {
-            const float a2v = a2[r];
             s1 = fmaf(av, a2v, s1);
             s2 = fmaf(q, a2v, s2);
-            if (h3) s3 = fmaf(q, a3[r], s3);
+            if (h3) s3 = fmaf(q, a3v, s3);
           }
         }
       }
-      if (more) {
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-          s0 += __shfl_xor_sync(0xffffffffu, s0, o);
-          s1 += __shfl_xor_sync(0xffffffffu, s1, o);
-          s2 += __shfl_xor_sync(0xffffffffu, s2, o);
-          s3 += __shfl_xor_sync(0xffffffffu, s3, o);
-        }
-        if (lane == 0) {
-          cpart[warp][0] = s0;
-          cpart[warp][1] = s1;
-          cpart[warp][2] = s2;
-          cpart[warp][3] = s3;
-        }
-      }
     }
-    __syncthreads();
-    DBG_STAMP(3);
     if (!more) break;
-    // ---- publish round t+1's critical values: [0], [1], [2] and [3 + t] ----
+    // the critical reducer's lane 8c will add value c of round t+1: its fixed-point scale now
+    double crit_scale = 0.0;
+    if (warp == CRIT_W && (lane & 7) == 0) {
+      const int c = lane >> 3;
+      crit_scale = pow2d(fx_exp(t + 1, c < 3 ? c : 3 + t));
+    }
+    // warp sums of the 4 critical values by a transposing butterfly (6 shuffles): afterwards
+    // lane 8k holds value k (fixed tree per value)
     {
+      const bool b16 = lane & 16, b8 = lane & 8;
+      float k0 = b16 ? s2 : s0, k1 = b16 ? s3 : s1;
+      const float x0 = b16 ? s0 : s2, x1 = b16 ? s1 : s3;
+      k0 += __shfl_xor_sync(0xffffffffu, x0, 16);
+      k1 += __shfl_xor_sync(0xffffffffu, x1, 16);
+      float kk = b8 ? k1 : k0;
+      kk += __shfl_xor_sync(0xffffffffu, b8 ? k0 : k1, 8);
+      kk += __shfl_xor_sync(0xffffffffu, kk, 4);
+      kk += __shfl_xor_sync(0xffffffffu, kk, 2);
+      kk += __shfl_xor_sync(0xffffffffu, kk, 1);
+      if ((lane & 7) == 0) cpart[warp][lane >> 3] = kk;
+    }
+    DBG_STAMP(3);
+    // ---- publish round t+1's critical values [0], [1], [2] and [3 + t] (warp CRIT_W) right
+    //      after the barrier, before the other warps' lookahead loads fill the smem pipe ----
+    __syncthreads();
+    if (warp == CRIT_W) {
       const int n = !h2 ? 1 : (!h3 ? 3 : 4);
-      const float s = cta_sum(&cpart[0][0], 4, n);
-      const int c = threadIdx.x >> 2;
-      if ((threadIdx.x & 3) == 0 && c < n) fx_add(t + 1, c < 3 ? c : 3 + t, s);
+      const int c = lane >> 3, j = lane & 7;
+      float s = 0.f;
+      if (j < row_warps) s = cpart[j][c];
+      if (j + 8 < row_warps) s += cpart[j + 8][c];
+      s += __shfl_xor_sync(0xffffffffu, s, 4);
+      s += __shfl_xor_sync(0xffffffffu, s, 2);
+      s += __shfl_xor_sync(0xffffffffu, s, 1);
+      if (j == 0 && c < n) fx_add_scaled(t + 1, c < 3 ? c : 3 + t, s, crit_scale);
+      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && lane == 0) p.dbg[(size_t)t * 8 + 7] = clock64();
     }
     DBG_STAMP(4);
     // ---- while round t+1's exchange is in flight:
-    //      (a) round t+2's lookahead values q_i.a_{t+4}, i <= t (index 3 + i), computed and
-    //          added to round t+2's words now;
+    //      (a) round t+2's lookahead values q_i.a_{t+4}, i <= t (index 3 + i), over this warp's
+    //          row blocks (lane = i), reduced by warp LA_W and added to round t+2's words now;
     //      (b) w_{t+2} = a_{t+2} - sum_{i <= t-1} q_i r_{i,t+2}  (coefficients from round t) ----
     if (t + 4 < w) {
       const int cnt = t + 1;                              // i in [0, t]
       const bool ha = kq < cnt, hb = kq + 32 < cnt;
+      float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
       if (ha && !(p.skip & 2)) {
         const float4* y = reinterpret_cast<const float4*>(sp + (t + 4) * LD);
         const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
         const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
-        float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
-        for (int i = v_lo; i < v_hi; ++i) {
-          const float4 yy = y[i], a = xa[i];
-          a0 = fmaf(a.x, yy.x, a0);
-          a1 = fmaf(a.y, yy.y, a1);
-          a0 = fmaf(a.z, yy.z, a0);
-          a1 = fmaf(a.w, yy.w, a1);
-          if (hb) {
-            const float4 b = xb[i];
-            b0 = fmaf(b.x, yy.x, b0);
-            b1 = fmaf(b.y, yy.y, b1);
-            b0 = fmaf(b.z, yy.z, b0);
-            b1 = fmaf(b.w, yy.w, b1);
+        // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
+        for (int base = 8 * warp; base < nv4; base += LEAF_THREADS / 4) {
+#pragma unroll
+          for (int i = base; i < base + 8; ++i) {
+            const float4 yy = y[i], a = xa[i];
+            a0 = fmaf(a.x, yy.x, a0);
+            a1 = fmaf(a.y, yy.y, a1);
+            a0 = fmaf(a.z, yy.z, a0);
+            a1 = fmaf(a.w, yy.w, a1);
+            if (hb) {
+              const float4 b = xb[i];
+              b0 = fmaf(b.x, yy.x, b0);
+              b1 = fmaf(b.y, yy.y, b1);
+              b0 = fmaf(b.z, yy.z, b0);
+              b1 = fmaf(b.w, yy.w, b1);
+            }
           }
         }
-        part[warp][kq] = a0 + a1;
-        if (hb) part[warp][kq + 32] = b0 + b1;
       }
-      __syncthreads();
-      const float s = cta_sum(&part[0][0], LEAF_MAX_W + 2, cnt);
-      const int i = threadIdx.x >> 2;
-      if ((threadIdx.x & 3) == 0 && i < cnt) fx_add(t + 2, 3 + i, s);
+      if (warp < row_warps) {
+        part[warp][kq] = a0 + a1;
+        part[warp][kq + 32] = b0 + b1;
+      }
+      if (warp == LA_W) {
+        bar_sync_n(2, LEAF_THREADS);
+        float sa = 0.f, sb = 0.f;
+        for (int v = 0; v < row_warps; ++v) {
+          sa += part[v][lane];
+          sb += part[v][lane + 32];
+        }
+        if (lane < cnt) fx_add(t + 2, 3 + lane, sa);
+        if (lane + 32 < cnt) fx_add(t + 2, 3 + lane + 32, sb);
+      } else {
+        bar_arrive_n(2, LEAF_THREADS);
+      }
     }
     DBG_STAMP(5);
-    if (t + 2 < w && t >= 1 && !(p.skip & 4)) project_out(t + 2, t, coef[t & 1]);
+    // prefetch round t+1's words: the load is in flight during the projection below
+    {
+      const int L1 = round_len(t + 1);
+      have_pre = threadIdx.x < L1;
+      if (have_pre) pre = ld_word(p.xw + (size_t)xw_index(t + 1, threadIdx.x) * LEAF_XW_STRIDE, p.sys);
+    }
+    if (t + 2 < w && t >= 1 && !(p.skip & 4)) {
+      // thread-per-row: w_{t+2}[r] -= sum_{i < t} q_i[r] r_{i,t+2}  (two fixed-order partial sums)
+      const float* cf = coef[t % 3];
+      float* an = sp + (t + 2) * LD;
+      for (int r = threadIdx.x; r < rows; r += LEAF_THREADS) {
+        float e0 = 0.f, e1 = 0.f;
+        int k = 0;
+        for (; k + 8 <= t; k += 8) {
+          const float4 c0 = *reinterpret_cast<const float4*>(cf + k);
+          const float4 c1 = *reinterpret_cast<const float4*>(cf + k + 4);
+          const float x0 = sp[(k + 0) * LD + r], x1 = sp[(k + 1) * LD + r], x2 = sp[(k + 2) * LD + r],
+                      x3 = sp[(k + 3) * LD + r], x4 = sp[(k + 4) * LD + r], x5 = sp[(k + 5) * LD + r],
+                      x6 = sp[(k + 6) * LD + r], x7 = sp[(k + 7) * LD + r];
+          e0 = fmaf(x0, c0.x, e0);
+          e1 = fmaf(x1, c0.y, e1);
+          e0 = fmaf(x2, c0.z, e0);
+          e1 = fmaf(x3, c0.w, e1);
+          e0 = fmaf(x4, c1.x, e0);
+          e1 = fmaf(x5, c1.y, e1);
+          e0 = fmaf(x6, c1.z, e0);
+          e1 = fmaf(x7, c1.w, e1);
+        }
+        for (; k + 2 <= t; k += 2) {
+          e0 = fmaf(sp[k * LD + r], cf[k], e0);
+          e1 = fmaf(sp[(k + 1) * LD + r], cf[k + 1], e1);
+        }
+        if (k < t) e0 = fmaf(sp[k * LD + r], cf[k], e0);
+        an[r] -= e0 + e1;
+      }
+    }
     DBG_STAMP(6);
   }
   // every CTA ends with the same last-seen words; CTA 0 persists them for the next launch

@@ -24,6 +24,9 @@
 //           transferring" D2D copy, used here to build the resident A2').
 // The blocked algorithm (option ALGO=1) reuses the same node primitives
 // with a fixed panel width instead of the recursion.
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+
 #include <chrono>
 #include <climits>
 #include <cstring>
@@ -52,6 +55,7 @@ struct Exec {
   int K;
   int64_t tmin, tmax;
   bool reuse;
+  bool reorth;
 
   // ---- timing / accounting helpers ----
   cudaEvent_t seg_begin(cudaStream_t st) {
@@ -311,12 +315,13 @@ struct Exec {
     const size_t dB = (size_t)m * w1 * s + 256;
     const size_t left_ws = incore_need(w1) - dB;
     const size_t right_ws = incore_need(w2) - (size_t)m * w2 * s;
-    bool q1_res = reuse && dB + r12b + r12ob + left_ws + (size_t)K * 128 * w2 * s <= free0;
+    bool q1_res = reuse && dB + r12b * (reorth ? 2 : 1) + r12ob + left_ws + (size_t)K * 128 * w2 * s <= free0;
     bool a2_to_d = q1_res && recursive && w2 <= w1 && dB + right_ws <= free0;
     if (q1_res) {
       char* D = static_cast<char*>(c->arena.alloc(dB));
       float* R12 = static_cast<float*>(c->arena.alloc(r12b));
       void* R12op = c->arena.alloc(r12ob);
+      float* S = reorth ? static_cast<float*>(c->arena.alloc(r12b)) : R12;
       // the left child's R block lives below the ring for the whole node, so neither the
       // uploads of the inner pass nor its kernels wait for that block's download
       const size_t rsb = (size_t)w1 * w1 * 4;
@@ -325,7 +330,7 @@ struct Exec {
       const size_t ws_left = left_ws > rsb ? left_ws - rsb : 0;
       const size_t avail = c->arena.free_bytes() > ws_left + 4096 ? c->arena.free_bytes() - ws_left - 4096 : 0;
       const int64_t t = pick_tile(avail, w2);
-      if (!D || !R12 || !R12op || !Rs1 || t < 128) {
+      if (!D || !R12 || !R12op || !S || !Rs1 || t < 128) {
         c->arena.release(mark0);
         q1_res = a2_to_d = false;
       } else {
@@ -337,15 +342,23 @@ struct Exec {
         if (rc < 0) return rc;
         rc = stream_inner(c0, w1, w2, src_q, D, R12, R12op, ring, t, ev_free);
         if (rc < 0) return rc;
-        wait(sd, sc);
-        rc = d2h_r(c0, h, w1, w2, R12, w1);
+        cudaEvent_t r12_out = nullptr;
+        if (!reorth) {
+          wait(sd, sc);
+          rc = d2h_r(c0, h, w1, w2, R12, w1);
+          if (rc < 0) return rc;
+          r12_out = c->ev();
+          cudaEventRecord(r12_out, sd);
+        }
+        rc = stream_outer(c0, w1, w2, src_q, D, a2_to_d && !reorth, q1_done, R12op, ring, t, ev_free);
         if (rc < 0) return rc;
-        cudaEvent_t r12_out = c->ev();
-        cudaEventRecord(r12_out, sd);
-        rc = stream_outer(c0, w1, w2, src_q, D, a2_to_d, q1_done, R12op, ring, t, ev_free);
-        if (rc < 0) return rc;
+        if (reorth) {
+          // CGS2: S = Q1^T A2' (A2' from the host copy just written), R12 += S, A2' -= Q1 S
+          rc = reorth_pass(c0, w1, w2, D, a2_to_d, q1_done, R12, S, R12op, ring, t, ev_free, &r12_out);
+          if (rc < 0) return rc;
+        }
         // R12 / ring memory is released below: make every stream wait for its last users
-        cudaStreamWaitEvent(sc, r12_out, 0);
+        if (r12_out) cudaStreamWaitEvent(sc, r12_out, 0);
         join_all();
         c->arena.release(mark0 + 0);
         if (a2_to_d) {
@@ -368,7 +381,8 @@ struct Exec {
     join_all();
     float* R12 = static_cast<float*>(c->arena.alloc(r12b));
     void* R12op = c->arena.alloc(r12ob);
-    if (!R12 || !R12op) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: no space for R12");
+    float* S = reorth ? static_cast<float*>(c->arena.alloc(r12b)) : R12;
+    if (!R12 || !R12op || !S) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: no space for R12");
     const int64_t t = pick_tile(c->arena.free_bytes() > 4096 ? c->arena.free_bytes() - 4096 : 0, w1 + w2);
     if (t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: ring does not fit the budget");
     char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
@@ -376,14 +390,52 @@ struct Exec {
     for (int k = 0; k < K; ++k) ev_free[k] = c->ev();
     rc = stream_inner(c0, w1, w2, src_q, nullptr, R12, R12op, ring, t, ev_free);
     if (rc < 0) return rc;
-    wait(sd, sc);
-    rc = d2h_r(c0, h, w1, w2, R12, w1);
-    if (rc < 0) return rc;
+    if (!reorth) {
+      wait(sd, sc);
+      rc = d2h_r(c0, h, w1, w2, R12, w1);
+      if (rc < 0) return rc;
+    }
     rc = stream_outer(c0, w1, w2, src_q, nullptr, false, nullptr, R12op, ring, t, ev_free);
     if (rc < 0) return rc;
+    if (reorth) {
+      rc = reorth_pass(c0, w1, w2, nullptr, false, nullptr, R12, S, R12op, ring, t, ev_free, nullptr);
+      if (rc < 0) return rc;
+    }
     join_all();
     c->arena.release(mark0);
     return recursive ? node(h, w2, true) : RGSQR_OK;
+  }
+
+  // CGS2 second projection of an OOC node: A2' lives in the host Q copy (written by the
+  // first outer pass).  S = Q1^T A2', R12 += S (then R12 is written out once), A2'' =
+  // A2' - Q1 S (to D when to_D: Q1 is no longer needed after this pass).
+  int reorth_pass(int64_t c0, int64_t w1, int64_t w2, char* D, bool to_D, cudaEvent_t q1_done, float* R12,
+                  float* S, void* Sop, char* ring, int64_t t, std::vector<cudaEvent_t>& ev_free,
+                  cudaEvent_t* r12_out) {
+    const int64_t h = c0 + w1;
+    int rc = stream_inner(c0, w1, w2, true, D, S, Sop, ring, t, ev_free);
+    if (rc < 0) return rc;
+    cudaEvent_t a = seg_begin(sc);
+    switch (prec) {
+      case RGSQR_FP16:
+        RGSQR_CUDA(c, launch_splitk_reduce<__half>(S, w1 * w2, w1, 1, R12, w1, 1, nullptr, 0, w1, w2, sc));
+        break;
+      case RGSQR_BF16:
+        RGSQR_CUDA(c, launch_splitk_reduce<__nv_bfloat16>(S, w1 * w2, w1, 1, R12, w1, 1, nullptr, 0, w1, w2, sc));
+        break;
+      default:
+        RGSQR_CUDA(c, launch_splitk_reduce<float>(S, w1 * w2, w1, 1, R12, w1, 1, nullptr, 0, w1, w2, sc));
+    }
+    c->stats.n_other_launches++;
+    seg_end(2, sc, a);
+    wait(sd, sc);
+    rc = d2h_r(c0, h, w1, w2, R12, w1);
+    if (rc < 0) return rc;
+    if (r12_out) {
+      *r12_out = c->ev();
+      cudaEventRecord(*r12_out, sd);
+    }
+    return stream_outer(c0, w1, w2, true, D, to_D, q1_done, Sop, ring, t, ev_free);
   }
 
   int panel(int64_t c0, int64_t w, bool src_q) {
@@ -469,7 +521,7 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   }
   Exec x{c, prec, s, static_cast<const char*>(A), static_cast<char*>(Q), lda, m, n, R,
          c->compute(), c->st_h2d, c->st_d2h, (int)c->opt.ring_depth, c->opt.tile_rows_min,
-         c->opt.tile_rows_max, c->opt.reuse != 0};
+         c->opt.tile_rows_max, c->opt.reuse != 0, c->opt.reorth != 0};
   if (c->opt.serialize) x.sh = x.sd = x.sc;
   // make the copy streams start after prior work of the compute stream
   x.join_all();

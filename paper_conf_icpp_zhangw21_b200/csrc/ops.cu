@@ -392,7 +392,14 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
       fprintf(stderr, " %s %.0f", names[i], ph[i] / std::max(1, cnt));
       sum += ph[i];
     }
-    fprintf(stderr, " | total %.0f\n", sum / std::max(1, cnt));
+    // stamp 7: the critical reducer warp published round t+1's values
+    double pub = 0, xl = 0;
+    for (int t = 1; t + 2 < w; ++t) {
+      pub += (double)(hb[t * 8 + 7] - hb[t * 8 + 1]);
+      xl += (double)(hb[(t + 1) * 8 + 1] - hb[t * 8 + 7]);
+    }
+    fprintf(stderr, " | total %.0f | publish@%.0f publish->next-barrier %.0f\n", sum / std::max(1, cnt),
+            pub / std::max(1, cnt - 1), xl / std::max(1, cnt - 1));
   }
   c->stats.n_leaf_launches++;
   return RGSQR_OK;
@@ -417,6 +424,10 @@ size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n) {
   if (w1 > 0) b += (size_t)w1 * (n - w1) * elem_bytes(prec) + 1024;  // R12 operand copy
   if (w1 > 0 && c->nccl_comm) b += (size_t)w1 * (n - w1) * 4 + 1024;  // R12 rank-reduction buffer
   if (prec == RGSQR_TF32X3) b += (size_t)m * n * 4 + 4096;              // lo operands of the top node
+  if (c->opt.reorth) {                                                   // CGS2: S (fp32) + leaf S block
+    if (w1 > 0) b += (size_t)w1 * (n - w1) * 4 + 1024;
+    b += (size_t)LEAF_MAX_W * LEAF_MAX_W * 4 + 1024;
+  }
   // split-K partials: op_inner adapts its split factor to what is free; reserve a
   // quarter of the node's matrix bytes, clamped to [1, 16] MiB
   const size_t node_bytes = (size_t)m * n * elem_bytes(prec);
@@ -434,6 +445,8 @@ struct IncoreCtx {
   int64_t ldr;
   int64_t leaf;
   void* r12op;
+  float* S;        // CGS2: second-pass R12 (fp32, ld w1) of the widest node
+  float* S11;      // CGS2: second-pass leaf R block (LEAF_MAX_W x LEAF_MAX_W)
   int64_t col_offset;
   cudaStream_t st;
   IncoreHooks* hooks;
@@ -443,8 +456,17 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
   const int64_t w1 = split_width(w, k.leaf);
   if (w1 == 0) {
     if (k.hooks && k.hooks->need) k.hooks->need(c0 + w);
-    int rc = op_leaf(k.c, k.prec, k.A + c0 * k.lda * k.s, k.lda, k.m, w, k.R + c0 + c0 * k.ldr, k.ldr,
-                     k.col_offset + c0, k.st);
+    char* P = k.A + c0 * k.lda * k.s;
+    float* R11 = k.R + c0 + c0 * k.ldr;
+    int rc = op_leaf(k.c, k.prec, P, k.lda, k.m, w, R11, k.ldr, k.col_offset + c0, k.st);
+    if (rc == 0 && k.S11) {
+      // CGS2 leaf: factor Q' again, Q' = Q S, and R11 <- S R11
+      rc = op_leaf(k.c, k.prec, P, k.lda, k.m, w, k.S11, w, k.col_offset + c0, k.st);
+      if (rc == 0) {
+        RGSQR_CUDA(k.c, launch_trmm_upper(k.S11, w, R11, k.ldr, (int)w, k.st));
+        k.c->stats.n_other_launches++;
+      }
+    }
     if (rc == 0 && k.hooks && k.hooks->leaf_done) k.hooks->leaf_done(c0 + w);
     return rc;
   }
@@ -454,11 +476,28 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
   if (k.hooks && k.hooks->need) k.hooks->need(c0 + w);
   const char* Q1 = k.A + c0 * k.lda * k.s;
   char* A2 = k.A + h * k.lda * k.s;
-  rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, k.R + c0 + h * k.ldr, k.ldr, k.r12op, w1, 0,
-                k.st);
+  float* R12 = k.R + c0 + h * k.ldr;
+  rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.r12op, w1, 0, k.st);
   if (rc < 0) return rc;
   rc = op_outer(k.c, k.prec, Q1, k.lda, k.r12op, w1, A2, k.lda, k.m, w1, w2, k.st);
   if (rc < 0) return rc;
+  if (k.S) {
+    // CGS2: S = Q1^T A2', A2' -= Q1 S, R12 += S (fixed order)
+    rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, k.S, w1, k.r12op, w1, 0, k.st);
+    if (rc < 0) return rc;
+    rc = op_outer(k.c, k.prec, Q1, k.lda, k.r12op, w1, A2, k.lda, k.m, w1, w2, k.st);
+    if (rc < 0) return rc;
+    cudaError_t e;
+    switch (k.prec) {
+      case RGSQR_FP16: e = launch_splitk_reduce<__half>(k.S, w1 * w2, w1, 1, R12, k.ldr, 1, nullptr, 0, w1, w2, k.st); break;
+      case RGSQR_BF16:
+        e = launch_splitk_reduce<__nv_bfloat16>(k.S, w1 * w2, w1, 1, R12, k.ldr, 1, nullptr, 0, w1, w2, k.st);
+        break;
+      default: e = launch_splitk_reduce<float>(k.S, w1 * w2, w1, 1, R12, k.ldr, 1, nullptr, 0, w1, w2, k.st);
+    }
+    if (e != cudaSuccess) return fail(k.c, RGSQR_ERR_CUDA, std::string("reorth R12 += S: ") + cudaGetErrorString(e));
+    k.c->stats.n_other_launches++;
+  }
   k.c->stats.n_incore_nodes++;
   return incore_rec(k, h, w2);
 }
@@ -466,13 +505,21 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
 int incore_factor(Ctx* c, int prec, void* A, int64_t lda, int64_t m, int64_t n, float* R, int64_t ldr,
                   int64_t col_offset, cudaStream_t st, IncoreHooks* hooks) {
   IncoreCtx k{c, prec, static_cast<char*>(A), lda, m, elem_bytes(prec), R, ldr, leaf_width_for(c, m), nullptr,
-              col_offset, st, hooks};
+              nullptr, nullptr, col_offset, st, hooks};
   if (k.leaf < 1) return fail(c, RGSQR_ERR_UNSUPPORTED, "in-core: m too large for the on-chip leaf");
   const int64_t w1 = split_width(n, k.leaf);
   size_t mark = c->arena.mark();
   if (w1 > 0) {
     k.r12op = c->arena.alloc((size_t)w1 * (n - w1) * k.s);
     if (!k.r12op) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core: no arena space for R12");
+    if (c->opt.reorth) {
+      k.S = static_cast<float*>(c->arena.alloc((size_t)w1 * (n - w1) * 4));
+      if (!k.S) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core: no arena space for the CGS2 R12");
+    }
+  }
+  if (c->opt.reorth) {
+    k.S11 = static_cast<float*>(c->arena.alloc((size_t)LEAF_MAX_W * LEAF_MAX_W * 4));
+    if (!k.S11) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core: no arena space for the CGS2 leaf block");
   }
   int rc = incore_rec(k, 0, n);
   c->arena.release(mark);

@@ -5,7 +5,7 @@ import numpy as np
 import pytest
 
 import oracle
-from oracle import cgs, cgs2, rgs, blocked_cgs, rgs_emulated
+from oracle import cgs, cgs2, rgs, rgs2, blocked_cgs, rgs_emulated
 import rgsqr_inputs as gi
 
 
@@ -22,6 +22,8 @@ ALGOS = {
     "O3": lambda X: rgs(X, leaf=4),
     "O3-leaf1": lambda X: rgs(X, leaf=1),
     "O4": lambda X: blocked_cgs(X, 3),
+    "O6": lambda X: rgs2(X, leaf=4),
+    "O6-leaf1": lambda X: rgs2(X, leaf=1),
 }
 
 
@@ -157,3 +159,48 @@ def test_gaussian_shard_reproducible():
     full = gi.gaussian(3 * gi.ROW_BLOCK, 16, seed=9, dtype="fp16")
     part = gi.gaussian(gi.ROW_BLOCK, 16, seed=9, dtype="fp16", row0=gi.ROW_BLOCK)
     np.testing.assert_array_equal(full[gi.ROW_BLOCK:2 * gi.ROW_BLOCK], part)
+
+
+def test_rgs2_orthogonality_signature():
+    """O6 (recursive CGS2) keeps O(u) orthogonality where CGS (O3) loses u*kappa^2:
+    the property that makes it the reorthogonalized variant.  A
+    missing second projection at the nodes or a missing second leaf pass fails here."""
+    A, _ = gi.usv(512, 64, kappa=1e7, seed=2)
+    loss_rgs = oracle.orthogonality(rgs(A, leaf=8).Q)
+    loss_rgs2 = oracle.orthogonality(rgs2(A, leaf=8).Q)
+    assert loss_rgs > 1e-7            # measured 9.7e-7 (u kappa^2 = 1e-2 is the worst case)
+    assert loss_rgs2 < 1e-12          # measured 3.8e-13
+    # a version with only the node reorthogonalization (single-pass leaves) is not enough
+    X = np.array(A, order="F", copy=True)
+    res = rgs2(A, leaf=64)          # one leaf = panel twice, no nodes
+    assert oracle.orthogonality(res.Q) < 1e-13
+    # and R is still the unique positive-diagonal R (Gram-Cholesky of the input, kappa^2 u ~ 1e-2
+    # is too large for that route, so compare with Householder)
+    _, Rh = _householder_ref(X)
+    assert oracle.r_rel_error(rgs2(A, leaf=8).R, Rh) < 1e-8
+
+
+def test_rgs2_dyadic_exact():
+    # exact-dyadic input: the second projections are exactly 0 and the second leaf passes
+    # exactly I, so O6 reproduces R0 and Q = H bitwise, like O3
+    A, R0 = gi.dyadic_mixed(1024, 96, seed=5)
+    res = rgs2(A, leaf=16)
+    np.testing.assert_array_equal(res.R, R0)
+    np.testing.assert_array_equal(res.Q, gi.hadamard(1024, 96))
+
+
+@pytest.mark.parametrize("mode", ["fp16", "tf32x3"])
+def test_emulated_reorth_levels(mode):
+    """O5 with reorth=True: at kappa = 1e3 CGS2 keeps orthogonality at the storage level
+    (the GPU CGS2 test thresholds come from here), single-pass CGS does not."""
+    A, _ = gi.usv(2048, 128, kappa=1e3, seed=3)
+    X = gi.to_float64(gi.to_storage(A.astype(np.float32), "fp16" if mode == "fp16" else "fp32"),
+                      "fp16" if mode == "fp16" else "fp32")
+    one = oracle.orthogonality(rgs_emulated(X, mode, leaf=32).Q)
+    two = oracle.orthogonality(rgs_emulated(X, mode, leaf=32, reorth=True).Q)
+    if mode == "fp16":
+        assert one > 0.1 and two < 0.05
+    else:
+        assert one > 1e-4 and two < 1e-5
+    ref = rgs(X, leaf=32)
+    assert oracle.r_rel_error(rgs_emulated(X, mode, leaf=32, reorth=True).R, ref.R) < (5e-3 if mode == "fp16" else 1e-5)
