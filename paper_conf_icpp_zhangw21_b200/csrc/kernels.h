@@ -58,8 +58,10 @@ struct LeafParams {
   float* partials;          // [2][LEAF_MAX_W+2][grid] per-CTA partial sums
   unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
   long long* dbg;           // optional [w][8] clock64 stamps of CTA dbg_cta
+  long long* dbg2;          // optional [grid][LEAF_MAX_W][2] globaltimer: critical publish, poll done
   int dbg_cta;
   int skip;                 // diagnostics only (RGSQR_LEAF_SKIP): 2 lookahead dots, 4 projection
+  int poll_sleep_ns;        // backoff between exchange polls (RGSQR_LEAF_POLL_NS, default 0)
   int vec_ok;               // P and ldp*sizeof(elem) 16-byte aligned: vector panel loads
   unsigned int epoch;       // launch counter
   unsigned long long* xw;   // LEAF_XW_WORDS words (stride LEAF_XW_STRIDE), this GPU's, never reset

@@ -58,6 +58,12 @@ static constexpr int FX_VBITS = 41;
 __device__ __forceinline__ void bar_sync_n(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 __device__ __forceinline__ void bar_arrive_n(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
+__device__ __forceinline__ long long gtimer() {
+  long long v;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
+  return v;
+}
+
 // exact power of two as a double (|e| < 1000)
 __device__ __forceinline__ double pow2d(int e) { return __hiloint2double((1023 + e) << 20, 0); }
 
@@ -367,14 +373,16 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         unsigned long long now = have_pre ? pre : ld_word(wp, p.sys), d = now - prev;
         long long spins = 0;
         while ((unsigned)(d >> FX_CNT_SHIFT) != cnt) {
+          if (p.poll_sleep_ns) __nanosleep(p.poll_sleep_ns);
           now = ld_word(wp, p.sys);
           d = now - prev;
-          if (++spins > (1ll << 27)) {            // ~seconds: a peer is missing -- fail, never hang
+          if (++spins > (1ll << 22)) {            // ~seconds: a peer is missing -- fail, never hang
             atomicExch(p.breakdown, -2);
             break;
           }
         }
         xprev[widx] = now;
+        if (p.dbg2 != nullptr && k == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 1] = gtimer();
         const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
         const float val = (float)((double)total * pow2d(-fx_exp(t, k)));
         tot[t & 1][k] = val;
@@ -478,6 +486,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       s += __shfl_xor_sync(0xffffffffu, s, 1);
       if (j == 0 && c < n) fx_add_scaled(t + 1, c < 3 ? c : 3 + t, s, crit_scale);
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && lane == 0) p.dbg[(size_t)t * 8 + 7] = clock64();
+      if (p.dbg2 != nullptr && lane == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 0] = gtimer();
     }
     DBG_STAMP(4);
     // ---- while round t+1's exchange is in flight:

@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <climits>
 #include <mutex>
+#include <vector>
 
 #include "engine.h"
 
@@ -337,9 +338,15 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   p.vec_ok = ((ldp * elem_bytes(prec)) % 16 == 0) && (reinterpret_cast<uintptr_t>(P) % 16 == 0);
   if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 8 * LEAF_MAX_W);
   p.dbg = dbg ? dbg_buf : nullptr;
+  static const bool dbg2 = getenv("RGSQR_LEAF_DEBUG2") != nullptr;
+  static long long* dbg2_buf = nullptr;
+  if (dbg2 && !dbg2_buf) cudaMalloc(&dbg2_buf, sizeof(long long) * 2 * LEAF_MAX_W * LEAF_MAX_G);
+  p.dbg2 = dbg2 ? dbg2_buf : nullptr;
   p.dbg_cta = dbg ? atoi(getenv("RGSQR_LEAF_DEBUG")) : 0;
   static const int skip = getenv("RGSQR_LEAF_SKIP") ? atoi(getenv("RGSQR_LEAF_SKIP")) : 0;
   p.skip = dbg ? skip : 0;
+  static const int poll_ns = getenv("RGSQR_LEAF_POLL_NS") ? atoi(getenv("RGSQR_LEAF_POLL_NS")) : 0;
+  p.poll_sleep_ns = poll_ns;
   p.breakdown = c->d_breakdown;
   p.col_offset = col_offset;
   auto launch = [&](const LeafParams& q) -> cudaError_t {
@@ -400,6 +407,32 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
     }
     fprintf(stderr, " | total %.0f | publish@%.0f publish->next-barrier %.0f\n", sum / std::max(1, cnt),
             pub / std::max(1, cnt - 1), xl / std::max(1, cnt - 1));
+  }
+  if (p.dbg2) {
+    std::vector<long long> hb((size_t)2 * LEAF_MAX_W * G);
+    cudaMemcpyAsync(hb.data(), p.dbg2, sizeof(long long) * hb.size(), cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+    // exchange round r: published in iteration r-1 (slot 0), detected in iteration r (slot 1)
+    double skew = 0, first = 0, last = 0, mean = 0, per = 0;
+    int cnt = 0;
+    for (int r = 2; r + 1 < w; ++r, ++cnt) {
+      long long pmax = LLONG_MIN, pmin = LLONG_MAX, dmin = LLONG_MAX, dmax = LLONG_MIN;
+      double dsum = 0;
+      for (int g = 0; g < G; ++g) {
+        const long long P = hb[((size_t)g * LEAF_MAX_W + r - 1) * 2], D = hb[((size_t)g * LEAF_MAX_W + r) * 2 + 1];
+        pmax = std::max(pmax, P); pmin = std::min(pmin, P);
+        dmax = std::max(dmax, D); dmin = std::min(dmin, D);
+        dsum += (double)D;
+      }
+      skew += (double)(pmax - pmin);
+      first += (double)(dmin - pmax);
+      last += (double)(dmax - pmax);
+      mean += dsum / G - (double)pmax;
+      per += (double)(hb[((size_t)0 * LEAF_MAX_W + r) * 2] - hb[((size_t)0 * LEAF_MAX_W + r - 1) * 2]);
+    }
+    cnt = std::max(cnt, 1);
+    fprintf(stderr, "[leaf2 m=%lld w=%lld G=%d] ns/round %.0f | publish skew %.0f | last publish -> detect: first %.0f mean %.0f last %.0f\n",
+            (long long)m, (long long)w, G, per / cnt, skew / cnt, first / cnt, mean / cnt, last / cnt);
   }
   c->stats.n_leaf_launches++;
   return RGSQR_OK;
