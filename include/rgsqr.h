@@ -76,11 +76,15 @@ enum rgsqr_option {
   RGSQR_OPT_LEAF_CTAS = 9,      /* CTAs of the leaf kernel (0 = automatic) */
   RGSQR_OPT_SPLITK = 10,        /* force split-K factor of the TN product (0 = automatic) */
   RGSQR_OPT_PROFILE = 11,       /* 1 = time every kernel with CUDA events (rgsqr_stats.kern_*) */
-  RGSQR_OPT_REORTH = 12         /* 1 = CGS2: every projection R12 = Q1^T A2, A2 -= Q1 R12 and every leaf
+  RGSQR_OPT_REORTH = 12,        /* 1 = CGS2: every projection R12 = Q1^T A2, A2 -= Q1 R12 and every leaf
                                    panel factorization applied twice ("twice is enough"
                                    reorthogonalization; CGS2 is named with CGS at PAPER.md:109 as the
                                    stable relative, reading R22).
                                    R12 = R12' + S, R_leaf = S R'.  Default 0 (the paper's CGS) */
+  RGSQR_OPT_PREFETCH = 13       /* 1 = an OOC node uploads its first K ring tiles of A2 while its
+                                   left child is being factored (cross-operation overlap,
+                                   PAPER.md:231-233; tiles then start at full height instead of
+                                   the ramp).  Default 1 */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

@@ -401,6 +401,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_SPLITK: return &o.splitk;
     case RGSQR_OPT_PROFILE: return &o.profile;
     case RGSQR_OPT_REORTH: return &o.reorth;
+    case RGSQR_OPT_PREFETCH: return &o.prefetch;
   }
   return nullptr;
 }

@@ -27,6 +27,7 @@ struct Options {
   int64_t splitk = 0;
   int64_t profile = 0;
   int64_t reorth = 0;        // CGS2 (RGSQR_OPT_REORTH)
+  int64_t prefetch = 1;      // OOC: upload the first ring tiles during the left child (RGSQR_OPT_PREFETCH)
 };
 
 struct KernSeg {

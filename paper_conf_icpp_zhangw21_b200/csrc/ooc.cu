@@ -116,9 +116,10 @@ struct Exec {
   size_t incore_need(int64_t w) const {
     return (size_t)m * w * s + 256 + (size_t)w * w * 4 + 256 + incore_workspace_bytes(c, prec, m, w) + 4096;
   }
+  bool flat = false;   // no ramp: the first tiles were prefetched (see prefetch_tiles)
   std::vector<int64_t> tiles(int64_t t) const {
     std::vector<int64_t> v;
-    int64_t r = 0, cur = std::min(tmin, t);
+    int64_t r = 0, cur = flat ? t : std::min(tmin, t);
     while (r < m) {
       int64_t h = std::min(cur, m - r);
       v.push_back(h);
@@ -203,7 +204,8 @@ struct Exec {
 
   // ---- streamed inner product  R12 = Q1^T A2  (Q1 resident in D when D != null) ----
   int stream_inner(int64_t c0, int64_t w1, int64_t w2, bool a2_src_q, const char* D, float* R12, void* R12op,
-                   char* ring, int64_t t, std::vector<cudaEvent_t>& ev_free) {
+                   char* ring, int64_t t, std::vector<cudaEvent_t>& ev_free,
+                   const std::vector<cudaEvent_t>* pre = nullptr) {
     const int64_t h = c0 + w1;
     const int64_t slot_cols = (D ? 0 : w1) + w2;
     std::vector<cudaEvent_t> loaded(K);
@@ -216,15 +218,20 @@ struct Exec {
       char* slot = ring + (size_t)k * t * slot_cols * s;
       char* sq = slot;
       char* sa = slot + (D ? 0 : (size_t)t * w1 * s);
-      cudaStreamWaitEvent(sh, ev_free[k], 0);
-      if (!D) {
-        int rc = h2d(sq, t, Q, r0, tr, c0, w1);
+      int rc;
+      if (pre && i < pre->size()) {
+        cudaStreamWaitEvent(sc, (*pre)[i], 0);            // uploaded during the left child
+      } else {
+        cudaStreamWaitEvent(sh, ev_free[k], 0);
+        if (!D) {
+          rc = h2d(sq, t, Q, r0, tr, c0, w1);
+          if (rc < 0) return rc;
+        }
+        rc = h2d(sa, t, hsrc(a2_src_q), r0, tr, h, w2);
         if (rc < 0) return rc;
+        cudaEventRecord(loaded[k], sh);
+        cudaStreamWaitEvent(sc, loaded[k], 0);
       }
-      int rc = h2d(sa, t, hsrc(a2_src_q), r0, tr, h, w2);
-      if (rc < 0) return rc;
-      cudaEventRecord(loaded[k], sh);
-      cudaStreamWaitEvent(sc, loaded[k], 0);
       cudaEvent_t a = seg_begin(sc);
       const bool last = (i + 1 == tl.size());
       // distributed: accumulate the LOCAL partial over all tiles, reduce across ranks once
@@ -239,6 +246,24 @@ struct Exec {
       seg_end(2, sc, a);
       cudaEventRecord(ev_free[k], sc);
       r0 += tr;
+    }
+    return RGSQR_OK;
+  }
+
+  // ---- cross-operation overlap: upload the first ring slots of the
+  //      node's A2 while the left child is still being factored (the copy engine is idle
+  //      once the left child's own columns are in); Q1 resident (rule 1) ----
+  int prefetch_tiles(int64_t h, int64_t w2, bool a2_src_q, char* ring, int64_t t, std::vector<cudaEvent_t>* pre) {
+    auto tl = tiles(t);
+    int64_t r0 = 0;
+    for (size_t i = 0; i < tl.size() && i < (size_t)K; ++i) {
+      char* slot = ring + (size_t)i * t * w2 * s;
+      int rc = h2d(slot, t, hsrc(a2_src_q), r0, tl[i], h, w2);
+      if (rc < 0) return rc;
+      cudaEvent_t e = c->ev();
+      cudaEventRecord(e, sh);
+      pre->push_back(e);
+      r0 += tl[i];
     }
     return RGSQR_OK;
   }
@@ -338,9 +363,16 @@ struct Exec {
         std::vector<cudaEvent_t> ev_free(K);
         for (int k = 0; k < K; ++k) ev_free[k] = c->ev();
         cudaEvent_t q1_done = nullptr;
+        const bool saved_flat = flat;
+        flat = c->opt.prefetch != 0;
         int rc = incore_node(c0, w1, src_q, D, false, &q1_done, Rs1);
         if (rc < 0) return rc;
-        rc = stream_inner(c0, w1, w2, src_q, D, R12, R12op, ring, t, ev_free);
+        std::vector<cudaEvent_t> pre;
+        if (flat) {
+          rc = prefetch_tiles(h, w2, src_q, ring, t, &pre);
+          if (rc < 0) return rc;
+        }
+        rc = stream_inner(c0, w1, w2, src_q, D, R12, R12op, ring, t, ev_free, &pre);
         if (rc < 0) return rc;
         cudaEvent_t r12_out = nullptr;
         if (!reorth) {
@@ -361,6 +393,7 @@ struct Exec {
         if (r12_out) cudaStreamWaitEvent(sc, r12_out, 0);
         join_all();
         c->arena.release(mark0 + 0);
+        flat = saved_flat;
         if (a2_to_d) {
           // keep D (now holding A2', rows permuted by nothing: same row order) for the right child
           char* D2 = static_cast<char*>(c->arena.alloc(dB));  // same address as D (LIFO)
