@@ -12,10 +12,15 @@ constexpr int LEAF_PARTS = 4;         // row quarters of the per-CTA partial sum
 // leaf exchange words: [LEAF_XW_SETS round sets][LEAF_MAX_W+2 values], word i at
 // xw[i * LEAF_XW_STRIDE] (one 256-byte line each: concurrent atomics and polls of different
 // values land in different L2 slices)
-constexpr int LEAF_XW_SETS = 4;
+constexpr int LEAF_XW_SETS = 8;
 constexpr int LEAF_XW_STRIDE = 32;
 constexpr int LEAF_XW_WORDS = LEAF_XW_SETS * (LEAF_MAX_W + 2);
 constexpr size_t LEAF_SMEM_BUDGET = 200 * 1024;
+// the leaf keeps its projected columns w_j in a ring of LEAF_WRING extra smem columns (the
+// original a_j stay intact until u_j replaces them, see leaf.cu)
+constexpr int LEAF_WRING = 3;
+// rows per CTA the leaf's critical group holds in registers (8 rows x 256 threads)
+constexpr int LEAF_MAX_RP = 2048;
 // smem column stride of the leaf panel slice: >= rows and == 4 (mod 32), so that the
 // float4 reads of 8 threads at the same row in 8 different columns hit 32 distinct banks
 __host__ __device__ inline int leaf_ld(int rows) { return ((rows + 31) / 32) * 32 + 4; }

@@ -54,6 +54,15 @@ __device__ __forceinline__ unsigned long long ld_word(const unsigned long long* 
 static constexpr int FX_CNT_SHIFT = 53;
 static constexpr int FX_VBITS = 41;
 
+__device__ __forceinline__ void st_release_shared(int* p, int v) {
+  asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(p)), "r"(v) : "memory");
+}
+__device__ __forceinline__ int ld_acquire_shared(const int* p) {
+  int v;
+  asm volatile("ld.acquire.cta.shared.b32 %0, [%1];" : "=r"(v) : "r"((unsigned)__cvta_generic_to_shared(p)) : "memory");
+  return v;
+}
+
 // named barriers: the reducing warp waits for all threads, the others only arrive
 __device__ __forceinline__ void bar_sync_n(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 __device__ __forceinline__ void bar_arrive_n(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
@@ -140,16 +149,18 @@ __device__ __forceinline__ void store4<float>(float* dst, float4 v) {
   *reinterpret_cast<float4*>(dst) = v;
 }
 
-template <typename T>
+// NR: rows per critical-group thread (rows_per_cta <= 256 NR)
+template <typename T, int NR>
 __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p) {
   extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
   __shared__ float tot[2][LEAF_MAX_W + 2];         // reduced round vector, by parity of the round
   __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];        // round 0 / lookahead partials
-  __shared__ float cpart[GEMV_PARTS][4];                    // critical-dot partials
+  __shared__ float cpart[GEMV_PARTS][8];                    // critical-dot partials
   __shared__ unsigned long long xprev[LEAF_XW_WORDS];      // last seen exchange words
-  __shared__ __align__(16) float coef[3][LEAF_MAX_W + 4];   // r_{i,t+2}, i < t, by t mod 3
+  __shared__ __align__(16) float coef[3][LEAF_MAX_W + 4];   // r_{i,t+3}, i < t, by t mod 3
   __shared__ int exS[LEAF_MAX_W];                           // 2||a_j|| < 2^exS[j]
   __shared__ float tauc[LEAF_MAX_W];                        // breakdown thresholds
+  __shared__ double fxs[LEAF_MAX_W][5], fxi[LEAF_MAX_W][5];  // fixed-point scales by (round, class)
   // last-seen exchange words persist across launches (words are never reset, see fx_exp)
   for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) xprev[i] = p.xprev_g[i];
 
@@ -216,19 +227,20 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   // (deterministic) and exact in fixed point; words are never reset: readers take the
   // difference with the value they saw at the previous use of the word.
   auto fx_exp = [&](int t, int k) -> int {
-    // |partial| <= bound: 4||a_t||^2, 4||a_t|| ||a_{t+1}||, 4||a_{t+1}||, 4||a_{t+2}|| for value
-    // classes 0, 1, 2, 3+ (u_t shrinks a_t, ||q_i|| <= 1); 2||a_j|| < 2^exS[j]
+    // |partial| <= bound: ||a_t||^2, ||a_t|| ||a_{t+1}||, ||a_{t+1}||, ||a_{t+2}||, ||a_{t+3}|| for
+    // value classes 0, 1, 2, 3, 4+ (u_t shrinks a_t, ||q_i|| <= 1); 2||a_j|| < 2^exS[j]
     if (k == 0) return FX_VBITS - 2 * exS[t];
     if (k == 1) return FX_VBITS - (exS[t] + exS[t + 1]);
     if (k == 2) return FX_VBITS - (exS[t + 1] + 1);
-    return FX_VBITS - (exS[t + 2] + 1);
+    if (k == 3) return FX_VBITS - (exS[t + 2] + 1);
+    return FX_VBITS - (exS[t + 3] + 1);
   };
   // Words of round t: set t mod LEAF_XW_SETS (a round's words are reused only after every
   // CTA has read them: the lookahead values of round t are added two rounds early), one
   // 256-byte line per word so that concurrent atomics and polls land in different L2 slices.
   auto xw_index = [&](int t, int k) -> int { return (t & (LEAF_XW_SETS - 1)) * (LEAF_MAX_W + 2) + k; };
-  auto fx_add = [&](int t, int k, float s) {
-    long long v = __double2ll_rn((double)s * pow2d(fx_exp(t, k)));
+  auto fx_add_scaled = [&](int t, int k, float s, double scale) {
+    long long v = __double2ll_rn((double)s * scale);
     const long long vb = 1ll << FX_VBITS;
     v = v > vb ? vb : (v < -vb ? -vb : v);
     const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
@@ -242,20 +254,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
                      : "memory");
     }
   };
-  auto fx_add_scaled = [&](int t, int k, float s, double scale) {
-    long long v = __double2ll_rn((double)s * scale);
-    const long long vb = 1ll << FX_VBITS;
-    v = v > vb ? vb : (v < -vb ? -vb : v);
-    const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
-    const size_t off = (size_t)xw_index(t, k) * LEAF_XW_STRIDE;
-    if (!p.sys) {
-      asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p.xw + off), "l"(add) : "memory");
-    } else {
-      for (int j = 0; j < p.nranks; ++j)
-        asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(p.xw_peers[j] + off), "l"(add)
-                     : "memory");
-    }
-  };
+  auto fx_add = [&](int t, int k, float s) { fx_add_scaled(t, k, s, fxs[t][k < 4 ? k : 4]); };
   // CTA total of values [0, n) of a [GEMV_PARTS][ld] partial buffer: 4 threads per value, each
   // adds a quarter of the parts, then a 2-level xor tree (fixed order).  Called by all threads;
   // the returned sum is valid on the thread with (threadIdx.x & 3) == 0 of value threadIdx.x >> 2.
@@ -271,19 +270,27 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     return s;
   };
 
-  // Round layout (t >= 1), R19:  [0] u_t.u_t  [1] u_t.a_{t+1}  [2] q_{t-1}.a_{t+1}
-  // [3+i] q_i.a_{t+2} (i <= t-1).  Values [3+i], i <= t-2 ("lookahead") only need q's known
-  // two rounds earlier: they are computed AND added to round t's words during round t-2's
-  // exchange.  Round t's critical values [0], [1], [2], [3+t-1] are formed in one pass over
-  // the rows right after round t-1's scalars.  After round t every CTA knows r_{i,t+2}
-  // (i <= t-1) and subtracts those projections from a_{t+2} while round t+1's exchange is in
-  // flight; after that exchange only q_t and q_{t+1} remain to be subtracted.
+  // Round layout (t >= 1), R19/R22:
+  //   [0] u_t.u_t   [1] u_t.a_{t+1}   [2] q_{t-1}.a_{t+1}   [3] q_{t-1}.a_{t+2}
+  //   [4+i] q_i.a_{t+3}  (i <= t-1)
+  // [0..3] and [4+(t-1)] are the CRITICAL values, formed in one pass over the rows right after
+  // round t-1's scalars; [4+i], i <= t-2 ("lookahead") only need q's known two rounds earlier
+  // and are computed AND added during round t-2's exchange.  After round t every CTA knows
+  //   r_tt, r_{t,t+1} = [1]/r_tt, r_{t-1,t+1} = [2], r_{t-1,t+2} = [3], r_{i,t+3} = [4+i],
+  // and forms  u_{t+1} = w_{t+1} - q_{t-2} r_{t-2,t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1},
+  // where the projected column w_j = a_j - sum_{i <= j-4} q_i r_ij was formed two rounds
+  // earlier (after round j-3) into a ring of LEAF_WRING smem columns, so that the projection
+  // has a whole round of slack and never sits between an exchange and the next row pass.
+  // The original a_j stay in place (CGS takes every r_ij from the original column,
+  // PAPER.md:109) until u_j overwrites them.
   auto round_len = [&](int t) -> int {
     if (t == 0) return w + (w > 1 ? 1 : 0);
-    if (t == w - 1) return 1;
-    if (t == w - 2) return 3;
-    return t + 3;
+    if (t + 3 < w) return t + 4;
+    if (t + 2 < w) return 4;
+    if (t + 1 < w) return 3;
+    return 1;
   };
+  float* wring = sp + (size_t)w * LD;               // [LEAF_WRING][LD] projected columns
   // ---- round 0 vector: [ ||a_k||^2 (k < w), a_0^T a_1 ]: counter barrier + fixed-order gather
   //      (its column norms fix the fixed-point scales of the later rounds) ----
   // (r0_mode 2: the globally reduced round-0 vector is given in p.r0buf)
@@ -345,248 +352,358 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     exS[k] = ex;
     tauc[k] = (float)p.m_global * u_work * sqrtf(s);
   }
+  __syncthreads();
+  // fixed-point scales 2^fx_exp(t, class) and their inverses, value classes 0..4 (fx_exp)
+  for (int i = threadIdx.x; i < w * 5; i += LEAF_THREADS) {
+    const int t = i / 5, c = i - t * 5;
+    const int need = c <= 1 ? t + c : (c == 2 ? t + 1 : (c == 3 ? t + 2 : t + 3));   // last column used
+    const int e = need < w ? fx_exp(t, c) : 0;
+    fxs[t][c] = pow2d(e);
+    fxi[t][c] = pow2d(-e);
+  }
   // (the __syncthreads at the top of the round loop publishes exS / tauc)
 
-  // Warp roles inside a round (all warps own rows: thread-per-row in the row pass and the
-  // projection, warp-per-32-row-block in the lookahead GEMV, so every phase of warp v only
-  // touches the rows [32v + 512k, 32v + 512k + 32) it wrote itself and needs no CTA barrier):
-  //   CRIT_W reduces the critical partials (named barrier 1, the other warps only arrive)
-  //   LA_W   reduces the lookahead partials (named barrier 2)
-  // Only the exchange result is broadcast with a full barrier.  tot[] is double- and coef[]
-  // triple-buffered because a warp may run one round ahead of a slower one.
-  constexpr int CRIT_W = LEAF_WARPS - 1, LA_W = LEAF_WARPS - 2;
-  const int row_warps = rows >= LEAF_THREADS ? LEAF_WARPS : (rows + 31) / 32;   // warps owning rows
-  unsigned long long pre = 0;                      // prefetched exchange word (pollers)
-  bool have_pre = false;
-  for (int t = 0; t < w; ++t) {
-    DBG_STAMP(0);
-    if (t > 0) {
-      // ---- round t's exchange: each value's word is polled by its thread until all
-      //      ranks x G CTAs have added (lookahead words are complete long before) ----
-      const int L = round_len(t);
-      if (threadIdx.x < L) {
-        const int k = threadIdx.x;
-        const int widx = xw_index(t, k);
+  // Warp specialisation (the 3-deep round layout above makes it legal):
+  //   CRITICAL group, warps [0, 8):  poll round t -> scalars -> row pass (u_{t+1}, q_t, round
+  //     t+1's critical dots) -> publish -> poll round t+1 ...   (rows ctid + 256k)
+  //   BULK group, warps [8, 16):  after q_t is in shared memory: round t+2's lookahead dots and
+  //     the projection w_{t+3}, concurrently with the critical group's next rounds.
+  // The groups hand off through producer/consumer named barriers (one per direction and
+  // round parity, so that a group can never arrive twice on a barrier its partner has not
+  // yet waited on -- each direction's round t+2 depends on the other direction's round t):
+  //   BAR_Q + (t&1): critical arrives once q_0..q_t (and coef of round t) are in smem, the
+  //                  bulk waits before its round t;
+  //   BAR_W + (t&1): the bulk arrives after its round t (w_{t+3} in the ring), the critical
+  //                  group waits before its row pass after round t+2.
+  // Barriers order shared memory without draining the threads' outstanding global stores
+  // (a release store would).  Within a group: named barrier 1 (critical), 3 (lookahead
+  // reduction); CRIT_W reduces the critical partials, LA_W the lookahead partials.
+  constexpr int GROUP = LEAF_THREADS / 2, GROUP_W = LEAF_WARPS / 2;
+  constexpr int CRIT_W = GROUP_W - 1, LA_W = LEAF_WARPS - 1;
+  const bool is_crit = threadIdx.x < GROUP;
+  const int crit_warps = rows >= GROUP ? GROUP_W : (rows + 31) / 32;   // critical warps owning rows
+  constexpr int BAR_Q = 4, BAR_W = 6;
+  if (is_crit) {
+    // row state of this thread's rows rr[j] = tid + 256 j, j < NR
+    int rr[NR];
+    bool vr[NR];
+    float ru[NR], rq1[NR], rq2[NR], ra2[NR], ra3[NR];
+#pragma unroll
+    for (int j = 0; j < NR; ++j) {
+      rr[j] = threadIdx.x + GROUP * j;
+      vr[j] = rr[j] < rows;
+      ru[j] = vr[j] ? sp[rr[j]] : 0.0f;                              // u_0 = a_0
+      ra2[j] = (vr[j] && w > 2) ? sp[2 * LD + rr[j]] : 0.0f;
+      ra3[j] = (vr[j] && w > 3) ? sp[3 * LD + rr[j]] : 0.0f;
+      rq1[j] = rq2[j] = 0.0f;
+    }
+    for (int t = 0; t < w; ++t) {
+      DBG_STAMP(0);
+      if (t > 0) {
+        // ---- round t's exchange: each of the (at most 4) values the scalars need is polled
+        //      by its thread until all ranks x G CTAs have added; values [4+i] (coefficients
+        //      of the projection) are polled by the bulk group ----
+        const int L = min(round_len(t), 4);
+        if (threadIdx.x < L) {
+          const int k = threadIdx.x;
+          const int widx = xw_index(t, k);
+          const unsigned cnt = (unsigned)(p.nranks * G);
+          const unsigned long long* wp = p.xw + (size_t)widx * LEAF_XW_STRIDE;
+          const unsigned long long prev = xprev[widx];
+          unsigned long long now = ld_word(wp, p.sys), d = now - prev;
+          long long spins = 0;
+          while ((unsigned)(d >> FX_CNT_SHIFT) != cnt) {
+            if (p.poll_sleep_ns) __nanosleep(p.poll_sleep_ns);
+            now = ld_word(wp, p.sys);
+            d = now - prev;
+            if (++spins > (1ll << 22)) {            // ~seconds: a peer is missing -- fail, never hang
+              atomicExch(p.breakdown, -2);
+              break;
+            }
+          }
+          xprev[widx] = now;
+          if (p.dbg2 != nullptr && k == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 1] = gtimer();
+          const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
+          const float val = (float)((double)total * fxi[t][k]);
+          tot[t & 1][k] = val;
+        }
+      }
+      // the row pass after round t reads w_{t+1}, projected by the bulk after round t-2: wait
+      // for that bulk round (this barrier also publishes the polled values to the group)
+      if (t >= 2 && t + 1 < w)
+        bar_sync_n(BAR_W + (t & 1), LEAF_THREADS);
+      else
+        bar_sync_n(1, GROUP);
+      DBG_STAMP(1);
+      // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{t,t+1}, r_{t-1,t+1}, r_{t-2,t+1} ----
+      const bool more = t + 1 < w;
+      const float* tt = tot[t & 1];
+      const float uu = tt[0];
+      const float ua = (t == 0) ? ((w > 1) ? tt[w] : 0.0f) : (more ? tt[1] : 0.0f);
+      const float c1 = (t >= 1 && more) ? tt[2] : 0.0f;    // r_{t-1,t+1} = q_{t-1}^T a_{t+1}
+      const float c2 = (t >= 2 && more) ? tot[(t - 1) & 1][3] : 0.0f;   // r_{t-2,t+1} (round t-1)
+      float rtt = sqrtf(uu);
+      const float tau = tauc[t];
+      const bool bad = !(rtt > tau) || !isfinite(rtt);
+      const float inv = bad ? 0.0f : __frcp_rn(rtt);     // == 1/rtt (correctly rounded)
+      if (bad) rtt = 0.0f;
+      const float ct = ua * inv;                            // r_{t,t+1}
+      if (g == 0) {
+        if (threadIdx.x == 0) {
+          p.R[t + (int64_t)t * p.ldr] = rtt;
+          if (bad) atomicMin(p.breakdown, (int)(p.col_offset + t));
+          if (more) p.R[t + (int64_t)(t + 1) * p.ldr] = ct;
+        } else if (threadIdx.x == 1) {
+          if (t >= 1 && more) p.R[(t - 1) + (int64_t)(t + 1) * p.ldr] = c1;
+          if (t >= 1 && t + 2 < w) p.R[(t - 1) + (int64_t)(t + 2) * p.ldr] = tt[3];   // r_{t-1,t+2}
+        }
+        if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
+      }
+      DBG_STAMP(2);
+      // ---- one pass over this thread's (at most 2) rows, both rows interleaved, the row
+      //      state in registers (u_t, q_{t-1}, q_{t-2}, a_{t+2}, a_{t+3}):
+      //      q_t = u_t / r_tt (to smem for the bulk group, rounded to global Q),
+      //      u_{t+1} = w_{t+1} - q_{t-2} r_{t-2,t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1}
+      //      (w_{t+1} = a_{t+1} for t+1 <= 3), and round t+1's critical dots
+      //      u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2}, q_t.a_{t+2}, q_t.a_{t+3}, q_t.a_{t+4} ----
+      const bool h2 = t + 2 < w, h3 = t + 3 < w, h4 = t + 4 < w;
+      float s0, s1, s2, s3;
+      {
+        const float* wsrc = (t + 1 <= 3) ? sp + (more ? t + 1 : t) * LD : wring + ((t + 1) % LEAF_WRING) * LD;
+        const float* a4p = sp + (h4 ? t + 4 : t) * LD;
+        float* ut = sp + t * LD;
+        float wv[NR], a4v[NR], q[NR], av[NR];
+#pragma unroll
+        for (int j = 0; j < NR; ++j) {
+          const int r = rr[j];
+          wv[j] = (vr[j] && more) ? wsrc[r] : 0.0f;
+          a4v[j] = (vr[j] && h4) ? a4p[r] : 0.0f;
+        }
+#pragma unroll
+        for (int j = 0; j < NR; ++j) {
+          q[j] = ru[j] * inv;
+          float x = fmaf(-rq2[j], c2, wv[j]);
+          x = fmaf(-rq1[j], c1, x);
+          av[j] = fmaf(-q[j], ct, x);
+        }
+#pragma unroll
+        for (int j = 0; j < NR; ++j)
+          if (vr[j]) ut[rr[j]] = q[j];   // Q goes to global memory at the end
+        s0 = s1 = s2 = s3 = 0.0f;
+#pragma unroll
+        for (int j = 0; j < NR; ++j) {
+          s0 = fmaf(av[j], av[j], s0);
+          s1 = fmaf(av[j], ra2[j], s1);
+          s2 = fmaf(q[j], ra2[j], s2);
+          s3 = fmaf(q[j], ra3[j], s3);
+        }
+#pragma unroll
+        for (int j = 0; j < NR; ++j) {
+          rq2[j] = rq1[j];
+          rq1[j] = q[j];
+          ru[j] = av[j];
+          ra2[j] = ra3[j];
+          ra3[j] = a4v[j];
+        }
+      }
+      if (!more) break;
+      // the critical reducer's lane 4c (c < 5) adds value c of round t+1: its fixed-point scale now
+      const int n_crit = !h2 ? 1 : (!h3 ? 3 : 4);   // critical values of round t+1
+      double crit_scale = 0.0;
+      if (warp == CRIT_W && (lane & 7) == 0 && (lane >> 3) < n_crit) crit_scale = fxs[t + 1][lane >> 3];
+      // warp sums of the 5 critical values: a transposing butterfly (6 shuffles) leaves value k
+      // < 4 in lane 8k, an xor tree the fifth (fixed tree per value)
+      {
+        const bool b16 = lane & 16, b8 = lane & 8;
+        float k0 = b16 ? s2 : s0, k1 = b16 ? s3 : s1;
+        const float x0 = b16 ? s0 : s2, x1 = b16 ? s1 : s3;
+        k0 += __shfl_xor_sync(0xffffffffu, x0, 16);
+        k1 += __shfl_xor_sync(0xffffffffu, x1, 16);
+        float kk = b8 ? k1 : k0;
+        kk += __shfl_xor_sync(0xffffffffu, b8 ? k0 : k1, 8);
+        kk += __shfl_xor_sync(0xffffffffu, kk, 4);
+        kk += __shfl_xor_sync(0xffffffffu, kk, 2);
+        kk += __shfl_xor_sync(0xffffffffu, kk, 1);
+        if ((lane & 7) == 0) cpart[warp][lane >> 3] = kk;
+      }
+      DBG_STAMP(3);
+      bar_sync_n(1, GROUP);
+      // q_0..q_t (and coef of round t) are in smem: release the bulk group for round t
+      if (t + 3 < w) bar_arrive_n(BAR_Q + (t & 1), LEAF_THREADS);
+      // ---- publish round t+1's critical values [0..3] and [4 + t] (warp CRIT_W) ----
+      if (warp == CRIT_W) {
+        const int c = lane >> 3, j = lane & 7;
+        float s = j < crit_warps ? cpart[j][c] : 0.0f;
+        s += __shfl_xor_sync(0xffffffffu, s, 4);
+        s += __shfl_xor_sync(0xffffffffu, s, 2);
+        s += __shfl_xor_sync(0xffffffffu, s, 1);
+        if (j == 0 && c < n_crit) fx_add_scaled(t + 1, c, s, crit_scale);
+        if (p.dbg != nullptr && blockIdx.x == DBG_CTA && lane == 0) p.dbg[(size_t)t * 8 + 7] = clock64();
+        if (p.dbg2 != nullptr && lane == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 0] = gtimer();
+      }
+      DBG_STAMP(4);
+    }
+  } else {
+    // ---- BULK group: for each round t, after q_t is in smem:
+    //      (a) round t+2's lookahead values q_i.a_{t+5}, i <= t (index 4 + i), over this warp's
+    //          32-row blocks (lane = i), reduced by warp LA_W and added to round t+2's words;
+    //      (b) w_{t+3} = a_{t+3} - sum_{i <= t-1} q_i r_{i,t+3}  (coefficients of round t) into
+    //          the ring; the critical group first reads it after round t+2 ----
+    const int btid = threadIdx.x - GROUP, bw = warp - GROUP_W;
+    for (int t = 0; t + 3 < w; ++t) {
+      bar_sync_n(BAR_Q + (t & 1), LEAF_THREADS);
+      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 8 + 5] = clock64();
+      // round t's values [4+i] = r_{i,t+3}, i <= t-1: round t is complete (the critical group
+      // has seen it); the loads are issued now and checked after the dot products below
+      const int pk = 4 + btid;
+      const int pidx = xw_index(t, pk);
+      const unsigned long long* pwp = p.xw + (size_t)pidx * LEAF_XW_STRIDE;
+      unsigned long long pnow = 0;
+      if (btid < t) pnow = ld_word(pwp, p.sys);
+      if (t + 4 < w) {
+        // (a') q_t.a_{t+4}: round t+1's value [4+t] (it only feeds the projection of w_{t+4},
+        //      so it is kept off the critical group's reduction)
+        float e = 0.f;
+        {
+          const float* qt = sp + t * LD;
+          const float* a4 = sp + (t + 4) * LD;
+          for (int r = 32 * bw + lane; r < rows; r += GROUP) e = fmaf(qt[r], a4[r], e);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
+        const int cnt = t + 5 < w ? t + 1 : 0;              // (a): i in [0, t]
+        const bool ha = kq < cnt, hb = kq + 32 < cnt;
+        float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+        if (ha && !(p.skip & 2)) {
+          const float4* y = reinterpret_cast<const float4*>(sp + (t + 5) * LD);
+          const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
+          const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
+          // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
+          for (int base = 8 * bw; base < nv4; base += 8 * GROUP_W) {
+#pragma unroll
+            for (int i = base; i < base + 8; ++i) {
+              const float4 yy = y[i], a = xa[i];
+              a0 = fmaf(a.x, yy.x, a0);
+              a1 = fmaf(a.y, yy.y, a1);
+              a0 = fmaf(a.z, yy.z, a0);
+              a1 = fmaf(a.w, yy.w, a1);
+              if (hb) {
+                const float4 b = xb[i];
+                b0 = fmaf(b.x, yy.x, b0);
+                b1 = fmaf(b.y, yy.y, b1);
+                b0 = fmaf(b.z, yy.z, b0);
+                b1 = fmaf(b.w, yy.w, b1);
+              }
+            }
+          }
+        }
+        part[bw][kq] = a0 + a1;
+        part[bw][kq + 32] = b0 + b1;
+        if (lane == 0) part[bw][64] = e;
+        if (warp == LA_W) {
+          bar_sync_n(3, GROUP);
+          float sa = 0.f, sb = 0.f, se = 0.f;
+#pragma unroll
+          for (int v = 0; v < GROUP_W; ++v) {
+            sa += part[v][lane];
+            sb += part[v][lane + 32];
+            se += part[v][64];
+          }
+          if (lane < cnt) fx_add(t + 2, 4 + lane, sa);
+          if (lane + 32 < cnt) fx_add(t + 2, 4 + lane + 32, sb);
+          if (lane == 0) fx_add(t + 1, 4 + t, se);
+        } else {
+          bar_arrive_n(3, GROUP);
+        }
+      }
+      if (btid < t) {
         const unsigned cnt = (unsigned)(p.nranks * G);
-        const unsigned long long* wp = p.xw + (size_t)widx * LEAF_XW_STRIDE;
-        const unsigned long long prev = xprev[widx];
-        unsigned long long now = have_pre ? pre : ld_word(wp, p.sys), d = now - prev;
+        const unsigned long long prev = xprev[pidx];
+        unsigned long long d = pnow - prev;
         long long spins = 0;
         while ((unsigned)(d >> FX_CNT_SHIFT) != cnt) {
-          if (p.poll_sleep_ns) __nanosleep(p.poll_sleep_ns);
-          now = ld_word(wp, p.sys);
-          d = now - prev;
-          if (++spins > (1ll << 22)) {            // ~seconds: a peer is missing -- fail, never hang
+          pnow = ld_word(pwp, p.sys);
+          d = pnow - prev;
+          if (++spins > (1ll << 22)) {
             atomicExch(p.breakdown, -2);
             break;
           }
         }
-        xprev[widx] = now;
-        if (p.dbg2 != nullptr && k == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 1] = gtimer();
+        xprev[pidx] = pnow;
         const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
-        const float val = (float)((double)total * pow2d(-fx_exp(t, k)));
-        tot[t & 1][k] = val;
-        if (k >= 3) coef[t % 3][k - 3] = val;
+        const float val = (float)((double)total * fxi[t][4]);
+        coef[t % 3][btid] = val;
+        if (g == 0) p.R[btid + (int64_t)(t + 3) * p.ldr] = val;
       }
-    }
-    __syncthreads();
-    DBG_STAMP(1);
-    // ---- scalars (every thread, identical): r_tt, 1/r_tt, r_{t,t+1}, r_{t-1,t+1} ----
-    const bool more = t + 1 < w;
-    const float* tt = tot[t & 1];
-    const float uu = tt[0];
-    const float ua = (t == 0) ? ((w > 1) ? tt[w] : 0.0f) : (more ? tt[1] : 0.0f);
-    const float cq = (t >= 1 && more) ? tt[2] : 0.0f;    // r_{t-1,t+1} = q_{t-1}^T a_{t+1}
-    float rtt = sqrtf(uu);
-    const float tau = tauc[t];
-    const bool bad = !(rtt > tau) || !isfinite(rtt);
-    const float inv = bad ? 0.0f : 1.0f / rtt;
-    if (bad) rtt = 0.0f;
-    const float ct = ua * inv;                            // r_{t,t+1}
-    if (g == 0) {
-      if (threadIdx.x == 0) {
-        p.R[t + (int64_t)t * p.ldr] = rtt;
-        if (bad) atomicMin(p.breakdown, (int)(p.col_offset + t));
-      }
-      if (more && threadIdx.x <= t) {
-        const int i = threadIdx.x;
-        const float r = (i == t) ? ct : (i == t - 1) ? cq : coef[(t + 2) % 3][i];   // i <= t-2: round t-1
-        p.R[i + (int64_t)(t + 1) * p.ldr] = r;
-      }
-      if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
-    }
-    DBG_STAMP(2);
-    // ---- one pass over this thread's rows:  q_t = u_t / r_tt (stored rounded),
-    //      u_{t+1} = w_{t+1} - q_{t-1} r_{t-1,t+1} - q_t r_{t,t+1}, where w_{t+1} = a_{t+1} -
-    //      sum_{i<=t-2} q_i r_{i,t+1} was formed during round t-1; and round t+1's critical
-    //      dots u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2}, q_t.a_{t+2}, q_t.a_{t+3} ----
-    const bool h2 = t + 2 < w, h3 = t + 3 < w;
-    float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
-    {
-      float* ut = sp + t * LD;
-      float* an = sp + (more ? t + 1 : t) * LD;
-      const float* qp = sp + (t >= 1 ? t - 1 : 0) * LD;
-      const float* a2 = sp + (h2 ? t + 2 : t) * LD;
-      const float* a3 = sp + (h3 ? t + 3 : t) * LD;
-      T* qdst = P + r0 + (int64_t)t * p.ldp;
-      for (int r = threadIdx.x; r < rows; r += LEAF_THREADS) {
-        // all loads first (the columns are distinct whenever their values are used)
-        const float uv = ut[r], av0 = an[r], qpv = qp[r], a2v = a2[r], a3v = a3[r];
-        const float q = uv * inv;
-        ut[r] = q;
-        qdst[r] = Elem<T>::store(q);
-        if (more) {
-          float av = av0;
-          if (t >= 1) av = fmaf(-qpv, cq, av);
-          av = fmaf(-q, ct, av);
-          an[r] = av;
-          s0 = fmaf(av, av, s0);
-          if (h2) {
-            s1 = fmaf(av, a2v, s1);
-            s2 = fmaf(q, a2v, s2);
-            if (h3) s3 = fmaf(q, a3v, s3);
-          }
-        }
-      }
-    }
-    if (!more) break;
-    // the critical reducer's lane 8c will add value c of round t+1: its fixed-point scale now
-    double crit_scale = 0.0;
-    if (warp == CRIT_W && (lane & 7) == 0) {
-      const int c = lane >> 3;
-      crit_scale = pow2d(fx_exp(t + 1, c < 3 ? c : 3 + t));
-    }
-    // warp sums of the 4 critical values by a transposing butterfly (6 shuffles): afterwards
-    // lane 8k holds value k (fixed tree per value)
-    {
-      const bool b16 = lane & 16, b8 = lane & 8;
-      float k0 = b16 ? s2 : s0, k1 = b16 ? s3 : s1;
-      const float x0 = b16 ? s0 : s2, x1 = b16 ? s1 : s3;
-      k0 += __shfl_xor_sync(0xffffffffu, x0, 16);
-      k1 += __shfl_xor_sync(0xffffffffu, x1, 16);
-      float kk = b8 ? k1 : k0;
-      kk += __shfl_xor_sync(0xffffffffu, b8 ? k0 : k1, 8);
-      kk += __shfl_xor_sync(0xffffffffu, kk, 4);
-      kk += __shfl_xor_sync(0xffffffffu, kk, 2);
-      kk += __shfl_xor_sync(0xffffffffu, kk, 1);
-      if ((lane & 7) == 0) cpart[warp][lane >> 3] = kk;
-    }
-    DBG_STAMP(3);
-    // ---- publish round t+1's critical values [0], [1], [2] and [3 + t] (warp CRIT_W) right
-    //      after the barrier, before the other warps' lookahead loads fill the smem pipe ----
-    __syncthreads();
-    if (warp == CRIT_W) {
-      const int n = !h2 ? 1 : (!h3 ? 3 : 4);
-      const int c = lane >> 3, j = lane & 7;
-      float s = 0.f;
-      if (j < row_warps) s = cpart[j][c];
-      if (j + 8 < row_warps) s += cpart[j + 8][c];
-      s += __shfl_xor_sync(0xffffffffu, s, 4);
-      s += __shfl_xor_sync(0xffffffffu, s, 2);
-      s += __shfl_xor_sync(0xffffffffu, s, 1);
-      if (j == 0 && c < n) fx_add_scaled(t + 1, c < 3 ? c : 3 + t, s, crit_scale);
-      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && lane == 0) p.dbg[(size_t)t * 8 + 7] = clock64();
-      if (p.dbg2 != nullptr && lane == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 0] = gtimer();
-    }
-    DBG_STAMP(4);
-    // ---- while round t+1's exchange is in flight:
-    //      (a) round t+2's lookahead values q_i.a_{t+4}, i <= t (index 3 + i), over this warp's
-    //          row blocks (lane = i), reduced by warp LA_W and added to round t+2's words now;
-    //      (b) w_{t+2} = a_{t+2} - sum_{i <= t-1} q_i r_{i,t+2}  (coefficients from round t) ----
-    if (t + 4 < w) {
-      const int cnt = t + 1;                              // i in [0, t]
-      const bool ha = kq < cnt, hb = kq + 32 < cnt;
-      float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
-      if (ha && !(p.skip & 2)) {
-        const float4* y = reinterpret_cast<const float4*>(sp + (t + 4) * LD);
-        const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
-        const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
-        // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
-        for (int base = 8 * warp; base < nv4; base += LEAF_THREADS / 4) {
+      bar_sync_n(2, GROUP);
+      if (t >= 1 && !(p.skip & 4)) {
+        // thread-per-row: w_{t+3}[r] = a_{t+3}[r] - sum_{i < t} q_i[r] r_{i,t+3}  (two fixed-order
+        // partial sums)
+        const float* cf = coef[t % 3];
+        const float* an = sp + (t + 3) * LD;
+        float* wd = wring + ((t + 3) % LEAF_WRING) * LD;
+        // this thread's rows btid + 256 j, j < NR, interleaved (independent chains)
+        float e0[NR], e1[NR];
+        int rb[NR];
 #pragma unroll
-          for (int i = base; i < base + 8; ++i) {
-            const float4 yy = y[i], a = xa[i];
-            a0 = fmaf(a.x, yy.x, a0);
-            a1 = fmaf(a.y, yy.y, a1);
-            a0 = fmaf(a.z, yy.z, a0);
-            a1 = fmaf(a.w, yy.w, a1);
-            if (hb) {
-              const float4 b = xb[i];
-              b0 = fmaf(b.x, yy.x, b0);
-              b1 = fmaf(b.y, yy.y, b1);
-              b0 = fmaf(b.z, yy.z, b0);
-              b1 = fmaf(b.w, yy.w, b1);
-            }
+        for (int j = 0; j < NR; ++j) {
+          e0[j] = e1[j] = 0.f;
+          rb[j] = min(btid + GROUP * j, LD - 1);       // rows >= `rows` are computed, not stored
+        }
+        int k = 0;
+        for (; k + 4 <= t; k += 4) {
+          const float4 c0 = *reinterpret_cast<const float4*>(cf + k);
+#pragma unroll
+          for (int j = 0; j < NR; ++j) {
+            const float x0 = sp[(k + 0) * LD + rb[j]], x1 = sp[(k + 1) * LD + rb[j]],
+                        x2 = sp[(k + 2) * LD + rb[j]], x3 = sp[(k + 3) * LD + rb[j]];
+            e0[j] = fmaf(x0, c0.x, e0[j]);
+            e1[j] = fmaf(x1, c0.y, e1[j]);
+            e0[j] = fmaf(x2, c0.z, e0[j]);
+            e1[j] = fmaf(x3, c0.w, e1[j]);
           }
         }
-      }
-      if (warp < row_warps) {
-        part[warp][kq] = a0 + a1;
-        part[warp][kq + 32] = b0 + b1;
-      }
-      if (warp == LA_W) {
-        bar_sync_n(2, LEAF_THREADS);
-        float sa = 0.f, sb = 0.f;
-        for (int v = 0; v < row_warps; ++v) {
-          sa += part[v][lane];
-          sb += part[v][lane + 32];
+        for (; k < t; ++k) {
+          const float c0 = cf[k];
+#pragma unroll
+          for (int j = 0; j < NR; ++j) e0[j] = fmaf(sp[k * LD + rb[j]], c0, e0[j]);
         }
-        if (lane < cnt) fx_add(t + 2, 3 + lane, sa);
-        if (lane + 32 < cnt) fx_add(t + 2, 3 + lane + 32, sb);
-      } else {
-        bar_arrive_n(2, LEAF_THREADS);
+#pragma unroll
+        for (int j = 0; j < NR; ++j)
+          if (btid + GROUP * j < rows) wd[rb[j]] = an[rb[j]] - (e0[j] + e1[j]);
       }
+      bar_arrive_n(BAR_W + (t & 1), LEAF_THREADS);
+      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 8 + 6] = clock64();
     }
-    DBG_STAMP(5);
-    // prefetch round t+1's words: the load is in flight during the projection below
-    {
-      const int L1 = round_len(t + 1);
-      have_pre = threadIdx.x < L1;
-      if (have_pre) pre = ld_word(p.xw + (size_t)xw_index(t + 1, threadIdx.x) * LEAF_XW_STRIDE, p.sys);
+  }
+  __syncthreads();
+  // ---- Q: the panel slice (now q_0..q_{w-1} in fp32) rounded once to the storage type ----
+  {
+    constexpr int V = Vec<T>::N;
+    const int nvec = p.vec_ok ? rows / V : 0;
+    for (int idx = threadIdx.x; idx < w * nvec; idx += LEAF_THREADS) {
+      const int j = idx / nvec, i = (idx - j * nvec) * V;
+#pragma unroll
+      for (int e = 0; e < V; e += 4)
+        store4<T>(P + r0 + i + e + (int64_t)j * p.ldp, *reinterpret_cast<const float4*>(sp + j * LD + i + e));
     }
-    if (t + 2 < w && t >= 1 && !(p.skip & 4)) {
-      // thread-per-row: w_{t+2}[r] -= sum_{i < t} q_i[r] r_{i,t+2}  (two fixed-order partial sums)
-      const float* cf = coef[t % 3];
-      float* an = sp + (t + 2) * LD;
-      for (int r = threadIdx.x; r < rows; r += LEAF_THREADS) {
-        float e0 = 0.f, e1 = 0.f;
-        int k = 0;
-        for (; k + 8 <= t; k += 8) {
-          const float4 c0 = *reinterpret_cast<const float4*>(cf + k);
-          const float4 c1 = *reinterpret_cast<const float4*>(cf + k + 4);
-          const float x0 = sp[(k + 0) * LD + r], x1 = sp[(k + 1) * LD + r], x2 = sp[(k + 2) * LD + r],
-                      x3 = sp[(k + 3) * LD + r], x4 = sp[(k + 4) * LD + r], x5 = sp[(k + 5) * LD + r],
-                      x6 = sp[(k + 6) * LD + r], x7 = sp[(k + 7) * LD + r];
-          e0 = fmaf(x0, c0.x, e0);
-          e1 = fmaf(x1, c0.y, e1);
-          e0 = fmaf(x2, c0.z, e0);
-          e1 = fmaf(x3, c0.w, e1);
-          e0 = fmaf(x4, c1.x, e0);
-          e1 = fmaf(x5, c1.y, e1);
-          e0 = fmaf(x6, c1.z, e0);
-          e1 = fmaf(x7, c1.w, e1);
-        }
-        for (; k + 2 <= t; k += 2) {
-          e0 = fmaf(sp[k * LD + r], cf[k], e0);
-          e1 = fmaf(sp[(k + 1) * LD + r], cf[k + 1], e1);
-        }
-        if (k < t) e0 = fmaf(sp[k * LD + r], cf[k], e0);
-        an[r] -= e0 + e1;
-      }
+    const int span = rows - nvec * V;
+    for (int idx = threadIdx.x; idx < w * span; idx += LEAF_THREADS) {
+      const int j = idx / span, i = nvec * V + (idx - j * span);
+      P[r0 + i + (int64_t)j * p.ldp] = Elem<T>::store(sp[j * LD + i]);
     }
-    DBG_STAMP(6);
   }
   // every CTA ends with the same last-seen words; CTA 0 persists them for the next launch
   if (g == 0)
     for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) p.xprev_g[i] = xprev[i];
 }
 
-template <typename T>
-cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
-  const size_t smem = (size_t)p.w * leaf_ld(p.rows_per_cta) * sizeof(float);
+template <typename T, int NR>
+static cudaError_t launch_leaf_nr(const LeafParams& p, int grid, cudaStream_t st) {
+  const size_t smem = (size_t)(p.w + LEAF_WRING) * leaf_ld(p.rows_per_cta) * sizeof(float);
   static size_t attr_smem = 0;
   if (smem > attr_smem) {
-    cudaError_t e = cudaFuncSetAttribute(leaf_cgs_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(leaf_cgs_kernel<T, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)smem);
     if (e != cudaSuccess) return e;
     attr_smem = smem;
@@ -603,10 +720,19 @@ cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
   attr[0].val.cooperative = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, leaf_cgs_kernel<T>, p);
+  return cudaLaunchKernelEx(&cfg, leaf_cgs_kernel<T, NR>, p);
 }
 
-int leaf_max_smem_rows(int w) { return (int)((LEAF_SMEM_BUDGET) / ((size_t)w * sizeof(float))); }
+template <typename T>
+cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
+  const int per = (p.rows_per_cta + LEAF_THREADS / 2 - 1) / (LEAF_THREADS / 2);
+  if (per <= 2) return launch_leaf_nr<T, 2>(p, grid, st);
+  if (per <= 4) return launch_leaf_nr<T, 4>(p, grid, st);
+  if (per <= 8) return launch_leaf_nr<T, 8>(p, grid, st);
+  return cudaErrorInvalidValue;   // rows_per_cta > LEAF_MAX_RP: rejected by op_leaf
+}
+
+int leaf_max_smem_rows(int w) { return (int)((LEAF_SMEM_BUDGET) / ((size_t)(w + LEAF_WRING) * sizeof(float))); }
 
 template cudaError_t launch_leaf<__half>(const LeafParams&, int, cudaStream_t);
 template cudaError_t launch_leaf<__nv_bfloat16>(const LeafParams&, int, cudaStream_t);
