@@ -149,8 +149,9 @@ __device__ __forceinline__ void store4<float>(float* dst, float4 v) {
   *reinterpret_cast<float4*>(dst) = v;
 }
 
-// NR: rows per critical-group thread (rows_per_cta <= 256 NR)
-template <typename T, int NR>
+// CW: warps of the critical group (the other 16 - CW are the bulk group);
+// NR: rows per critical-group thread (rows_per_cta <= 32 CW NR)
+template <typename T, int NR, int CW>
 __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p) {
   extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
   __shared__ float tot[2][LEAF_MAX_W + 2];         // reduced round vector, by parity of the round
@@ -378,16 +379,17 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   // Barriers order shared memory without draining the threads' outstanding global stores
   // (a release store would).  Within a group: named barrier 1 (critical), 3 (lookahead
   // reduction); CRIT_W reduces the critical partials, LA_W the lookahead partials.
-  constexpr int GROUP = LEAF_THREADS / 2, GROUP_W = LEAF_WARPS / 2;
+  constexpr int GROUP = 32 * CW, GROUP_W = CW;                       // critical group
+  constexpr int BULK = LEAF_THREADS - GROUP, BULK_W = LEAF_WARPS - CW;   // bulk group
   constexpr int CRIT_W = GROUP_W - 1, LA_W = LEAF_WARPS - 1;
   const bool is_crit = threadIdx.x < GROUP;
   const int crit_warps = rows >= GROUP ? GROUP_W : (rows + 31) / 32;   // critical warps owning rows
   constexpr int BAR_Q = 4, BAR_W = 6;
   if (is_crit) {
-    // row state of this thread's rows rr[j] = tid + 256 j, j < NR
+    // row state of this thread's rows rr[j] = tid + 32 CW j, j < NR
     int rr[NR];
     bool vr[NR];
-    float ru[NR], rq1[NR], rq2[NR], ra2[NR], ra3[NR];
+    float ru[NR], rq1[NR], rq2[NR], rq3[NR], ra2[NR], ra3[NR];
 #pragma unroll
     for (int j = 0; j < NR; ++j) {
       rr[j] = threadIdx.x + GROUP * j;
@@ -395,7 +397,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       ru[j] = vr[j] ? sp[rr[j]] : 0.0f;                              // u_0 = a_0
       ra2[j] = (vr[j] && w > 2) ? sp[2 * LD + rr[j]] : 0.0f;
       ra3[j] = (vr[j] && w > 3) ? sp[3 * LD + rr[j]] : 0.0f;
-      rq1[j] = rq2[j] = 0.0f;
+      rq1[j] = rq2[j] = rq3[j] = 0.0f;
     }
     for (int t = 0; t < w; ++t) {
       DBG_STAMP(0);
@@ -403,10 +405,14 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         // ---- round t's exchange: each of the (at most 4) values the scalars need is polled
         //      by its thread until all ranks x G CTAs have added; values [4+i] (coefficients
         //      of the projection) are polled by the bulk group ----
+        // thread 4: r_{t-3,t+1} = value [4+(t-3)] of round t-2 (added by the bulk groups after
+        // round t-3, so normally complete long before)
         const int L = min(round_len(t), 4);
-        if (threadIdx.x < L) {
-          const int k = threadIdx.x;
-          const int widx = xw_index(t, k);
+        const bool late = threadIdx.x == 4 && t >= 3 && t + 1 < w;
+        if (threadIdx.x < L || late) {
+          const int k = late ? 4 + (t - 3) : threadIdx.x;
+          const int tr = late ? t - 2 : t;
+          const int widx = xw_index(tr, k);
           const unsigned cnt = (unsigned)(p.nranks * G);
           const unsigned long long* wp = p.xw + (size_t)widx * LEAF_XW_STRIDE;
           const unsigned long long prev = xprev[widx];
@@ -424,8 +430,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           xprev[widx] = now;
           if (p.dbg2 != nullptr && k == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 1] = gtimer();
           const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
-          const float val = (float)((double)total * fxi[t][k]);
-          tot[t & 1][k] = val;
+          const float val = (float)((double)total * fxi[tr][k < 4 ? k : 4]);
+          tot[t & 1][late ? 4 : k] = val;
         }
       }
       // the row pass after round t reads w_{t+1}, projected by the bulk after round t-2: wait
@@ -442,6 +448,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       const float ua = (t == 0) ? ((w > 1) ? tt[w] : 0.0f) : (more ? tt[1] : 0.0f);
       const float c1 = (t >= 1 && more) ? tt[2] : 0.0f;    // r_{t-1,t+1} = q_{t-1}^T a_{t+1}
       const float c2 = (t >= 2 && more) ? tot[(t - 1) & 1][3] : 0.0f;   // r_{t-2,t+1} (round t-1)
+      const float c3 = (t >= 3 && more) ? tt[4] : 0.0f;    // r_{t-3,t+1} (round t-2)
       float rtt = sqrtf(uu);
       const float tau = tauc[t];
       const bool bad = !(rtt > tau) || !isfinite(rtt);
@@ -456,6 +463,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         } else if (threadIdx.x == 1) {
           if (t >= 1 && more) p.R[(t - 1) + (int64_t)(t + 1) * p.ldr] = c1;
           if (t >= 1 && t + 2 < w) p.R[(t - 1) + (int64_t)(t + 2) * p.ldr] = tt[3];   // r_{t-1,t+2}
+          if (t >= 3 && more) p.R[(t - 3) + (int64_t)(t + 1) * p.ldr] = c3;
         }
         if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
       }
@@ -469,7 +477,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       const bool h2 = t + 2 < w, h3 = t + 3 < w, h4 = t + 4 < w;
       float s0, s1, s2, s3;
       {
-        const float* wsrc = (t + 1 <= 3) ? sp + (more ? t + 1 : t) * LD : wring + ((t + 1) % LEAF_WRING) * LD;
+        const float* wsrc = (t + 1 <= 4) ? sp + (more ? t + 1 : t) * LD : wring + ((t + 1) % LEAF_WRING) * LD;
         const float* a4p = sp + (h4 ? t + 4 : t) * LD;
         float* ut = sp + t * LD;
         float wv[NR], a4v[NR], q[NR], av[NR];
@@ -482,7 +490,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
 #pragma unroll
         for (int j = 0; j < NR; ++j) {
           q[j] = ru[j] * inv;
-          float x = fmaf(-rq2[j], c2, wv[j]);
+          float x = fmaf(-rq3[j], c3, wv[j]);
+          x = fmaf(-rq2[j], c2, x);
           x = fmaf(-rq1[j], c1, x);
           av[j] = fmaf(-q[j], ct, x);
         }
@@ -499,6 +508,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
 #pragma unroll
         for (int j = 0; j < NR; ++j) {
+          rq3[j] = rq2[j];
           rq2[j] = rq1[j];
           rq1[j] = q[j];
           ru[j] = av[j];
@@ -559,7 +569,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       const int pidx = xw_index(t, pk);
       const unsigned long long* pwp = p.xw + (size_t)pidx * LEAF_XW_STRIDE;
       unsigned long long pnow = 0;
-      if (btid < t) pnow = ld_word(pwp, p.sys);
+      if (btid < t - 1) pnow = ld_word(pwp, p.sys);
       if (t + 4 < w) {
         // (a') q_t.a_{t+4}: round t+1's value [4+t] (it only feeds the projection of w_{t+4},
         //      so it is kept off the critical group's reduction)
@@ -567,7 +577,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         {
           const float* qt = sp + t * LD;
           const float* a4 = sp + (t + 4) * LD;
-          for (int r = 32 * bw + lane; r < rows; r += GROUP) e = fmaf(qt[r], a4[r], e);
+          for (int r = 32 * bw + lane; r < rows; r += BULK) e = fmaf(qt[r], a4[r], e);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
@@ -579,7 +589,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
           const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
           // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
-          for (int base = 8 * bw; base < nv4; base += 8 * GROUP_W) {
+          for (int base = 8 * bw; base < nv4; base += 8 * BULK_W) {
 #pragma unroll
             for (int i = base; i < base + 8; ++i) {
               const float4 yy = y[i], a = xa[i];
@@ -600,11 +610,16 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         part[bw][kq] = a0 + a1;
         part[bw][kq + 32] = b0 + b1;
         if (lane == 0) part[bw][64] = e;
+      }
+      // reduction of the lookahead partials (rounds t+1 and t+2); before the projection: the
+      // bulk round's total length gates the critical group through BAR_W
+      if (t + 4 < w) {
+        const int cnt = t + 5 < w ? t + 1 : 0;
         if (warp == LA_W) {
-          bar_sync_n(3, GROUP);
+          bar_sync_n(3, BULK);
           float sa = 0.f, sb = 0.f, se = 0.f;
 #pragma unroll
-          for (int v = 0; v < GROUP_W; ++v) {
+          for (int v = 0; v < BULK_W; ++v) {
             sa += part[v][lane];
             sb += part[v][lane + 32];
             se += part[v][64];
@@ -613,10 +628,10 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           if (lane + 32 < cnt) fx_add(t + 2, 4 + lane + 32, sb);
           if (lane == 0) fx_add(t + 1, 4 + t, se);
         } else {
-          bar_arrive_n(3, GROUP);
+          bar_arrive_n(3, BULK);
         }
       }
-      if (btid < t) {
+      if (btid < t - 1) {
         const unsigned cnt = (unsigned)(p.nranks * G);
         const unsigned long long prev = xprev[pidx];
         unsigned long long d = pnow - prev;
@@ -635,42 +650,57 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         coef[t % 3][btid] = val;
         if (g == 0) p.R[btid + (int64_t)(t + 3) * p.ldr] = val;
       }
-      bar_sync_n(2, GROUP);
-      if (t >= 1 && !(p.skip & 4)) {
+      bar_sync_n(2, BULK);
+      if (t >= 2 && !(p.skip & 4)) {
         // thread-per-row: w_{t+3}[r] = a_{t+3}[r] - sum_{i < t} q_i[r] r_{i,t+3}  (two fixed-order
         // partial sums)
         const float* cf = coef[t % 3];
         const float* an = sp + (t + 3) * LD;
         float* wd = wring + ((t + 3) % LEAF_WRING) * LD;
-        // this thread's rows btid + 256 j, j < NR, interleaved (independent chains)
-        float e0[NR], e1[NR];
-        int rb[NR];
+        // row pairs (2 pi, 2 pi + 1), pi = btid + BULK j: float2 loads, 4 independent chains
+        constexpr int NP = (NR * GROUP + 2 * BULK - 1) / (2 * BULK);
+        const int npairs = (rows + 1) / 2;
+        float2 e0[NP], e1[NP];
+        int pb[NP];
 #pragma unroll
-        for (int j = 0; j < NR; ++j) {
-          e0[j] = e1[j] = 0.f;
-          rb[j] = min(btid + GROUP * j, LD - 1);       // rows >= `rows` are computed, not stored
+        for (int j = 0; j < NP; ++j) {
+          e0[j] = e1[j] = make_float2(0.f, 0.f);
+          pb[j] = 2 * min(btid + BULK * j, LD / 2 - 1);   // pairs >= npairs: computed, not stored
         }
         int k = 0;
-        for (; k + 4 <= t; k += 4) {
+        for (; k + 4 <= t - 1; k += 4) {
           const float4 c0 = *reinterpret_cast<const float4*>(cf + k);
 #pragma unroll
-          for (int j = 0; j < NR; ++j) {
-            const float x0 = sp[(k + 0) * LD + rb[j]], x1 = sp[(k + 1) * LD + rb[j]],
-                        x2 = sp[(k + 2) * LD + rb[j]], x3 = sp[(k + 3) * LD + rb[j]];
-            e0[j] = fmaf(x0, c0.x, e0[j]);
-            e1[j] = fmaf(x1, c0.y, e1[j]);
-            e0[j] = fmaf(x2, c0.z, e0[j]);
-            e1[j] = fmaf(x3, c0.w, e1[j]);
+          for (int j = 0; j < NP; ++j) {
+            const float2 x0 = *reinterpret_cast<const float2*>(sp + (k + 0) * LD + pb[j]);
+            const float2 x1 = *reinterpret_cast<const float2*>(sp + (k + 1) * LD + pb[j]);
+            const float2 x2 = *reinterpret_cast<const float2*>(sp + (k + 2) * LD + pb[j]);
+            const float2 x3 = *reinterpret_cast<const float2*>(sp + (k + 3) * LD + pb[j]);
+            e0[j].x = fmaf(x0.x, c0.x, e0[j].x);
+            e0[j].y = fmaf(x0.y, c0.x, e0[j].y);
+            e1[j].x = fmaf(x1.x, c0.y, e1[j].x);
+            e1[j].y = fmaf(x1.y, c0.y, e1[j].y);
+            e0[j].x = fmaf(x2.x, c0.z, e0[j].x);
+            e0[j].y = fmaf(x2.y, c0.z, e0[j].y);
+            e1[j].x = fmaf(x3.x, c0.w, e1[j].x);
+            e1[j].y = fmaf(x3.y, c0.w, e1[j].y);
           }
         }
-        for (; k < t; ++k) {
+        for (; k < t - 1; ++k) {
           const float c0 = cf[k];
 #pragma unroll
-          for (int j = 0; j < NR; ++j) e0[j] = fmaf(sp[k * LD + rb[j]], c0, e0[j]);
+          for (int j = 0; j < NP; ++j) {
+            const float2 x0 = *reinterpret_cast<const float2*>(sp + k * LD + pb[j]);
+            e0[j].x = fmaf(x0.x, c0, e0[j].x);
+            e0[j].y = fmaf(x0.y, c0, e0[j].y);
+          }
         }
 #pragma unroll
-        for (int j = 0; j < NR; ++j)
-          if (btid + GROUP * j < rows) wd[rb[j]] = an[rb[j]] - (e0[j] + e1[j]);
+        for (int j = 0; j < NP; ++j)
+          if (btid + BULK * j < npairs) {
+            const float2 av = *reinterpret_cast<const float2*>(an + pb[j]);
+            *reinterpret_cast<float2*>(wd + pb[j]) = make_float2(av.x - (e0[j].x + e1[j].x), av.y - (e0[j].y + e1[j].y));
+          }
       }
       bar_arrive_n(BAR_W + (t & 1), LEAF_THREADS);
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 8 + 6] = clock64();
@@ -698,12 +728,12 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) p.xprev_g[i] = xprev[i];
 }
 
-template <typename T, int NR>
+template <typename T, int NR, int CW>
 static cudaError_t launch_leaf_nr(const LeafParams& p, int grid, cudaStream_t st) {
   const size_t smem = (size_t)(p.w + LEAF_WRING) * leaf_ld(p.rows_per_cta) * sizeof(float);
   static size_t attr_smem = 0;
   if (smem > attr_smem) {
-    cudaError_t e = cudaFuncSetAttribute(leaf_cgs_kernel<T, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(leaf_cgs_kernel<T, NR, CW>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)smem);
     if (e != cudaSuccess) return e;
     attr_smem = smem;
@@ -720,15 +750,15 @@ static cudaError_t launch_leaf_nr(const LeafParams& p, int grid, cudaStream_t st
   attr[0].val.cooperative = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, leaf_cgs_kernel<T, NR>, p);
+  return cudaLaunchKernelEx(&cfg, leaf_cgs_kernel<T, NR, CW>, p);
 }
 
 template <typename T>
 cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
-  const int per = (p.rows_per_cta + LEAF_THREADS / 2 - 1) / (LEAF_THREADS / 2);
-  if (per <= 2) return launch_leaf_nr<T, 2>(p, grid, st);
-  if (per <= 4) return launch_leaf_nr<T, 4>(p, grid, st);
-  if (per <= 8) return launch_leaf_nr<T, 8>(p, grid, st);
+  // 8 critical + 8 bulk warps (4 + 12 measured slower at 448 rows per CTA)
+  if (p.rows_per_cta <= 512) return launch_leaf_nr<T, 2, 8>(p, grid, st);
+  if (p.rows_per_cta <= 1024) return launch_leaf_nr<T, 4, 8>(p, grid, st);
+  if (p.rows_per_cta <= 2048) return launch_leaf_nr<T, 8, 8>(p, grid, st);
   return cudaErrorInvalidValue;   // rows_per_cta > LEAF_MAX_RP: rejected by op_leaf
 }
 
