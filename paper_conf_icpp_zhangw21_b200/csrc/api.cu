@@ -152,6 +152,7 @@ int create_impl(rgsqr_handle* h, int device) {
   if (cudaStreamCreateWithFlags(&c->st_own, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_h2d, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->st_d2r, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
       cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess ||
       cudaMalloc(&c->d_xw, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
@@ -297,6 +298,7 @@ int rgsqr_destroy(rgsqr_handle h) {
   cudaStreamDestroy(c->st_own);
   cudaStreamDestroy(c->st_h2d);
   cudaStreamDestroy(c->st_d2h);
+  cudaStreamDestroy(c->st_d2r);
   delete c;
   return RGSQR_OK;
 }

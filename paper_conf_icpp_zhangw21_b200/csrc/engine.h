@@ -65,7 +65,7 @@ struct Ctx {
   int num_sms = 148;
   cudaStream_t st_user = nullptr;   // set by rgsqr_set_stream
   cudaStream_t st_own = nullptr;
-  cudaStream_t st_h2d = nullptr, st_d2h = nullptr;
+  cudaStream_t st_h2d = nullptr, st_d2h = nullptr, st_d2r = nullptr;   // copies: in, Q out, R out
   Options opt;
   rgsqr_stats stats{};
   std::string last_error;
@@ -154,8 +154,10 @@ size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n);
 //   need(c)      -- called before any op that reads columns [0, c) of the node
 //   leaf_done(c) -- called after the leaf ending at column c (Q[:, 0:c) is final)
 struct IncoreHooks {
-  std::function<void(int64_t)> need;
-  std::function<void(int64_t)> leaf_done;
+  std::function<void(int64_t)> need;          // make the compute stream wait for columns < col_end
+  std::function<void(int64_t)> leaf_done;     // columns < col_end are final
+  std::function<bool(int64_t)> pending;       // need(col_end) would still wait on an upload
+  int64_t chunk = 0;                          // upload chunk width (columns)
 };
 int incore_factor(Ctx* c, int prec, void* A, int64_t lda, int64_t m, int64_t n, float* R, int64_t ldr,
                   int64_t col_offset, cudaStream_t st, IncoreHooks* hooks = nullptr);

@@ -450,30 +450,35 @@ cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMa
   return launch_gemm_t<T, false, 64>(ma, mb, p, splits, st);
 }
 
-// Many splits (small nodes): one warp per output element; lane l sums splits
-// l, l+32, ... in order, then a fixed xor tree -- deterministic, and the split loads of
-// a warp are issued together instead of as one long dependent chain.
+// Many splits: a CTA owns 32 consecutive output elements (coalesced 128-byte reads of every
+// split's partial); its 8 warps each sum every 8th split (two interleaved chains), then warp 0
+// adds the 8 group sums -- a fixed order, so the result is deterministic.
 template <typename T>
-__global__ void splitk_reduce_warp_kernel(const float* __restrict__ P, int64_t split_stride, int64_t ldp,
-                                          int splits, float* C, int64_t ldc, int accumulate, T* Cop,
-                                          int64_t ldop, int64_t M, int64_t N) {
-  const int64_t idx = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
-  if (idx >= M * N) return;
-  const int64_t i = idx % M, n = idx / M;
-  float v[8];
-#pragma unroll
-  for (int q = 0; q < 8; ++q) {
-    const int s = lane + 32 * q;
-    v[q] = s < splits ? __ldcs(P + s * split_stride + i + n * ldp) : 0.0f;
+__global__ void __launch_bounds__(256) splitk_reduce_group_kernel(const float* __restrict__ P, int64_t split_stride,
+                                                                  int64_t ldp, int splits, float* C, int64_t ldc,
+                                                                  int accumulate, T* Cop, int64_t ldop, int64_t M,
+                                                                  int64_t N) {
+  __shared__ float red[8][33];
+  const int o = threadIdx.x & 31, g = threadIdx.x >> 5;
+  const int64_t idx = (int64_t)blockIdx.x * 32 + o;
+  const bool ok = idx < M * N;
+  const int64_t i = ok ? idx % M : 0, n = ok ? idx / M : 0;
+  const float* base = P + i + n * ldp;
+  float a0 = 0.f, a1 = 0.f;
+  if (ok) {
+    int s = g;
+    for (; s + 8 < splits; s += 16) {
+      a0 += __ldcs(base + s * split_stride);
+      a1 += __ldcs(base + (s + 8) * split_stride);
+    }
+    if (s < splits) a0 += __ldcs(base + s * split_stride);
   }
-  float acc = v[0];
+  red[g][o] = a0 + a1;
+  __syncthreads();
+  if (g == 0 && ok) {
+    float acc = red[0][o];
 #pragma unroll
-  for (int q = 1; q < 8; ++q) acc += v[q];
-  for (int s = lane + 256; s < splits; s += 32) acc += P[s * split_stride + i + n * ldp];
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-  if (lane == 0) {
+    for (int q = 1; q < 8; ++q) acc += red[q][o];
     if (accumulate) acc = C[i + n * ldc] + acc;
     C[i + n * ldc] = acc;
     if (Cop != nullptr) Cop[i + n * ldop] = Elem<T>::store(acc);
@@ -486,8 +491,8 @@ cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t l
                                  int64_t M, int64_t N, cudaStream_t st) {
   const int64_t total = M * N;
   const int threads = 256;
-  if (splits >= 16) {
-    splitk_reduce_warp_kernel<T><<<(unsigned)((total * 32 + threads - 1) / threads), threads, 0, st>>>(
+  if (splits >= 8) {
+    splitk_reduce_group_kernel<T><<<(unsigned)((total + 31) / 32), 256, 0, st>>>(
         P, split_stride, ldp, splits, C, ldc, accumulate, Cop, ldop, M, N);
   } else {
     splitk_reduce_kernel<T><<<(unsigned)((total + threads - 1) / threads), threads, 0, st>>>(

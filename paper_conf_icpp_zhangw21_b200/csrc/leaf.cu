@@ -560,6 +560,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     //      (b) w_{t+3} = a_{t+3} - sum_{i <= t-1} q_i r_{i,t+3}  (coefficients of round t) into
     //          the ring; the critical group first reads it after round t+2 ----
     const int btid = threadIdx.x - GROUP, bw = warp - GROUP_W;
+    // the last bulk warp owns no projection row pairs: it can reduce the lookahead partials
+    // while the others project
+    const bool la_free = (NR * GROUP + 2 * BULK - 1) / (2 * BULK) == 1 && (rows + 1) / 2 <= BULK - 32;
     for (int t = 0; t + 3 < w; ++t) {
       bar_sync_n(BAR_Q + (t & 1), LEAF_THREADS);
       if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 8 + 5] = clock64();
@@ -611,22 +614,26 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         part[bw][kq + 32] = b0 + b1;
         if (lane == 0) part[bw][64] = e;
       }
-      // reduction of the lookahead partials (rounds t+1 and t+2); before the projection: the
-      // bulk round's total length gates the critical group through BAR_W
+      // reduction of the lookahead partials (rounds t+1 and t+2) by warp LA_W.  When LA_W owns no
+      // projection rows (la_free) it reduces while the other warps project; otherwise before
+      // the projection (the bulk round's total length gates the critical group through BAR_W)
+      const int la_cnt = t + 5 < w ? t + 1 : 0;
+      auto la_reduce = [&]() {
+        float sa = 0.f, sb = 0.f, se = 0.f;
+#pragma unroll
+        for (int v = 0; v < BULK_W; ++v) {
+          sa += part[v][lane];
+          sb += part[v][lane + 32];
+          se += part[v][64];
+        }
+        if (lane < la_cnt) fx_add(t + 2, 4 + lane, sa);
+        if (lane + 32 < la_cnt) fx_add(t + 2, 4 + lane + 32, sb);
+        if (lane == 0) fx_add(t + 1, 4 + t, se);
+      };
       if (t + 4 < w) {
-        const int cnt = t + 5 < w ? t + 1 : 0;
         if (warp == LA_W) {
           bar_sync_n(3, BULK);
-          float sa = 0.f, sb = 0.f, se = 0.f;
-#pragma unroll
-          for (int v = 0; v < BULK_W; ++v) {
-            sa += part[v][lane];
-            sb += part[v][lane + 32];
-            se += part[v][64];
-          }
-          if (lane < cnt) fx_add(t + 2, 4 + lane, sa);
-          if (lane + 32 < cnt) fx_add(t + 2, 4 + lane + 32, sb);
-          if (lane == 0) fx_add(t + 1, 4 + t, se);
+          if (!la_free) la_reduce();
         } else {
           bar_arrive_n(3, BULK);
         }
@@ -650,8 +657,14 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         coef[t % 3][btid] = val;
         if (g == 0) p.R[btid + (int64_t)(t + 3) * p.ldr] = val;
       }
-      bar_sync_n(2, BULK);
-      if (t >= 2 && !(p.skip & 4)) {
+      if (!la_free) {
+        bar_sync_n(2, BULK);
+      } else if (warp != LA_W) {
+        bar_sync_n(2, BULK - 32);
+      } else if (t + 4 < w) {
+        la_reduce();
+      }
+      if (t >= 2 && !(p.skip & 4) && !(la_free && warp == LA_W)) {
         // thread-per-row: w_{t+3}[r] = a_{t+3}[r] - sum_{i < t} q_i[r] r_{i,t+3}  (two fixed-order
         // partial sums)
         const float* cf = coef[t % 3];

@@ -51,7 +51,7 @@ struct Exec {
   char* Q;
   int64_t lda, m, n;
   float* R;
-  cudaStream_t sc, sh, sd;
+  cudaStream_t sc, sh, sd, sr;   // compute, h2d, Q d2h, R d2h
   int K;
   int64_t tmin, tmax;
   bool reuse;
@@ -77,8 +77,10 @@ struct Exec {
   void join_all() {
     wait(sc, sh);
     wait(sc, sd);
+    wait(sc, sr);
     wait(sh, sc);
     wait(sd, sc);
+    wait(sr, sc);
   }
   const char* hsrc(bool q) const { return q ? Q : A; }
   const char* hptr(const char* base, int64_t r0, int64_t col) const { return base + (r0 + col * lda) * s; }
@@ -103,10 +105,14 @@ struct Exec {
   }
   int d2h_r(int64_t r0, int64_t c0, int64_t rows, int64_t cols, const float* src, int64_t lds) {
     if (!R) return RGSQR_OK;  // non-zero ranks of a distributed run
-    cudaEvent_t a = seg_begin(sd);
+    // R blocks go out on their own stream: they never queue behind a backlog of Q columns
+    wait(sr, sc);
+    cudaEvent_t a = seg_begin(sr);
     RGSQR_CUDA(c, cudaMemcpy2DAsync(R + r0 + c0 * n, n * sizeof(float), src, lds * sizeof(float),
-                                    rows * sizeof(float), cols, cudaMemcpyDeviceToHost, sd));
-    seg_end(1, sd, a);
+                                    rows * sizeof(float), cols, cudaMemcpyDeviceToHost, sr));
+    seg_end(1, sr, a);
+    r_done = c->ev();
+    cudaEventRecord(r_done, sr);
     c->stats.d2h_bytes += rows * cols * 4;
     c->stats.d2h_r_bytes += rows * cols * 4;
     return RGSQR_OK;
@@ -117,6 +123,7 @@ struct Exec {
     return (size_t)m * w * s + 256 + (size_t)w * w * 4 + 256 + incore_workspace_bytes(c, prec, m, w) + 4096;
   }
   bool flat = false;   // no ramp: the first tiles were prefetched (see prefetch_tiles)
+  cudaEvent_t r_done = nullptr;   // last R download issued
   std::vector<int64_t> tiles(int64_t t) const {
     std::vector<int64_t> v;
     int64_t r = 0, cur = flat ? t : std::min(tmin, t);
@@ -128,10 +135,12 @@ struct Exec {
     }
     return v;
   }
-  int64_t pick_tile(size_t avail, int64_t cols_per_slot) const {
+  int64_t pick_tile(size_t avail, int64_t cols_per_slot, bool uncapped = false) const {
     if (prec == RGSQR_TF32X3) avail /= 2;  // leave room for the per-tile lo operands
     int64_t t = (int64_t)(avail / ((size_t)K * cols_per_slot * s));
-    t = std::min<int64_t>(t, tmax);
+    // the ramp's cap bounds streamed tiles; prefetched (flat) rings hold as
+    // much of A2 as the budget allows
+    if (!uncapped) t = std::min<int64_t>(t, tmax);
     t = std::min<int64_t>(t, (m + 127) / 128 * 128);
     t = t / 128 * 128;
     return t;
@@ -170,10 +179,15 @@ struct Exec {
         ++next;
       }
     };
+    hk.pending = [&](int64_t col_end) { return next < chunks.size() && chunks[next].first < col_end; };
+    hk.chunk = cw;
+    // Q columns and the matching R columns (full height: entries below the diagonal are zero
+    // and stay zero) go out as soon as a chunk of leaves is final
     hk.leaf_done = [&](int64_t col_end) {
       if (col_end - flushed < cw && col_end < w) return;
       wait(sd, sc);
       int rc = d2h(Q, 0, m, c0 + flushed, col_end - flushed, D + flushed * m * s, m);
+      if (rc == 0) rc = d2h_r(c0, c0 + flushed, w, col_end - flushed, Rs + flushed * w, w);
       if (rc < 0) err = rc;
       flushed = col_end;
     };
@@ -187,16 +201,16 @@ struct Exec {
     if (flushed < w) {
       rc = d2h(Q, 0, m, c0 + flushed, w - flushed, D + flushed * m * s, m);
       if (rc < 0) return rc;
+      rc = d2h_r(c0, c0 + flushed, w, w - flushed, Rs + flushed * w, w);
+      if (rc < 0) return rc;
     }
-    rc = d2h_r(c0, c0, w, w, Rs, w);
-    if (rc < 0) return rc;
     cudaEvent_t done = c->ev();
     cudaEventRecord(done, sd);
     if (q_done) *q_done = done;
-    if (!Rs_ext) {
+    if (!Rs_ext && r_done) {
       // the R block lives in released arena space: nobody may reuse it before its download
-      cudaStreamWaitEvent(sc, done, 0);
-      cudaStreamWaitEvent(sh, done, 0);
+      cudaStreamWaitEvent(sc, r_done, 0);
+      cudaStreamWaitEvent(sh, r_done, 0);
     }
     c->arena.release(mark);
     return RGSQR_OK;
@@ -340,26 +354,25 @@ struct Exec {
     const size_t dB = (size_t)m * w1 * s + 256;
     const size_t left_ws = incore_need(w1) - dB;
     const size_t right_ws = incore_need(w2) - (size_t)m * w2 * s;
-    bool q1_res = reuse && dB + r12b * (reorth ? 2 : 1) + r12ob + left_ws + (size_t)K * 128 * w2 * s <= free0;
+    // the left child's R block + workspace and the node's R12 buffers are never live at the
+    // same time: they share one scratch region above the ring (R12 is allocated there once
+    // the left child's R block has been downloaded), so the ring can hold more of A2
+    const size_t rsb = (size_t)w1 * w1 * 4;
+    const size_t r12_all = r12b * (reorth ? 2 : 1) + r12ob;
+    const size_t scratch = std::max(left_ws, r12_all + 1024) + 4096;   // left_ws includes the R block
+    bool q1_res = reuse && dB + scratch + (size_t)K * 128 * w2 * s <= free0;
     bool a2_to_d = q1_res && recursive && w2 <= w1 && dB + right_ws <= free0;
     if (q1_res) {
       char* D = static_cast<char*>(c->arena.alloc(dB));
-      float* R12 = static_cast<float*>(c->arena.alloc(r12b));
-      void* R12op = c->arena.alloc(r12ob);
-      float* S = reorth ? static_cast<float*>(c->arena.alloc(r12b)) : R12;
-      // the left child's R block lives below the ring for the whole node, so neither the
-      // uploads of the inner pass nor its kernels wait for that block's download
-      const size_t rsb = (size_t)w1 * w1 * 4;
-      float* Rs1 = static_cast<float*>(c->arena.alloc(rsb));
-      // ring sized to leave room for the left child's in-core workspace
-      const size_t ws_left = left_ws > rsb ? left_ws - rsb : 0;
-      const size_t avail = c->arena.free_bytes() > ws_left + 4096 ? c->arena.free_bytes() - ws_left - 4096 : 0;
-      const int64_t t = pick_tile(avail, w2);
-      if (!D || !R12 || !R12op || !S || !Rs1 || t < 128) {
+      const size_t avail = c->arena.free_bytes() > scratch ? c->arena.free_bytes() - scratch : 0;
+      const int64_t t = D ? pick_tile(avail, w2, c->opt.prefetch != 0) : 0;
+      char* ring = t >= 128 ? static_cast<char*>(c->arena.alloc((size_t)K * t * w2 * s)) : nullptr;
+      const size_t mark_s = c->arena.mark();
+      float* Rs1 = ring ? static_cast<float*>(c->arena.alloc(rsb)) : nullptr;
+      if (!D || !ring || !Rs1) {
         c->arena.release(mark0);
         q1_res = a2_to_d = false;
       } else {
-        char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * w2 * s));
         std::vector<cudaEvent_t> ev_free(K);
         for (int k = 0; k < K; ++k) ev_free[k] = c->ev();
         cudaEvent_t q1_done = nullptr;
@@ -372,6 +385,13 @@ struct Exec {
           rc = prefetch_tiles(h, w2, src_q, ring, t, &pre);
           if (rc < 0) return rc;
         }
+        // the scratch region now holds R12: wait for the left child's R block download
+        c->arena.release(mark_s);
+        if (r_done) cudaStreamWaitEvent(sc, r_done, 0);
+        float* R12 = static_cast<float*>(c->arena.alloc(r12b));
+        void* R12op = c->arena.alloc(r12ob);
+        float* S = reorth ? static_cast<float*>(c->arena.alloc(r12b)) : R12;
+        if (!R12 || !R12op || !S) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: no space for R12");
         rc = stream_inner(c0, w1, w2, src_q, D, R12, R12op, ring, t, ev_free, &pre);
         if (rc < 0) return rc;
         cudaEvent_t r12_out = nullptr;
@@ -379,8 +399,7 @@ struct Exec {
           wait(sd, sc);
           rc = d2h_r(c0, h, w1, w2, R12, w1);
           if (rc < 0) return rc;
-          r12_out = c->ev();
-          cudaEventRecord(r12_out, sd);
+          r12_out = r_done;
         }
         rc = stream_outer(c0, w1, w2, src_q, D, a2_to_d && !reorth, q1_done, R12op, ring, t, ev_free);
         if (rc < 0) return rc;
@@ -465,8 +484,7 @@ struct Exec {
     rc = d2h_r(c0, h, w1, w2, R12, w1);
     if (rc < 0) return rc;
     if (r12_out) {
-      *r12_out = c->ev();
-      cudaEventRecord(*r12_out, sd);
+      *r12_out = r_done;
     }
     return stream_outer(c0, w1, w2, true, D, to_D, q1_done, Sop, ring, t, ev_free);
   }
@@ -553,9 +571,9 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
     return rc;
   }
   Exec x{c, prec, s, static_cast<const char*>(A), static_cast<char*>(Q), lda, m, n, R,
-         c->compute(), c->st_h2d, c->st_d2h, (int)c->opt.ring_depth, c->opt.tile_rows_min,
+         c->compute(), c->st_h2d, c->st_d2h, c->st_d2r, (int)c->opt.ring_depth, c->opt.tile_rows_min,
          c->opt.tile_rows_max, c->opt.reuse != 0, c->opt.reorth != 0};
-  if (c->opt.serialize) x.sh = x.sd = x.sc;
+  if (c->opt.serialize) x.sh = x.sd = x.sr = x.sc;
   // make the copy streams start after prior work of the compute stream
   x.join_all();
   cudaEvent_t t_ref = c->ev();
@@ -575,6 +593,7 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   cudaError_t e1 = cudaStreamSynchronize(x.sc);
   cudaError_t e2 = cudaStreamSynchronize(c->st_h2d);
   cudaError_t e3 = cudaStreamSynchronize(c->st_d2h);
+  if (e3 == cudaSuccess) e3 = cudaStreamSynchronize(c->st_d2r);
   if (zero.joinable()) zero.join();
   auto t1 = std::chrono::steady_clock::now();
   for (void* p : registered) cudaHostUnregister(p);

@@ -487,12 +487,47 @@ struct IncoreCtx {
   int64_t col_offset;
   cudaStream_t st;
   IncoreHooks* hooks;
+  // deferred products of nodes whose A2 was still being uploaded: R12 = Q1^T A2 and
+  // A2 -= Q1 R12 applied chunk by chunk when a descendant first needs the columns
+  // (applied in creation order = ancestors first, as the recursion would have)
+  struct Deferred {
+    int64_t c0, w1, end, applied;
+  };
+  std::vector<Deferred> deferred;
 };
+
+// columns < col_end: wait for their upload, then apply the deferred products to them
+static int incore_need(IncoreCtx& k, int64_t col_end) {
+  if (!k.hooks || !k.hooks->need) return RGSQR_OK;
+  for (auto& d : k.deferred) {
+    while (d.applied < std::min(col_end, d.end)) {
+      const int64_t a = d.applied;
+      const int64_t b = std::min(d.end, (a / k.hooks->chunk + 1) * k.hooks->chunk);
+      k.hooks->need(b);
+      const int64_t h = d.c0 + d.w1, off = a - h;
+      const char* Q1 = k.A + d.c0 * k.lda * k.s;
+      char* A2 = k.A + a * k.lda * k.s;
+      char* op = static_cast<char*>(k.r12op);
+      int rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, d.w1, b - a, k.R + d.c0 + a * k.ldr, k.ldr, op,
+                        d.w1, 0, k.st);
+      if (rc < 0) return rc;
+      rc = op_outer(k.c, k.prec, Q1, k.lda, op, d.w1, A2, k.lda, k.m, d.w1, b - a, k.st);
+      if (rc < 0) return rc;
+      (void)off;
+      d.applied = b;
+    }
+  }
+  k.hooks->need(col_end);
+  return RGSQR_OK;
+}
 
 static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
   const int64_t w1 = split_width(w, k.leaf);
   if (w1 == 0) {
-    if (k.hooks && k.hooks->need) k.hooks->need(c0 + w);
+    if (k.hooks && k.hooks->need) {
+      int rc = incore_need(k, c0 + w);
+      if (rc < 0) return rc;
+    }
     char* P = k.A + c0 * k.lda * k.s;
     float* R11 = k.R + c0 + c0 * k.ldr;
     int rc = op_leaf(k.c, k.prec, P, k.lda, k.m, w, R11, k.ldr, k.col_offset + c0, k.st);
@@ -510,10 +545,21 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
   const int64_t w2 = w - w1, h = c0 + w1;
   int rc = incore_rec(k, c0, w1);
   if (rc < 0) return rc;
-  if (k.hooks && k.hooks->need) k.hooks->need(c0 + w);
   const char* Q1 = k.A + c0 * k.lda * k.s;
   char* A2 = k.A + h * k.lda * k.s;
   float* R12 = k.R + c0 + h * k.ldr;
+  if (k.hooks && k.hooks->pending && k.hooks->chunk > 0 && !k.S && k.hooks->pending(c0 + w)) {
+    // A2 is still being uploaded: defer both products; the right child's recursion applies
+    // them column chunk by column chunk as it reaches the columns (the columns of
+    // R12 = Q1^T A2 and of A2 - Q1 R12 are independent)
+    k.deferred.push_back({c0, w1, c0 + w, h});
+    k.c->stats.n_incore_nodes++;
+    return incore_rec(k, h, w2);
+  }
+  if (k.hooks && k.hooks->need) {
+    rc = incore_need(k, c0 + w);
+    if (rc < 0) return rc;
+  }
   rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.r12op, w1, 0, k.st);
   if (rc < 0) return rc;
   rc = op_outer(k.c, k.prec, Q1, k.lda, k.r12op, w1, A2, k.lda, k.m, w1, w2, k.st);
@@ -559,6 +605,7 @@ int incore_factor(Ctx* c, int prec, void* A, int64_t lda, int64_t m, int64_t n, 
     if (!k.S11) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core: no arena space for the CGS2 leaf block");
   }
   int rc = incore_rec(k, 0, n);
+  if (rc >= 0) rc = incore_need(k, n);
   c->arena.release(mark);
   return rc;
 }
