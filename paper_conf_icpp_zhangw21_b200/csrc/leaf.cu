@@ -574,21 +574,14 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       unsigned long long pnow = 0;
       if (btid < t - 1) pnow = ld_word(pwp, p.sys);
       if (t + 4 < w) {
-        // (a') q_t.a_{t+4}: round t+1's value [4+t] (it only feeds the projection of w_{t+4},
-        //      so it is kept off the critical group's reduction)
-        float e = 0.f;
-        {
-          const float* qt = sp + t * LD;
-          const float* a4 = sp + (t + 4) * LD;
-          for (int r = 32 * bw + lane; r < rows; r += BULK) e = fmaf(qt[r], a4[r], e);
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
-        const int cnt = t + 5 < w ? t + 1 : 0;              // (a): i in [0, t]
+        // (a) round t+1's values [4+i] = q_i.a_{t+4}, i <= t, over this warp's 32-row blocks
+        //     (lane = i); they are first read after round t+1 (projection of w_{t+4}, and
+        //     [4+t] by the critical group after round t+3)
+        const int cnt = t + 1;                              // i in [0, t]
         const bool ha = kq < cnt, hb = kq + 32 < cnt;
         float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
         if (ha && !(p.skip & 2)) {
-          const float4* y = reinterpret_cast<const float4*>(sp + (t + 5) * LD);
+          const float4* y = reinterpret_cast<const float4*>(sp + (t + 4) * LD);
           const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
           const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
           // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
@@ -601,34 +594,31 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
               a0 = fmaf(a.z, yy.z, a0);
               a1 = fmaf(a.w, yy.w, a1);
               if (hb) {
-                const float4 b = xb[i];
-                b0 = fmaf(b.x, yy.x, b0);
-                b1 = fmaf(b.y, yy.y, b1);
-                b0 = fmaf(b.z, yy.z, b0);
-                b1 = fmaf(b.w, yy.w, b1);
+                const float4 bb = xb[i];
+                b0 = fmaf(bb.x, yy.x, b0);
+                b1 = fmaf(bb.y, yy.y, b1);
+                b0 = fmaf(bb.z, yy.z, b0);
+                b1 = fmaf(bb.w, yy.w, b1);
               }
             }
           }
         }
         part[bw][kq] = a0 + a1;
         part[bw][kq + 32] = b0 + b1;
-        if (lane == 0) part[bw][64] = e;
       }
-      // reduction of the lookahead partials (rounds t+1 and t+2) by warp LA_W.  When LA_W owns no
+      // reduction of the lookahead partials (round t+1) by warp LA_W.  When LA_W owns no
       // projection rows (la_free) it reduces while the other warps project; otherwise before
       // the projection (the bulk round's total length gates the critical group through BAR_W)
-      const int la_cnt = t + 5 < w ? t + 1 : 0;
+      const int la_cnt = t + 1;
       auto la_reduce = [&]() {
-        float sa = 0.f, sb = 0.f, se = 0.f;
+        float sa = 0.f, sb = 0.f;
 #pragma unroll
         for (int v = 0; v < BULK_W; ++v) {
           sa += part[v][lane];
           sb += part[v][lane + 32];
-          se += part[v][64];
         }
-        if (lane < la_cnt) fx_add(t + 2, 4 + lane, sa);
-        if (lane + 32 < la_cnt) fx_add(t + 2, 4 + lane + 32, sb);
-        if (lane == 0) fx_add(t + 1, 4 + t, se);
+        if (lane < la_cnt) fx_add(t + 1, 4 + lane, sa);
+        if (lane + 32 < la_cnt) fx_add(t + 1, 4 + lane + 32, sb);
       };
       if (t + 4 < w) {
         if (warp == LA_W) {
