@@ -85,6 +85,10 @@ enum rgsqr_option {
                                    left child is being factored (cross-operation overlap,
                                    PAPER.md:231-233; tiles then start at full height instead of
                                    the ramp).  Default 1 */
+  ,RGSQR_OPT_FUSE_SMALL = 14    /* 1 = nodes with w1, w2 <= 64 (fp16/bf16, one GPU) run R12 = Q1^T A2
+                                   and A2 -= Q1 R12 (Eq. 2) as one kernel that
+                                   reads Q1 and A2 once; 0 = the separate TN / NN products.
+                                   Default 1 */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

@@ -154,6 +154,8 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_d2r, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
+      cudaMalloc(&c->d_sn_partials, sizeof(float) * LEAF_MAX_G * 4096) != cudaSuccess ||
+      cudaMalloc(&c->d_sn_r12op, 64 * 64 * 4) != cudaSuccess ||
       cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess ||
       cudaMalloc(&c->d_xw, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
       cudaMalloc(&c->d_xprev, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||
@@ -288,6 +290,8 @@ int rgsqr_destroy(rgsqr_handle h) {
   if (c->nccl_comm && g_nccl.commDestroy) g_nccl.commDestroy(c->nccl_comm);
   if (c->arena.base) cudaFree(c->arena.base);
   cudaFree(c->d_partials);
+  cudaFree(c->d_sn_partials);
+  cudaFree(c->d_sn_r12op);
   cudaFree(c->d_counter);
   cudaFree(c->d_breakdown);
   cudaFree(c->d_xw);
@@ -404,6 +408,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_PROFILE: return &o.profile;
     case RGSQR_OPT_REORTH: return &o.reorth;
     case RGSQR_OPT_PREFETCH: return &o.prefetch;
+    case RGSQR_OPT_FUSE_SMALL: return &o.fuse_small;
   }
   return nullptr;
 }

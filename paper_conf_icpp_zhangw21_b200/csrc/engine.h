@@ -28,6 +28,7 @@ struct Options {
   int64_t profile = 0;
   int64_t reorth = 0;        // CGS2 (RGSQR_OPT_REORTH)
   int64_t prefetch = 1;      // OOC: upload the first ring tiles during the left child (RGSQR_OPT_PREFETCH)
+  int64_t fuse_small = 1;    // fused kernel for nodes with w1, w2 <= 64 (RGSQR_OPT_FUSE_SMALL)
 };
 
 struct KernSeg {
@@ -73,6 +74,8 @@ struct Ctx {
   size_t arena_alloc_size = 0;
   // small persistent device buffers (leaf barrier/partials, breakdown flag)
   float* d_partials = nullptr;
+  float* d_sn_partials = nullptr;   // fused bottom node: [LEAF_MAX_G][4096] partials
+  void* d_sn_r12op = nullptr;       // fused bottom node: 64 x 64 operand copy
   unsigned int* d_counter = nullptr;
   unsigned int leaf_epoch = 0;
   int* d_breakdown = nullptr;

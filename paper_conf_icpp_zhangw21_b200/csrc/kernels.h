@@ -81,6 +81,27 @@ struct LeafParams {
   int64_t col_offset;       // global index of the panel's first column
 };
 
+// fused bottom node (small.cu): R12 = Q1^T A2, A2 -= Q1 R12 for w1, w2 <= 64, fp16/bf16
+struct SmallNodeParams {
+  const void* Q1;
+  int64_t ldq;
+  void* A2;
+  int64_t lda;
+  int64_t m;
+  int w1, w2;
+  int rows_per_cta;         // multiple of 8
+  int vec_ok;               // Q1/A2 16-byte aligned columns
+  float* R12;               // fp32 out, ldr
+  int64_t ldr;
+  float* partials;          // [grid][4096]
+  void* r12op;              // [64][64] operand copy ([j][i])
+  unsigned* counter;        // zeroed by the launcher
+};
+constexpr int SN_MAX_RP = 768;  // rows per CTA the fused bottom node holds in shared memory
+size_t small_node_smem(int rp);
+template <typename T>
+cudaError_t launch_small_node(const SmallNodeParams& p, int grid, cudaStream_t st);
+
 int gemm_block_k(int elem_bytes);
 int leaf_max_smem_rows(int w);
 

@@ -181,13 +181,30 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   {
     constexpr int V = Vec<T>::N;
     const int nvec = p.vec_ok ? rows / V : 0;
-    for (int idx = threadIdx.x; idx < w * nvec; idx += LEAF_THREADS) {
-      const int j = idx / nvec, i = (idx - j * nvec) * V;
-      float f[V];
-      Vec<T>::load(P + r0 + i + (int64_t)j * p.ldp, f);
+    // batches of B independent 16-byte loads per thread in flight before the converting stores
+    constexpr int B = 8;
+    for (int base = threadIdx.x; base < w * nvec; base += B * LEAF_THREADS) {
+      uint4 raw[B];
 #pragma unroll
-      for (int e = 0; e < V; e += 4)
-        *reinterpret_cast<float4*>(sp + j * LD + i + e) = make_float4(f[e], f[e + 1], f[e + 2], f[e + 3]);
+      for (int u = 0; u < B; ++u) {
+        const int idx = base + u * LEAF_THREADS;
+        if (idx < w * nvec) {
+          const int j = idx / nvec, i = (idx - j * nvec) * V;
+          raw[u] = *reinterpret_cast<const uint4*>(P + r0 + i + (int64_t)j * p.ldp);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < B; ++u) {
+        const int idx = base + u * LEAF_THREADS;
+        if (idx < w * nvec) {
+          const int j = idx / nvec, i = (idx - j * nvec) * V;
+          float f[V];
+          Vec<T>::load(reinterpret_cast<const T*>(&raw[u]), f);
+#pragma unroll
+          for (int e = 0; e < V; e += 4)
+            *reinterpret_cast<float4*>(sp + j * LD + i + e) = make_float4(f[e], f[e + 1], f[e + 2], f[e + 3]);
+        }
+      }
     }
     const int span = LD - nvec * V;
     for (int idx = threadIdx.x; idx < w * span; idx += LEAF_THREADS) {

@@ -442,6 +442,39 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   return RGSQR_OK;
 }
 
+// fused bottom node (small.cu): returns 1 when done, 0 when the shape / precision / context
+// is not covered (the caller then runs the separate products), < 0 on error
+int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64_t lda, int64_t m, int64_t w1,
+                  int64_t w2, float* R12, int64_t ldr, cudaStream_t st) {
+  if (!c->opt.fuse_small || c->nccl_comm || w1 > 64 || w2 > 64 || w1 < 1 || w2 < 1) return 0;
+  if (prec != RGSQR_FP16 && prec != RGSQR_BF16) return 0;
+  int G, rp;
+  leaf_geometry(c, m, &G, &rp);
+  if (rp > SN_MAX_RP || small_node_smem(rp) > 227 * 1024) return 0;
+  SmallNodeParams p{};
+  p.Q1 = Q1;
+  p.ldq = ldq;
+  p.A2 = A2;
+  p.lda = lda;
+  p.m = m;
+  p.w1 = (int)w1;
+  p.w2 = (int)w2;
+  p.rows_per_cta = rp;
+  p.vec_ok = ((ldq * 2) % 16 == 0) && ((lda * 2) % 16 == 0) && (reinterpret_cast<uintptr_t>(Q1) % 16 == 0) &&
+             (reinterpret_cast<uintptr_t>(A2) % 16 == 0);
+  p.R12 = R12;
+  p.ldr = ldr;
+  p.partials = c->d_sn_partials;
+  p.r12op = c->d_sn_r12op;
+  p.counter = c->d_counter + 16;
+  cudaEvent_t kb = c->kbegin(st);
+  cudaError_t e = prec == RGSQR_FP16 ? launch_small_node<__half>(p, G, st) : launch_small_node<__nv_bfloat16>(p, G, st);
+  if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("fused node launch: ") + cudaGetErrorString(e));
+  c->kend(3, st, kb, 4.0 * m * w1 * w2, 2.0 * m * (w1 + w2) + 2.0 * m * w2 + 4.0 * w1 * w2);
+  c->stats.n_other_launches++;
+  return 1;
+}
+
 // ---------------------------------------------------------------------------------
 // in-core recursion (Eq. 2) on a device-resident m x n matrix
 // ---------------------------------------------------------------------------------
@@ -559,6 +592,14 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
   if (k.hooks && k.hooks->need) {
     rc = incore_need(k, c0 + w);
     if (rc < 0) return rc;
+  }
+  if (!k.S) {
+    rc = op_small_node(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.st);
+    if (rc < 0) return rc;
+    if (rc == 1) {   // done by the fused kernel
+      k.c->stats.n_incore_nodes++;
+      return incore_rec(k, h, w2);
+    }
   }
   rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.r12op, w1, 0, k.st);
   if (rc < 0) return rc;

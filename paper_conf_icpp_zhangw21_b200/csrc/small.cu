@@ -1,0 +1,259 @@
+// small.cu -- the bottom nodes of the recursion (Eq. 2) in one kernel:
+//     R12 = Q1^T A2        (inner product, w1 x w2, both <= 64)
+//     A2 <- A2 - Q1 R12    (outer product, fused subtraction, rounded once to storage)
+// for fp16 / bf16 storage.  Separately these are a split-K TN GEMM, a split-K reduction and
+// an NN GEMM -- three launches that each re-read the m x 64 operands; at the bottom of the
+// recursion they are bound by HBM bytes and launch latency, not by the tensor cores.
+//
+// Cooperative grid, one CTA per SM, CTA g owns rows [g RP, (g+1) RP):
+//   phase 1: the CTA's row slices of Q1 and A2 are loaded ONCE into shared memory; the partial
+//            Q1_s^T A2_s (64 x 64, fp32) is formed with mma.sync m16n8k16 and written out;
+//   barrier; phase 2: every CTA sums 1/G of the entries over all G partials in a fixed
+//            order (deterministic) -> R12 (fp32, the R block) and its operand copy (RN);
+//   barrier; phase 3: A2_s -= Q1_s R12 with mma.sync from the same shared-memory slices;
+//            A2' rounded RN and stored once.
+// Reads Q1 and A2 once and writes A2 once (plus 2 x G x 16 KB of partials in L2).
+#include "dtype.cuh"
+#include "kernels.h"
+
+namespace rgsqr {
+
+static constexpr int SN_THREADS = 256;
+static constexpr int SN_RS = 72;   // R12 operand tile stride (halves): 144 B == 16 (mod 128)
+
+// shared-memory column stride (halves) of a row slice: >= rows rounded to 16, and
+// 2 * stride == 16 (mod 128) bytes so that ldmatrix row addresses hit distinct banks
+__host__ __device__ inline int sn_stride(int rp) {
+  const int r16 = (rp + 15) & ~15;
+  return r16 + ((8 - (r16 % 64)) + 64) % 64;
+}
+
+size_t small_node_smem(int rp) { return (size_t)2 * 64 * sn_stride(rp) * 2 + 64 * SN_RS * 2 + 8 * 33 * 4 + 64; }
+
+template <typename T>
+struct MmaOp;
+template <>
+struct MmaOp<__half> {
+  __device__ static void mma(float* d, const uint32_t* a, const uint32_t* b) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b[0]), "r"(b[1]));
+  }
+};
+template <>
+struct MmaOp<__nv_bfloat16> {
+  __device__ static void mma(float* d, const uint32_t* a, const uint32_t* b) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b[0]), "r"(b[1]));
+  }
+};
+
+__device__ __forceinline__ void ldsm_x4(uint32_t* r, const void* p) {
+  const unsigned a = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+               : "r"(a));
+}
+__device__ __forceinline__ void ldsm_x4_t(uint32_t* r, const void* p) {
+  const unsigned a = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+               : "r"(a));
+}
+
+// grid barrier k (k = 1, 2, ...) on a zeroed counter: release this CTA's writes, acquire all
+__device__ __forceinline__ void sn_grid_barrier(unsigned* counter, unsigned target) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(counter) : "memory");
+    unsigned v;
+    do {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(counter) : "memory");
+    } while (v < target);
+  }
+  __syncthreads();
+}
+
+template <typename T>
+__global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodeParams p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const int RP = p.rows_per_cta;
+  const int S = sn_stride(RP);
+  const int RP16 = (RP + 15) & ~15;
+  T* qs = reinterpret_cast<T*>(smem);            // [64][S]: column i of the Q1 slice
+  T* as = qs + 64 * S;                           // [64][S]: column j of the A2 slice
+  T* rs = as + 64 * S;                           // [64][SN_RS]: R12 operand as [j][i]
+  float* red = reinterpret_cast<float*>(rs + 64 * SN_RS);   // [8][33]
+  const int G = gridDim.x, g = blockIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t r0 = (int64_t)g * RP;
+  const int64_t rem = p.m - r0;
+  const int rows = rem <= 0 ? 0 : (rem < RP ? (int)rem : RP);
+  const T* Q1 = static_cast<const T*>(p.Q1);
+  T* A2 = static_cast<T*>(p.A2);
+
+  // ---- load the slices (zero-padded to 64 columns and RP16 rows): cp.async, all in flight ----
+  {
+    const int nv = p.vec_ok ? rows / 8 : 0;      // 16-byte vectors per column
+    for (int idx = threadIdx.x; idx < 64 * (S / 8); idx += SN_THREADS) {
+      const int c = idx / (S / 8), v = idx - c * (S / 8);
+      const bool inq = v < nv && c < p.w1, ina = v < nv && c < p.w2;
+      const T* srcq = inq ? Q1 + r0 + 8 * v + (int64_t)c * p.ldq : Q1;
+      const T* srca = ina ? A2 + r0 + 8 * v + (int64_t)c * p.lda : A2;
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"((unsigned)__cvta_generic_to_shared(qs + c * S + 8 * v)),
+                   "l"(srcq), "r"(inq ? 16 : 0)
+                   : "memory");
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"((unsigned)__cvta_generic_to_shared(as + c * S + 8 * v)),
+                   "l"(srca), "r"(ina ? 16 : 0)
+                   : "memory");
+    }
+    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+    __syncthreads();
+    for (int idx = threadIdx.x; idx < 64 * (rows - 8 * nv); idx += SN_THREADS) {
+      const int c = idx / (rows - 8 * nv), r = 8 * nv + (idx - c * (rows - 8 * nv));
+      if (c < p.w1) qs[c * S + r] = Q1[r0 + r + (int64_t)c * p.ldq];
+      if (c < p.w2) as[c * S + r] = A2[r0 + r + (int64_t)c * p.lda];
+    }
+    __syncthreads();
+  }
+
+  // ---- phase 1: partial = Q1_s^T A2_s; warp: m-tile (16 rows of R12) warp & 3, n-tiles
+  //      (warp >> 2) * 4 .. + 3 (8 columns each) ----
+  {
+    const int mt = warp & 3, nt0 = (warp >> 2) * 4;
+    float acc[4][4] = {};
+    const int q = lane >> 3, l8 = lane & 7;
+    for (int kk = 0; kk < RP16; kk += 16) {
+      uint32_t a[4], b[2][4];
+      ldsm_x4(a, qs + (16 * mt + (q & 1) * 8 + l8) * S + kk + (q >> 1) * 8);
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+        ldsm_x4(b[h], as + (8 * (nt0 + 2 * h + (q >> 1)) + l8) * S + kk + (q & 1) * 8);
+#pragma unroll
+      for (int n = 0; n < 4; ++n) MmaOp<T>::mma(acc[n], a, &b[n >> 1][(n & 1) * 2]);
+    }
+    float* P = p.partials + (size_t)g * 4096;    // [j][i], i contiguous
+#pragma unroll
+    for (int n = 0; n < 4; ++n) {
+      const int i = 16 * mt + (lane >> 2), j = 8 * (nt0 + n) + 2 * (lane & 3);
+      P[j * 64 + i] = acc[n][0];
+      P[(j + 1) * 64 + i] = acc[n][1];
+      P[j * 64 + i + 8] = acc[n][2];
+      P[(j + 1) * 64 + i + 8] = acc[n][3];
+    }
+  }
+  sn_grid_barrier(p.counter, (unsigned)G);
+
+  // ---- phase 2: entries [g EPC, (g+1) EPC) summed over the G partials in a fixed order:
+  //      warp k adds partials k, k+8, ... in order, then warp 0 the 8 groups ----
+  {
+    const int EPC = (4096 + G - 1) / G;
+    for (int e0 = g * EPC; e0 < min(4096, (g + 1) * EPC); e0 += 32) {
+      const int e = e0 + lane;
+      const bool ok = e < min(4096, (g + 1) * EPC);
+      // all of this thread's partials in flight at once, then summed in order
+      constexpr int PMAX = (LEAF_MAX_G + 7) / 8;
+      float v[PMAX];
+#pragma unroll
+      for (int q = 0; q < PMAX; ++q) {
+        const int k = warp + 8 * q;
+        v[q] = (ok && k < G) ? __ldcg(p.partials + (size_t)k * 4096 + e) : 0.0f;
+      }
+      float s0 = v[0];
+#pragma unroll
+      for (int q = 1; q < PMAX; ++q) s0 += v[q];
+      red[warp * 33 + lane] = s0;
+      __syncthreads();
+      if (warp == 0 && ok) {
+        float v = red[lane];
+#pragma unroll
+        for (int k = 1; k < 8; ++k) v += red[k * 33 + lane];
+        const int i = e & 63, j = e >> 6;
+        if (i < p.w1 && j < p.w2) p.R12[i + (int64_t)j * p.ldr] = v;
+        static_cast<T*>(p.r12op)[e] = Elem<T>::store(v);    // [j][i]; zero outside w1 x w2
+      }
+      __syncthreads();
+    }
+  }
+  sn_grid_barrier(p.counter, (unsigned)(2 * G));
+
+  // ---- phase 3: A2_s -= Q1_s R12; warp: m-tiles warp, warp + 8, ... (16 rows), all 8 n-tiles ----
+  {
+    for (int idx = threadIdx.x; idx < 64 * 8; idx += SN_THREADS) {      // 64 x 64 halves, 16 B each
+      const int j = idx >> 3, v = idx & 7;
+      *reinterpret_cast<uint4*>(rs + j * SN_RS + 8 * v) =
+          __ldcg(reinterpret_cast<const uint4*>(static_cast<const T*>(p.r12op) + j * 64 + 8 * v));
+    }
+    __syncthreads();
+    const int q = lane >> 3, l8 = lane & 7;
+    for (int mt = warp; mt < RP16 / 16; mt += SN_THREADS / 32) {
+      float acc[8][4] = {};
+#pragma unroll
+      for (int ks = 0; ks < 4; ++ks) {
+        uint32_t a[4], b[4][4];
+        // A[m = row][k = i] lives as qs[i][row]: transposed 8x8 loads
+        ldsm_x4_t(a, qs + (16 * ks + (q >> 1) * 8 + l8) * S + 16 * mt + (q & 1) * 8);
+#pragma unroll
+        for (int h = 0; h < 4; ++h) ldsm_x4(b[h], rs + (8 * (2 * h + (q >> 1)) + l8) * SN_RS + 16 * ks + (q & 1) * 8);
+#pragma unroll
+        for (int n = 0; n < 8; ++n) MmaOp<T>::mma(acc[n], a, &b[n >> 1][(n & 1) * 2]);
+      }
+#pragma unroll
+      for (int n = 0; n < 8; ++n) {
+        const int r = 16 * mt + (lane >> 2), j = 8 * n + 2 * (lane & 3);
+        T* c0 = as + j * S + r;
+        T* c1 = as + (j + 1) * S + r;
+        c0[0] = Elem<T>::store(Elem<T>::load(c0[0]) - acc[n][0]);
+        c1[0] = Elem<T>::store(Elem<T>::load(c1[0]) - acc[n][1]);
+        c0[8] = Elem<T>::store(Elem<T>::load(c0[8]) - acc[n][2]);
+        c1[8] = Elem<T>::store(Elem<T>::load(c1[8]) - acc[n][3]);
+      }
+    }
+    __syncthreads();
+    // ---- store A2' (columns < w2, rows < rows) ----
+    const int nv = p.vec_ok ? rows / 8 : 0;
+    for (int idx = threadIdx.x; idx < p.w2 * nv; idx += SN_THREADS) {
+      const int c = idx / nv, v = idx - c * nv;
+      *reinterpret_cast<uint4*>(A2 + r0 + 8 * v + (int64_t)c * p.lda) = *reinterpret_cast<const uint4*>(as + c * S + 8 * v);
+    }
+    const int tail = rows - 8 * nv;
+    for (int idx = threadIdx.x; idx < p.w2 * tail; idx += SN_THREADS) {
+      const int c = idx / tail, r = 8 * nv + (idx - c * tail);
+      A2[r0 + r + (int64_t)c * p.lda] = as[c * S + r];
+    }
+  }
+}
+
+template <typename T>
+cudaError_t launch_small_node(const SmallNodeParams& p, int grid, cudaStream_t st) {
+  const size_t smem = small_node_smem(p.rows_per_cta);
+  static size_t attr = 0;
+  if (smem > attr) {
+    cudaError_t e = cudaFuncSetAttribute(small_node_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr = smem;
+  }
+  cudaError_t e = cudaMemsetAsync(p.counter, 0, sizeof(unsigned), st);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(SN_THREADS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr1[1];
+  attr1[0].id = cudaLaunchAttributeCooperative;
+  attr1[0].val.cooperative = 1;
+  cfg.attrs = attr1;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, small_node_kernel<T>, p);
+}
+
+template cudaError_t launch_small_node<__half>(const SmallNodeParams&, int, cudaStream_t);
+template cudaError_t launch_small_node<__nv_bfloat16>(const SmallNodeParams&, int, cudaStream_t);
+
+}  // namespace rgsqr

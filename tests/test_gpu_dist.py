@@ -17,6 +17,9 @@ MiB = 1 << 20
 def handles():
     from paper_conf_icpp_zhangw21_b200 import Handle
     plain = Handle(0)
+    # the fused bottom-node kernel is a single-GPU path (its R12 reduction cannot include other
+    # ranks); compare against the plain context running the same separate products
+    plain.set_option("fuse_small", 0)
     dist = Handle(0, rank=0, nranks=1, unique_id=Handle.unique_id())
     yield plain, dist
     dist.close()
