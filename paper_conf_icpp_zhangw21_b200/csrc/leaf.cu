@@ -78,9 +78,12 @@ __device__ __forceinline__ double pow2d(int e) { return __hiloint2double((1023 +
 
 // per-phase cycle stamps of CTA p.dbg_cta (diagnostics; p.dbg == nullptr in production)
 #define DBG_CTA p.dbg_cta
+// bulk-group stamps (slots 8..13 of round t, thread 0 of the bulk group)
+#define BULK_STAMP(i)                                                   \
+  if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 16 + (i)] = clock64();
 #define DBG_STAMP(i)                                           \
   if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) \
-    p.dbg[(size_t)t * 8 + (i)] = clock64();
+    p.dbg[(size_t)t * 16 + (i)] = clock64();
 
 // 16-byte vector load of consecutive storage elements widened to fp32.
 template <typename T>
@@ -156,6 +159,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
   __shared__ float tot[2][LEAF_MAX_W + 2];         // reduced round vector, by parity of the round
   __shared__ float part[GEMV_PARTS][LEAF_MAX_W + 2];        // round 0 / lookahead partials
+  __shared__ float part2[GEMV_PARTS / 2][LEAF_MAX_W];       // lookahead partials, second target
   __shared__ float cpart[GEMV_PARTS][8];                    // critical-dot partials
   __shared__ unsigned long long xprev[LEAF_XW_WORDS];      // last seen exchange words
   __shared__ __align__(16) float coef[3][LEAF_MAX_W + 4];   // r_{i,t+3}, i < t, by t mod 3
@@ -399,6 +403,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   constexpr int GROUP = 32 * CW, GROUP_W = CW;                       // critical group
   constexpr int BULK = LEAF_THREADS - GROUP, BULK_W = LEAF_WARPS - CW;   // bulk group
   constexpr int CRIT_W = GROUP_W - 1, LA_W = LEAF_WARPS - 1;
+  static_assert(BULK_W <= GEMV_PARTS / 2, "part2 holds one row per bulk warp");
   const bool is_crit = threadIdx.x < GROUP;
   const int crit_warps = rows >= GROUP ? GROUP_W : (rows + 31) / 32;   // critical warps owning rows
   constexpr int BAR_Q = 4, BAR_W = 6;
@@ -492,7 +497,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       //      (w_{t+1} = a_{t+1} for t+1 <= 3), and round t+1's critical dots
       //      u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2}, q_t.a_{t+2}, q_t.a_{t+3}, q_t.a_{t+4} ----
       const bool h2 = t + 2 < w, h3 = t + 3 < w, h4 = t + 4 < w;
-      float s0, s1, s2, s3;
+      float s0, s1, s2, s3, s4;
       {
         const float* wsrc = (t + 1 <= 4) ? sp + (more ? t + 1 : t) * LD : wring + ((t + 1) % LEAF_WRING) * LD;
         const float* a4p = sp + (h4 ? t + 4 : t) * LD;
@@ -515,13 +520,14 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
 #pragma unroll
         for (int j = 0; j < NR; ++j)
           if (vr[j]) ut[rr[j]] = q[j];   // Q goes to global memory at the end
-        s0 = s1 = s2 = s3 = 0.0f;
+        s0 = s1 = s2 = s3 = s4 = 0.0f;
 #pragma unroll
         for (int j = 0; j < NR; ++j) {
           s0 = fmaf(av[j], av[j], s0);
           s1 = fmaf(av[j], ra2[j], s1);
           s2 = fmaf(q[j], ra2[j], s2);
           s3 = fmaf(q[j], ra3[j], s3);
+          s4 = fmaf(q[j], a4v[j], s4);   // q_t.a_{t+4}: round t+1's [4+t], reduced after publishing
         }
 #pragma unroll
         for (int j = 0; j < NR; ++j) {
@@ -565,10 +571,23 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         s += __shfl_xor_sync(0xffffffffu, s, 2);
         s += __shfl_xor_sync(0xffffffffu, s, 1);
         if (j == 0 && c < n_crit) fx_add_scaled(t + 1, c, s, crit_scale);
-        if (p.dbg != nullptr && blockIdx.x == DBG_CTA && lane == 0) p.dbg[(size_t)t * 8 + 7] = clock64();
+        if (p.dbg != nullptr && blockIdx.x == DBG_CTA && lane == 0) p.dbg[(size_t)t * 16 + 7] = clock64();
         if (p.dbg2 != nullptr && lane == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 0] = gtimer();
       }
       DBG_STAMP(4);
+      // ---- inside round t+1's exchange wait: q_t.a_{t+4} (round t+1's value [4+t], read by this
+      //      group after round t+3) reduced and added off the critical chain ----
+      if (h4) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) s4 += __shfl_xor_sync(0xffffffffu, s4, o);
+        if (lane == 0) cpart[warp][4] = s4;
+        bar_sync_n(1, GROUP);
+        if (warp == CRIT_W && lane == 0) {
+          float v = 0.f;
+          for (int j = 0; j < crit_warps; ++j) v += cpart[j][4];
+          fx_add(t + 1, 4 + t, v);
+        }
+      }
     }
   } else {
     // ---- BULK group: for each round t, after q_t is in smem:
@@ -581,8 +600,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     // while the others project
     const bool la_free = (NR * GROUP + 2 * BULK - 1) / (2 * BULK) == 1 && (rows + 1) / 2 <= BULK - 32;
     for (int t = 0; t + 3 < w; ++t) {
+      BULK_STAMP(13);
       bar_sync_n(BAR_Q + (t & 1), LEAF_THREADS);
-      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 8 + 5] = clock64();
+      BULK_STAMP(8);
       // round t's values [4+i] = r_{i,t+3}, i <= t-1: round t is complete (the critical group
       // has seen it); the loads are issued now and checked after the dot products below
       const int pk = 4 + btid;
@@ -590,54 +610,73 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       const unsigned long long* pwp = p.xw + (size_t)pidx * LEAF_XW_STRIDE;
       unsigned long long pnow = 0;
       if (btid < t - 1) pnow = ld_word(pwp, p.sys);
-      if (t + 4 < w) {
-        // (a) round t+1's values [4+i] = q_i.a_{t+4}, i <= t, over this warp's 32-row blocks
-        //     (lane = i); they are first read after round t+1 (projection of w_{t+4}, and
-        //     [4+t] by the critical group after round t+3)
-        const int cnt = t + 1;                              // i in [0, t]
+      // (a) lookahead GEMV, every other round for two target columns (each q_i read once):
+      //     even t: round t+1's [4+i] = q_i.a_{t+4}, i <= t-1, and round t+2's [4+i] =
+      //     q_i.a_{t+5}, i <= t (lane = i).  Round t+1's [4+t] comes from the critical group.
+      const bool ev = (t & 1) == 0;
+      const bool g1 = ev && t >= 1 && t + 4 < w, g2 = ev && t + 5 < w;
+      if (g1 || g2) {
+        const int cnt1 = g1 ? t : 0, cnt2 = g2 ? t + 1 : 0;
+        const int cnt = max(cnt1, cnt2);
         const bool ha = kq < cnt, hb = kq + 32 < cnt;
-        float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+        float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f, c0 = 0.f, c1 = 0.f, d0 = 0.f, d1 = 0.f;
         if (ha && !(p.skip & 2)) {
-          const float4* y = reinterpret_cast<const float4*>(sp + (t + 4) * LD);
+          const float4* y1 = reinterpret_cast<const float4*>(sp + (g1 ? t + 4 : t) * LD);
+          const float4* y2 = reinterpret_cast<const float4*>(sp + (g2 ? t + 5 : t) * LD);
           const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
           const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
           // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
           for (int base = 8 * bw; base < nv4; base += 8 * BULK_W) {
-#pragma unroll
+#pragma unroll 4
             for (int i = base; i < base + 8; ++i) {
-              const float4 yy = y[i], a = xa[i];
-              a0 = fmaf(a.x, yy.x, a0);
-              a1 = fmaf(a.y, yy.y, a1);
-              a0 = fmaf(a.z, yy.z, a0);
-              a1 = fmaf(a.w, yy.w, a1);
+              const float4 u = y1[i], v = y2[i], a = xa[i];
+              a0 = fmaf(a.x, u.x, a0);
+              a1 = fmaf(a.y, u.y, a1);
+              a0 = fmaf(a.z, u.z, a0);
+              a1 = fmaf(a.w, u.w, a1);
+              c0 = fmaf(a.x, v.x, c0);
+              c1 = fmaf(a.y, v.y, c1);
+              c0 = fmaf(a.z, v.z, c0);
+              c1 = fmaf(a.w, v.w, c1);
               if (hb) {
                 const float4 bb = xb[i];
-                b0 = fmaf(bb.x, yy.x, b0);
-                b1 = fmaf(bb.y, yy.y, b1);
-                b0 = fmaf(bb.z, yy.z, b0);
-                b1 = fmaf(bb.w, yy.w, b1);
+                b0 = fmaf(bb.x, u.x, b0);
+                b1 = fmaf(bb.y, u.y, b1);
+                b0 = fmaf(bb.z, u.z, b0);
+                b1 = fmaf(bb.w, u.w, b1);
+                d0 = fmaf(bb.x, v.x, d0);
+                d1 = fmaf(bb.y, v.y, d1);
+                d0 = fmaf(bb.z, v.z, d0);
+                d1 = fmaf(bb.w, v.w, d1);
               }
             }
           }
         }
         part[bw][kq] = a0 + a1;
         part[bw][kq + 32] = b0 + b1;
+        part2[bw][kq] = c0 + c1;
+        part2[bw][kq + 32] = d0 + d1;
       }
-      // reduction of the lookahead partials (round t+1) by warp LA_W.  When LA_W owns no
-      // projection rows (la_free) it reduces while the other warps project; otherwise before
-      // the projection (the bulk round's total length gates the critical group through BAR_W)
-      const int la_cnt = t + 1;
+      BULK_STAMP(9);
+      // reduction of the lookahead partials by warp LA_W (while the others project, when
+      // LA_W owns no projection rows)
       auto la_reduce = [&]() {
-        float sa = 0.f, sb = 0.f;
+        const int cnt1 = g1 ? t : 0, cnt2 = g2 ? t + 1 : 0;
+        float sa = 0.f, sb = 0.f, sc = 0.f, sd = 0.f;
 #pragma unroll
         for (int v = 0; v < BULK_W; ++v) {
           sa += part[v][lane];
           sb += part[v][lane + 32];
+          sc += part2[v][lane];
+          sd += part2[v][lane + 32];
         }
-        if (lane < la_cnt) fx_add(t + 1, 4 + lane, sa);
-        if (lane + 32 < la_cnt) fx_add(t + 1, 4 + lane + 32, sb);
+        if (lane < cnt1) fx_add(t + 1, 4 + lane, sa);
+        if (lane + 32 < cnt1) fx_add(t + 1, 4 + lane + 32, sb);
+        if (lane < cnt2) fx_add(t + 2, 4 + lane, sc);
+        if (lane + 32 < cnt2) fx_add(t + 2, 4 + lane + 32, sd);
       };
-      if (t + 4 < w) {
+      const bool la_work = g1 || g2;
+      if (la_work) {
         if (warp == LA_W) {
           bar_sync_n(3, BULK);
           if (!la_free) la_reduce();
@@ -668,9 +707,10 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         bar_sync_n(2, BULK);
       } else if (warp != LA_W) {
         bar_sync_n(2, BULK - 32);
-      } else if (t + 4 < w) {
+      } else if (la_work) {
         la_reduce();
       }
+      BULK_STAMP(10);
       if (t >= 2 && !(p.skip & 4) && !(la_free && warp == LA_W)) {
         // thread-per-row: w_{t+3}[r] = a_{t+3}[r] - sum_{i < t} q_i[r] r_{i,t+3}  (two fixed-order
         // partial sums)
@@ -722,8 +762,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
             *reinterpret_cast<float2*>(wd + pb[j]) = make_float2(av.x - (e0[j].x + e1[j].x), av.y - (e0[j].y + e1[j].y));
           }
       }
+      BULK_STAMP(11);
       bar_arrive_n(BAR_W + (t & 1), LEAF_THREADS);
-      if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 8 + 6] = clock64();
+      BULK_STAMP(12);
     }
   }
   __syncthreads();

@@ -340,7 +340,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   p.r0buf = c->d_r0buf;
   p.m_global = c->m_global > 0 ? c->m_global : m;
   p.vec_ok = ((ldp * elem_bytes(prec)) % 16 == 0) && (reinterpret_cast<uintptr_t>(P) % 16 == 0);
-  if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 8 * LEAF_MAX_W);
+  if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 16 * LEAF_MAX_W);
   p.dbg = dbg ? dbg_buf : nullptr;
   static const bool dbg2 = getenv("RGSQR_LEAF_DEBUG2") != nullptr;
   static long long* dbg2_buf = nullptr;
@@ -386,31 +386,28 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   const int s = elem_bytes(prec);
   c->kend(0, st, kb, 2.0 * m * w * w, 2.0 * m * w * s + 4.0 * w * w);
   if (p.dbg) {
-    long long hb[8 * LEAF_MAX_W];
-    cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 8 * w, cudaMemcpyDeviceToHost, st);
+    long long hb[16 * LEAF_MAX_W];
+    cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 16 * w, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
-    // stamps of iteration t: 0 start, 1 round t exchanged, 2 scalars, 3 row pass (q_t, u_{t+1},
-    // round t+1's critical dots), 4 critical values added, 5 lookahead dots added, 6 projection
-    const int order[7] = {0, 1, 2, 3, 4, 5, 6};
-    const char* names[6] = {"exchange", "scalars", "rowpass", "publish", "lookahead", "project"};
-    double ph[6] = {0};
-    int cnt = 0;
-    for (int t = 1; t + 1 < w; ++t, ++cnt)
-      for (int i = 0; i < 6; ++i) ph[i] += (double)(hb[t * 8 + order[i + 1]] - hb[t * 8 + order[i]]);
-    fprintf(stderr, "[leaf m=%lld w=%lld G=%d RP=%d] cycles/round:", (long long)m, (long long)w, G, rp);
-    double sum = 0;
-    for (int i = 0; i < 6; ++i) {
-      fprintf(stderr, " %s %.0f", names[i], ph[i] / std::max(1, cnt));
-      sum += ph[i];
-    }
-    // stamp 7: the critical reducer warp published round t+1's values
-    double pub = 0, xl = 0;
-    for (int t = 1; t + 2 < w; ++t) {
-      pub += (double)(hb[t * 8 + 7] - hb[t * 8 + 1]);
-      xl += (double)(hb[(t + 1) * 8 + 1] - hb[t * 8 + 7]);
-    }
-    fprintf(stderr, " | total %.0f | publish@%.0f publish->next-barrier %.0f\n", sum / std::max(1, cnt),
-            pub / std::max(1, cnt - 1), xl / std::max(1, cnt - 1));
+    // critical stamps of round t: 0 start, 1 exchanged, 2 scalars, 3 row pass + butterfly,
+    // 4 group barrier, 7 published, 5 projection; bulk stamps: 13 before BAR_Q, 8 after,
+    // 9 lookahead GEMV, 11 reduced, 12 end
+    auto avg = [&](int a, int b, int t0, int t1) {
+      double sacc = 0;
+      int n = 0;
+      for (int t = t0; t < t1; ++t, ++n) sacc += (double)(hb[t * 16 + b] - hb[t * 16 + a]);
+      return n ? sacc / n : 0.0;
+    };
+    const int t0 = 2, t1 = (int)w - 5;
+    double per = 0;
+    for (int t = t0; t < t1; ++t) per += (double)(hb[(t + 1) * 16] - hb[t * 16]);
+    per /= std::max(1, t1 - t0);
+    fprintf(stderr,
+            "[leaf m=%lld w=%lld G=%d RP=%d] cycles/round %.0f | critical: exchange %.0f scalars %.0f rowpass %.0f "
+            "sync %.0f publish %.0f | bulk: wait %.0f gemv %.0f poll %.0f project %.0f busy %.0f\n",
+            (long long)m, (long long)w, G, rp, per, avg(0, 1, t0, t1), avg(1, 2, t0, t1), avg(2, 3, t0, t1),
+            avg(3, 4, t0, t1), avg(4, 7, t0, t1), avg(13, 8, t0, t1), avg(8, 9, t0, t1), avg(9, 10, t0, t1),
+            avg(10, 11, t0, t1), avg(8, 12, t0, t1));
   }
   if (p.dbg2) {
     std::vector<long long> hb((size_t)2 * LEAF_MAX_W * G);
