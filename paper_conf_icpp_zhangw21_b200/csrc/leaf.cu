@@ -78,6 +78,8 @@ __device__ __forceinline__ double pow2d(int e) { return __hiloint2double((1023 +
 
 // per-phase cycle stamps of CTA p.dbg_cta (diagnostics; p.dbg == nullptr in production)
 #define DBG_CTA p.dbg_cta
+#define PRO_STAMP(i)                                                       \
+  if (p.dbg != nullptr && blockIdx.x == DBG_CTA && threadIdx.x == 0) p.dbg[(size_t)LEAF_MAX_W * 16 + (i)] = clock64();
 // bulk-group stamps (slots 8..13 of round t, thread 0 of the bulk group)
 #define BULK_STAMP(i)                                                   \
   if (p.dbg != nullptr && blockIdx.x == DBG_CTA && btid == 0) p.dbg[(size_t)t * 16 + (i)] = clock64();
@@ -167,6 +169,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   __shared__ float tauc[LEAF_MAX_W];                        // breakdown thresholds
   __shared__ double fxs[LEAF_MAX_W][5], fxi[LEAF_MAX_W][5];  // fixed-point scales by (round, class)
   // last-seen exchange words persist across launches (words are never reset, see fx_exp)
+  PRO_STAMP(0);
   for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) xprev[i] = p.xprev_g[i];
 
   const int G = gridDim.x;
@@ -217,6 +220,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     }
   }
   __syncthreads();
+  PRO_STAMP(1);
 
   const float u_work = 5.9604645e-08f;             // 2^-24, fp32 accumulation
   // Bulk GEMV mapping: thread (kq = lane, part = warp) handles values kq and kq + 32
@@ -375,6 +379,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     tauc[k] = (float)p.m_global * u_work * sqrtf(s);
   }
   __syncthreads();
+  PRO_STAMP(2);
   // fixed-point scales 2^fx_exp(t, class) and their inverses, value classes 0..4 (fx_exp)
   for (int i = threadIdx.x; i < w * 5; i += LEAF_THREADS) {
     const int t = i / 5, c = i - t * 5;
@@ -406,6 +411,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   static_assert(BULK_W <= GEMV_PARTS / 2, "part2 holds one row per bulk warp");
   const bool is_crit = threadIdx.x < GROUP;
   const int crit_warps = rows >= GROUP ? GROUP_W : (rows + 31) / 32;   // critical warps owning rows
+  PRO_STAMP(3);
   constexpr int BAR_Q = 4, BAR_W = 6;
   if (is_crit) {
     // row state of this thread's rows rr[j] = tid + 32 CW j, j < NR
@@ -767,7 +773,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       BULK_STAMP(12);
     }
   }
+  PRO_STAMP(4);
   __syncthreads();
+  PRO_STAMP(5);
   // ---- Q: the panel slice (now q_0..q_{w-1} in fp32) rounded once to the storage type ----
   {
     constexpr int V = Vec<T>::N;
@@ -784,6 +792,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       P[r0 + i + (int64_t)j * p.ldp] = Elem<T>::store(sp[j * LD + i]);
     }
   }
+  PRO_STAMP(6);
   // every CTA ends with the same last-seen words; CTA 0 persists them for the next launch
   if (g == 0)
     for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) p.xprev_g[i] = xprev[i];

@@ -340,7 +340,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   p.r0buf = c->d_r0buf;
   p.m_global = c->m_global > 0 ? c->m_global : m;
   p.vec_ok = ((ldp * elem_bytes(prec)) % 16 == 0) && (reinterpret_cast<uintptr_t>(P) % 16 == 0);
-  if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 16 * LEAF_MAX_W);
+  if (dbg && !dbg_buf) cudaMalloc(&dbg_buf, sizeof(long long) * 16 * (LEAF_MAX_W + 1));
   p.dbg = dbg ? dbg_buf : nullptr;
   static const bool dbg2 = getenv("RGSQR_LEAF_DEBUG2") != nullptr;
   static long long* dbg2_buf = nullptr;
@@ -386,8 +386,8 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   const int s = elem_bytes(prec);
   c->kend(0, st, kb, 2.0 * m * w * w, 2.0 * m * w * s + 4.0 * w * w);
   if (p.dbg) {
-    long long hb[16 * LEAF_MAX_W];
-    cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 16 * w, cudaMemcpyDeviceToHost, st);
+    long long hb[16 * (LEAF_MAX_W + 1)];
+    cudaMemcpyAsync(hb, p.dbg, sizeof(long long) * 16 * (LEAF_MAX_W + 1), cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
     // critical stamps of round t: 0 start, 1 exchanged, 2 scalars, 3 row pass + butterfly,
     // 4 group barrier, 7 published, 5 projection; bulk stamps: 13 before BAR_Q, 8 after,
@@ -408,6 +408,13 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
             (long long)m, (long long)w, G, rp, per, avg(0, 1, t0, t1), avg(1, 2, t0, t1), avg(2, 3, t0, t1),
             avg(3, 4, t0, t1), avg(4, 7, t0, t1), avg(13, 8, t0, t1), avg(8, 9, t0, t1), avg(9, 10, t0, t1),
             avg(10, 11, t0, t1), avg(8, 12, t0, t1));
+  }
+  if (p.dbg) {
+    long long pb[8];
+    cudaMemcpyAsync(pb, p.dbg + 16 * LEAF_MAX_W, sizeof(long long) * 8, cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+    fprintf(stderr, "[leaf prologue/epilogue cycles] xprev+load %lld round0 %lld tables %lld rounds %lld join %lld store %lld\n",
+            pb[1] - pb[0], pb[2] - pb[1], pb[3] - pb[2], pb[4] - pb[3], pb[5] - pb[4], pb[6] - pb[5]);
   }
   if (p.dbg2) {
     std::vector<long long> hb((size_t)2 * LEAF_MAX_W * G);
