@@ -199,6 +199,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--skip-e2e", action="store_true")
+    ap.add_argument("--no-ablation", action="store_true", help="skip the split-ratio e2e ablation")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
     wl = WORKLOADS[args.workload]
@@ -356,6 +357,28 @@ def main():
                "ooc_nodes": so["n_ooc_nodes"], "arena_bytes": so["arena_bytes"],
                "gpu_launches": args.steps * sum(so[k] for k in ("n_leaf_launches", "n_tn_launches",
                                                                   "n_nn_launches", "n_other_launches"))}
+        # ablation (not the headline): OOC left child 62.5% of the columns instead of the paper's
+        # halves -- the right child's in-core factorization is the one phase that cannot overlap
+        # host transfers (RGSQR_OPT_SPLIT_PCT)
+        if world == 1 and not args.no_ablation:
+            h.set_option("split_pct", 62)
+            h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
+            torch.cuda.synchronize()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            for _ in range(2):
+                h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
+            a1.record(stream)
+            torch.cuda.synchronize()
+            ms_ab = a0.elapsed_time(a1) / 2
+            sa = h.stats()
+            tl_ab = max(sa["h2d_bytes"] / (link["h2d"] * 1e9), sa["d2h_bytes"] / (link["d2h"] * 1e9),
+                        (sa["h2d_bytes"] + sa["d2h_bytes"]) / (link["duplex_total"] * 1e9))
+            e2e["ablation_split_pct_62"] = {"value": flops / (ms_ab / 1e3) / 1e12, "ms_per_step": ms_ab,
+                                            "h2d_bytes_per_step": sa["h2d_bytes"],
+                                            "d2h_bytes_per_step": sa["d2h_bytes"],
+                                            "roofline_frac": max(t_tensor, tl_ab) / (ms_ab / 1e3)}
+            h.set_option("split_pct", 50)
         for p in (pa, pq, pr):
             h.host_free(p)
     clocks.stop()

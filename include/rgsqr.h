@@ -89,6 +89,10 @@ enum rgsqr_option {
                                    and A2 -= Q1 R12 (Eq. 2) as one kernel that
                                    reads Q1 and A2 once; 0 = the separate TN / NN products.
                                    Default 1 */
+  ,RGSQR_OPT_SPLIT_PCT = 15     /* width of an OUT-OF-CORE node's left child in percent of the node
+                                   (rounded to 64).  50 = "divide evenly its columns into two halves"
+                                   (PAPER.md:115), the default; other values are a scheduling ablation
+                                   (same factorization in exact arithmetic).  In-core nodes always halve */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

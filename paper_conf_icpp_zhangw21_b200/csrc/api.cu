@@ -409,6 +409,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_REORTH: return &o.reorth;
     case RGSQR_OPT_PREFETCH: return &o.prefetch;
     case RGSQR_OPT_FUSE_SMALL: return &o.fuse_small;
+    case RGSQR_OPT_SPLIT_PCT: return &o.split_pct;
   }
   return nullptr;
 }

@@ -29,6 +29,7 @@ struct Options {
   int64_t reorth = 0;        // CGS2 (RGSQR_OPT_REORTH)
   int64_t prefetch = 1;      // OOC: upload the first ring tiles during the left child (RGSQR_OPT_PREFETCH)
   int64_t fuse_small = 1;    // fused kernel for nodes with w1, w2 <= 64 (RGSQR_OPT_FUSE_SMALL)
+  int64_t split_pct = 50;    // OOC split: left child width in % (RGSQR_OPT_SPLIT_PCT; 50 = halves, the paper)
 };
 
 struct KernSeg {

@@ -504,8 +504,14 @@ struct Exec {
   // recursive algorithm (Eq. 2)
   int node(int64_t c0, int64_t w, bool src_q) {
     if (incore_need(w) <= c->arena.free_bytes()) return panel(c0, w, src_q);
-    const int64_t w1 = split_width(w, std::max(1, leaf_width_for(c, m)));
+    int64_t w1 = split_width(w, std::max(1, leaf_width_for(c, m)));
     if (w1 == 0) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "budget cannot hold one leaf panel");
+    if (c->opt.split_pct != 50 && w >= 256) {
+      // ablation (RGSQR_OPT_SPLIT_PCT): a larger left child, factored while the host link is
+      // busy anyway, leaves a shorter right child -- the one phase that cannot overlap transfers
+      const int64_t t = (w * c->opt.split_pct / 100 + 63) / 64 * 64;
+      if (t >= 64 && t <= w - 64) w1 = t;
+    }
     return ooc_node(c0, w1, w - w1, src_q, true);
   }
 
