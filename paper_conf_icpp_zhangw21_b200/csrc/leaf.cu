@@ -633,7 +633,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
           // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
           for (int base = 8 * bw; base < nv4; base += 8 * BULK_W) {
-#pragma unroll 4
+#pragma unroll
             for (int i = base; i < base + 8; ++i) {
               const float4 u = y1[i], v = y2[i], a = xa[i];
               a0 = fmaf(a.x, u.x, a0);
