@@ -312,6 +312,14 @@ def main():
             traffic = t
     roof["traffic"] = traffic
     roof["share_of_step"] = kms[dom] / sum(kms) if sum(kms) else None
+    if dom_name == "leaf":
+        # the leaf is bound by the latency of its dependent grid-wide reductions (one per
+        # column), not by a throughput: its per-column time against the measured floor of that
+        # exchange alone (profiles/r1_leaf_latency.md, scripts/crit_bench.cu variant V12)
+        us_col = kms[dom] * 1e3 / n
+        floor = 0.914
+        roof["latency"] = {"unit": "us per column", "achieved": us_col, "floor": floor, "frac": floor / us_col,
+                           "floor_source": "exchange-only round of 148 CTAs, measured on B200 (crit_bench V12)"}
     kernels = {KERNEL_CLASSES[i]: {"ms": kms[i], "launches": prof["kern_launches"][i],
                                    "tflops": (prof["kern_flops"][i] / (kms[i] / 1e3) / 1e12) if kms[i] else None,
                                    "gbps": (prof["kern_bytes"][i] / (kms[i] / 1e3) / 1e9) if kms[i] else None}

@@ -102,3 +102,26 @@ def test_tf32x3_usv_kappa_1e3(h):
     ref = oracle.gram_cholesky_r(X)
     assert oracle.backward_error(X, Q, R) <= 1e-5
     assert oracle.r_rel_error(R, ref) <= 1e-5
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16"])
+def test_fused_bottom_node_matches_separate_products(h, prec):
+    """The fused bottom-node kernel (small.cu, nodes with w1, w2 <= 64) against the separate
+    TN / NN products: both reach the oracle's R (Eq. 2), they differ only in
+    the order of the fp32 sums; a ragged m exercises the partial last row slice."""
+    m, n = 12345, 256
+    st = {"fp16": "fp16", "bf16": "bf16"}[prec]
+    A = gi.gaussian(m, n, seed=11, dtype=st)
+    X = gi.to_float64(A, st)
+    ref = oracle.rgs(X, leaf=64)
+    out = {}
+    for fuse in (0, 1):
+        h.set_option("fuse_small", fuse)
+        rc, Q, R = run(h, A, st, prec, m, n)
+        assert rc == 0
+        out[fuse] = (Q, R)
+        be = oracle.backward_error(X, Q, R)
+        re = oracle.r_rel_error(R, ref.R)
+        assert be < 5e-3 and re < 5e-3, (fuse, be, re)
+    h.set_option("fuse_small", 1)
+    assert oracle.r_rel_error(out[1][1], out[0][1]) < 2e-3
