@@ -69,7 +69,7 @@ def test_outer_product(h, prec, storage, m, w1, w2):
 
 
 @pytest.mark.parametrize("prec,storage", PRECS)
-@pytest.mark.parametrize("m,w", [(20000, 64), (4096, 32), (1000, 7), (300, 64), (65536, 64)])
+@pytest.mark.parametrize("m,w", [(20000, 64), (4096, 32), (1000, 7), (300, 64), (65536, 64), (131072, 48), (262144, 24)])
 def test_leaf_cgs(h, prec, storage, m, w):
     A = _rand(m, w, 31, storage)
     X = gi.to_float64(A, storage)
