@@ -147,7 +147,7 @@ constexpr int NCCL_INT64 = 4, NCCL_FLOAT32 = 7, NCCL_FLOAT64 = 8;
 int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2,
              int64_t lda, int64_t m, int64_t w1, int64_t w2, cudaStream_t st);
 int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float* R11, int64_t ldr,
-            int64_t col_offset, cudaStream_t st);
+            int64_t col_offset, cudaStream_t st, bool r0_pre = false);
 int leaf_width_for(Ctx* c, int64_t m);
 int64_t split_width(int64_t w, int64_t leaf);
 

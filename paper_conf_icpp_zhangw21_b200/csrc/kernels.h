@@ -74,7 +74,8 @@ struct LeafParams {
   unsigned long long* xprev_g;          // [LEAF_XW_WORDS] last-seen words, persistent
   int nranks;               // GPUs sharing the rows of the panel
   int sys;                  // distributed context: red.add into every rank's words, .sys scope
-  int r0_mode;              // 0 round 0 in-kernel, 1 round-0-only (write r0buf), 2 round 0 given
+  int r0_mode;              // 0 round 0 in-kernel, 1 round-0-only (write r0buf), 2 round 0 given,
+                            // 3 per-CTA round-0 partials already in `partials` (fused node)
   float* r0buf;             // [LEAF_MAX_W+2] round-0 vector (modes 1, 2)
   int64_t m_global;         // total rows (breakdown threshold)
   int* breakdown;           // device int, atomicMin of the first breakdown column
@@ -96,6 +97,8 @@ struct SmallNodeParams {
   float* partials;          // [grid][4096]
   void* r12op;              // [64][64] operand copy ([j][i])
   unsigned* counter;        // zeroed by the launcher
+  float* r0_partials;       // non-null: also write the next leaf's round-0 partials of the new A2
+                            // ([k][grid]: ||a_k||^2, k < w2, then a_0.a_1) -- leaf r0_mode 3
 };
 constexpr int SN_MAX_RP = 768;  // rows per CTA the fused bottom node holds in shared memory
 size_t small_node_smem(int rp);

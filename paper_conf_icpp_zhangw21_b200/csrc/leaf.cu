@@ -322,6 +322,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   // (r0_mode 2: the globally reduced round-0 vector is given in p.r0buf)
   if (p.r0_mode != 2) {
     const int L = round_len(0);
+    if (p.r0_mode != 3) {   // (mode 3: the partials were written by the preceding fused node)
     for (int k = kq; k < L; k += 32) {
       int cx = k < w ? k : 0, cy = k < w ? k : 1;
       part[warp][k] = dot4(cx, cy);
@@ -338,6 +339,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       } while (cv < (unsigned)G);
     }
     __syncthreads();
+    }
     constexpr int KPW = (LEAF_MAX_W + 2 + LEAF_WARPS - 1) / LEAF_WARPS;
     constexpr int QMAX = (LEAF_MAX_G + 31) / 32;
     float v[KPW][QMAX];

@@ -310,7 +310,7 @@ int leaf_width_for(Ctx* c, int64_t m) {
 }
 
 int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float* R11, int64_t ldr,
-            int64_t col_offset, cudaStream_t st) {
+            int64_t col_offset, cudaStream_t st, bool r0_pre) {
   int G, rp;
   leaf_geometry(c, m, &G, &rp);
   if (rp > LEAF_MAX_RP)
@@ -367,7 +367,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   cudaError_t e;
   cudaEvent_t kb = c->kbegin(st);
   if (!c->nccl_comm) {
-    p.r0_mode = 0;
+    p.r0_mode = r0_pre ? 3 : 0;
     e = launch(p);
   } else {
     // row-sharded: round 0 (column norms -> fixed-point scales) is summed over GPUs by NCCL
@@ -449,7 +449,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
 // fused bottom node (small.cu): returns 1 when done, 0 when the shape / precision / context
 // is not covered (the caller then runs the separate products), < 0 on error
 int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64_t lda, int64_t m, int64_t w1,
-                  int64_t w2, float* R12, int64_t ldr, cudaStream_t st) {
+                  int64_t w2, float* R12, int64_t ldr, cudaStream_t st, bool r0_for_leaf) {
   if (!c->opt.fuse_small || c->nccl_comm || w1 > 64 || w2 > 64 || w1 < 1 || w2 < 1) return 0;
   if (prec != RGSQR_FP16 && prec != RGSQR_BF16) return 0;
   int G, rp;
@@ -471,6 +471,7 @@ int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64
   p.partials = c->d_sn_partials;
   p.r12op = c->d_sn_r12op;
   p.counter = c->d_counter + 16;
+  p.r0_partials = r0_for_leaf ? c->d_partials : nullptr;
   cudaEvent_t kb = c->kbegin(st);
   cudaError_t e = prec == RGSQR_FP16 ? launch_small_node<__half>(p, G, st) : launch_small_node<__nv_bfloat16>(p, G, st);
   if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("fused node launch: ") + cudaGetErrorString(e));
@@ -527,6 +528,7 @@ struct IncoreCtx {
   // deferred products of nodes whose A2 was still being uploaded: R12 = Q1^T A2 and
   // A2 -= Q1 R12 applied chunk by chunk when a descendant first needs the columns
   // (applied in creation order = ancestors first, as the recursion would have)
+  bool r0_pre = false;   // the next leaf's round-0 partials were written by the fused node
   struct Deferred {
     int64_t c0, w1, end, applied;
   };
@@ -567,7 +569,8 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
     }
     char* P = k.A + c0 * k.lda * k.s;
     float* R11 = k.R + c0 + c0 * k.ldr;
-    int rc = op_leaf(k.c, k.prec, P, k.lda, k.m, w, R11, k.ldr, k.col_offset + c0, k.st);
+    const bool pre = k.r0_pre && !(k.hooks && k.hooks->need && k.hooks->pending && k.hooks->pending(c0 + w));
+    int rc = op_leaf(k.c, k.prec, P, k.lda, k.m, w, R11, k.ldr, k.col_offset + c0, k.st, pre);
     if (rc == 0 && k.S11) {
       // CGS2 leaf: factor Q' again, Q' = Q S, and R11 <- S R11
       rc = op_leaf(k.c, k.prec, P, k.lda, k.m, w, k.S11, w, k.col_offset + c0, k.st);
@@ -598,10 +601,18 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
     if (rc < 0) return rc;
   }
   if (!k.S) {
-    rc = op_small_node(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.st);
+    // when the right child is a leaf, the fused kernel also hands it its round-0 partials
+    const bool right_leaf = split_width(w2, k.leaf) == 0;
+    rc = op_small_node(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.st, right_leaf);
     if (rc < 0) return rc;
     if (rc == 1) {   // done by the fused kernel
       k.c->stats.n_incore_nodes++;
+      if (right_leaf) {
+        k.r0_pre = true;
+        rc = incore_rec(k, h, w2);
+        k.r0_pre = false;
+        return rc;
+      }
       return incore_rec(k, h, w2);
     }
   }

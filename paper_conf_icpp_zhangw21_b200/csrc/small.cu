@@ -28,7 +28,7 @@ __host__ __device__ inline int sn_stride(int rp) {
   return r16 + ((8 - (r16 % 64)) + 64) % 64;
 }
 
-size_t small_node_smem(int rp) { return (size_t)2 * 64 * sn_stride(rp) * 2 + 64 * SN_RS * 2 + 8 * 33 * 4 + 64; }
+size_t small_node_smem(int rp) { return (size_t)2 * 64 * sn_stride(rp) * 2 + 64 * SN_RS * 2 + 8 * 65 * 4 + 64; }
 
 template <typename T>
 struct MmaOp;
@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
   T* qs = reinterpret_cast<T*>(smem);            // [64][S]: column i of the Q1 slice
   T* as = qs + 64 * S;                           // [64][S]: column j of the A2 slice
   T* rs = as + 64 * S;                           // [64][SN_RS]: R12 operand as [j][i]
-  float* red = reinterpret_cast<float*>(rs + 64 * SN_RS);   // [8][33]
+  float* red = reinterpret_cast<float*>(rs + 64 * SN_RS);   // [8][33] phase 2, [8][65] phase 3
   const int G = gridDim.x, g = blockIdx.x;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t r0 = (int64_t)g * RP;
@@ -191,6 +191,10 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
     }
     __syncthreads();
     const int q = lane >> 3, l8 = lane & 7;
+    // the next leaf's round 0 (leaf r0_mode 3): squares of the ROUNDED A2' values per column
+    // (and a_0.a_1), accumulated from the epilogue registers, reduced in a fixed order below
+    float nrm[8][2] = {};
+    float d01 = 0.f;
     for (int mt = warp; mt < RP16 / 16; mt += SN_THREADS / 32) {
       float acc[8][4] = {};
 #pragma unroll
@@ -208,13 +212,56 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
         const int r = 16 * mt + (lane >> 2), j = 8 * n + 2 * (lane & 3);
         T* c0 = as + j * S + r;
         T* c1 = as + (j + 1) * S + r;
-        c0[0] = Elem<T>::store(Elem<T>::load(c0[0]) - acc[n][0]);
-        c1[0] = Elem<T>::store(Elem<T>::load(c1[0]) - acc[n][1]);
-        c0[8] = Elem<T>::store(Elem<T>::load(c0[8]) - acc[n][2]);
-        c1[8] = Elem<T>::store(Elem<T>::load(c1[8]) - acc[n][3]);
+        const T v00 = Elem<T>::store(Elem<T>::load(c0[0]) - acc[n][0]);
+        const T v01 = Elem<T>::store(Elem<T>::load(c1[0]) - acc[n][1]);
+        const T v10 = Elem<T>::store(Elem<T>::load(c0[8]) - acc[n][2]);
+        const T v11 = Elem<T>::store(Elem<T>::load(c1[8]) - acc[n][3]);
+        c0[0] = v00;
+        c1[0] = v01;
+        c0[8] = v10;
+        c1[8] = v11;
+        const float f00 = Elem<T>::load(v00), f01 = Elem<T>::load(v01), f10 = Elem<T>::load(v10),
+                    f11 = Elem<T>::load(v11);
+        nrm[n][0] = fmaf(f00, f00, fmaf(f10, f10, nrm[n][0]));
+        nrm[n][1] = fmaf(f01, f01, fmaf(f11, f11, nrm[n][1]));
+        if (n == 0) d01 = fmaf(f00, f01, fmaf(f10, f11, d01));   // columns 0, 1 on lanes with tig 0
+      }
+    }
+    if (p.r0_partials != nullptr) {
+      // lanes sharing tig (= lane & 3) hold the same columns: xor tree over the row groups
+#pragma unroll
+      for (int n = 0; n < 8; ++n)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) {
+          float v = nrm[n][c];
+          v += __shfl_xor_sync(0xffffffffu, v, 4);
+          v += __shfl_xor_sync(0xffffffffu, v, 8);
+          v += __shfl_xor_sync(0xffffffffu, v, 16);
+          nrm[n][c] = v;
+        }
+      d01 += __shfl_xor_sync(0xffffffffu, d01, 4);
+      d01 += __shfl_xor_sync(0xffffffffu, d01, 8);
+      d01 += __shfl_xor_sync(0xffffffffu, d01, 16);
+      if (lane < 4) {
+#pragma unroll
+        for (int n = 0; n < 8; ++n) {
+          red[warp * 65 + 8 * n + 2 * lane] = nrm[n][0];
+          red[warp * 65 + 8 * n + 2 * lane + 1] = nrm[n][1];
+        }
+        if (lane == 0) red[warp * 65 + 64] = d01;
       }
     }
     __syncthreads();
+    if (p.r0_partials != nullptr) {
+      const int L = p.w2 + (p.w2 > 1 ? 1 : 0);
+      for (int k = threadIdx.x; k < L; k += SN_THREADS) {
+        const int col = k < p.w2 ? k : 64;
+        float v = red[col];
+#pragma unroll
+        for (int wv = 1; wv < SN_THREADS / 32; ++wv) v += red[wv * 65 + col];
+        p.r0_partials[(size_t)k * G + g] = v;
+      }
+    }
     // ---- store A2' (columns < w2, rows < rows) ----
     const int nv = p.vec_ok ? rows / 8 : 0;
     for (int idx = threadIdx.x; idx < p.w2 * nv; idx += SN_THREADS) {
