@@ -14,8 +14,11 @@ using namespace rgsqr;
 namespace rgsqr {
 
 int ensure_arena(Ctx* c, size_t want) {
-  if (c->arena.base && c->arena.size >= want && c->arena.size <= want + ((size_t)64 << 20)) {
+  if (c->arena.base && c->arena.phys >= want && c->arena.phys <= want + ((size_t)64 << 20)) {
+    // reuse the allocation, but the budget stays exact: plans never depend on call history
+    c->arena.size = want;
     c->arena.top = 0;
+    c->arena.high = 0;
     return RGSQR_OK;
   }
   if (c->arena.base) {
@@ -28,6 +31,7 @@ int ensure_arena(Ctx* c, size_t want) {
     return fail(c, RGSQR_ERR_CUDA, "arena cudaMalloc(" + std::to_string(want) + "): " + cudaGetErrorString(e));
   c->arena.base = static_cast<char*>(p);
   c->arena.size = want;
+  c->arena.phys = want;
   c->arena.top = 0;
   c->arena.high = 0;
   return RGSQR_OK;
@@ -37,7 +41,7 @@ size_t resolve_budget(Ctx* c, size_t budget) {
   if (budget != 0) return budget;
   size_t fr = 0, tot = 0;
   cudaMemGetInfo(&fr, &tot);
-  size_t mine = c->arena.base ? c->arena.size : 0;
+  size_t mine = c->arena.base ? c->arena.phys : 0;
   size_t avail = fr + mine;
   const size_t reserve = (size_t)512 << 20;
   return avail > reserve ? avail - reserve : avail / 2;

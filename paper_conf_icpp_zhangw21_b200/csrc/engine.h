@@ -41,7 +41,8 @@ struct KernSeg {
 // Bump allocator over one cudaMalloc of at most the budget; LIFO release by mark.
 struct Arena {
   char* base = nullptr;
-  size_t size = 0;
+  size_t size = 0;             // this call's budget (the planner sees exactly this much)
+  size_t phys = 0;             // bytes actually allocated (a reused allocation may be larger)
   size_t top = 0;
   size_t high = 0;
   void* alloc(size_t bytes) {

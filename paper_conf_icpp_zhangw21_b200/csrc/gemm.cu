@@ -228,9 +228,13 @@ struct NNCfg {
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int CBOX_N = 64;                                 // columns per C TMA box
   static constexpr int C_BYTES = BM * BN * (int)sizeof(T);
-  static constexpr int STAGES_RAW = (220 * 1024 - C_BYTES - 2048) / STAGE_BYTES;
+  // two C tiles (the old-A2 load of tile j+1 overlaps the epilogue of tile j) when at least
+  // three k-stages still fit; otherwise one
+  static constexpr int STAGES2 = (220 * 1024 - 2 * C_BYTES - 2048) / STAGE_BYTES;
+  static constexpr int C_BUFS = STAGES2 >= 3 ? 2 : 1;
+  static constexpr int STAGES_RAW = (220 * 1024 - C_BUFS * C_BYTES - 2048) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + C_BYTES + 1024 + 512;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + C_BUFS * C_BYTES + 1024 + 512;
   static constexpr uint32_t TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
   static constexpr uint32_t IDESC = ptx::idesc_f32acc(Elem<T>::kUmmaFormat, 1u, 0u, BM, BN);
   static_assert(STAGES >= 2, "NN tile does not fit shared memory");
@@ -245,14 +249,14 @@ __global__ void __launch_bounds__(256, 1)
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = ptx::smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
-  T* Cs = reinterpret_cast<T*>(smem + C::STAGES * C::STAGE_BYTES);
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES + C::C_BYTES);
+  T* Cs0 = reinterpret_cast<T*>(smem + C::STAGES * C::STAGE_BYTES);   // [C_BUFS] C tiles
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES + C::C_BUFS * C::C_BYTES);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;   // [2]
   uint64_t* tempty = tfull + 2;          // [2]
-  uint64_t* cfull = tempty + 2;
-  uint64_t* cempty = cfull + 1;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(cempty + 1);
+  uint64_t* cfull = tempty + 2;          // [C_BUFS]
+  uint64_t* cempty = cfull + C::C_BUFS;  // [C_BUFS]
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(cempty + C::C_BUFS);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_tiles = p.tiles_m * p.tiles_n;
@@ -270,8 +274,10 @@ __global__ void __launch_bounds__(256, 1)
       ptx::mbar_init(&tfull[b], 1);
       ptx::mbar_init(&tempty[b], 4);
     }
-    ptx::mbar_init(cfull, 1);
-    ptx::mbar_init(cempty, 1);
+    for (int b = 0; b < C::C_BUFS; ++b) {
+      ptx::mbar_init(&cfull[b], 1);
+      ptx::mbar_init(&cempty[b], 1);
+    }
     ptx::fence_mbar_init();
   }
   if (warp == 2) ptx::tmem_alloc<C::TMEM_COLS>(tslot);
@@ -332,11 +338,14 @@ __global__ void __launch_bounds__(256, 1)
       int lt = 0;
       for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++lt) {
         const int32_t m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * BN;
-        ptx::mbar_wait(cempty, ((uint32_t)lt & 1u) ^ 1u);
-        ptx::mbar_arrive_expect_tx(cfull, C::C_BYTES);
+        const int cbuf = lt % C::C_BUFS;
+        const uint32_t cph = (uint32_t)(lt / C::C_BUFS) & 1u;
+        T* Cs = Cs0 + cbuf * (C::C_BYTES / (int)sizeof(T));
+        ptx::mbar_wait(&cempty[cbuf], cph ^ 1u);
+        ptx::mbar_arrive_expect_tx(&cfull[cbuf], C::C_BYTES);
 #pragma unroll
         for (int cb = 0; cb < BN / C::CBOX_N; ++cb)
-          ptx::tma_load_2d(Cs + cb * C::CBOX_N * C::BM, &mapC, cfull, m0, n0 + cb * C::CBOX_N);
+          ptx::tma_load_2d(Cs + cb * C::CBOX_N * C::BM, &mapC, &cfull[cbuf], m0, n0 + cb * C::CBOX_N);
       }
     }
   } else if (warp >= 4) {
@@ -346,9 +355,11 @@ __global__ void __launch_bounds__(256, 1)
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++lt) {
       const int32_t m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * BN;
       const int b = lt & 1;
+      const int cbuf = lt % C::C_BUFS;
+      T* Cs = Cs0 + cbuf * (C::C_BYTES / (int)sizeof(T));
       ptx::mbar_wait(&tfull[b], (uint32_t)(lt >> 1) & 1u);
       ptx::tc_fence_after();
-      ptx::mbar_wait(cfull, (uint32_t)lt & 1u);
+      ptx::mbar_wait(&cfull[cbuf], (uint32_t)(lt / C::C_BUFS) & 1u);
 #pragma unroll 1
       for (int cc = 0; cc < BN / 32; ++cc) {
         uint32_t v[32];
@@ -371,7 +382,7 @@ __global__ void __launch_bounds__(256, 1)
           ptx::tma_store_2d(&mapC, Cs + cb * C::CBOX_N * C::BM, m0, n0 + cb * C::CBOX_N);
         ptx::bulk_commit();
         ptx::bulk_wait_read0();
-        ptx::mbar_arrive(cempty);
+        ptx::mbar_arrive(&cempty[cbuf]);
       }
     }
     if (ew == 0 && lane == 0) ptx::bulk_wait0();

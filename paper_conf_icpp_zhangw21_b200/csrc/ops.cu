@@ -206,6 +206,9 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   const int EPB = 128 / s;
   int bn = pick_bn(w2);
   if (s == 4) bn = std::min(bn, 128);  // fp32 C tile must leave room for the k-ring
+  // short K (w1 <= 1024): the tile is bound by moving the old A2 tile in and A2' out; 128-wide
+  // tiles leave room for two C buffers, so the next tile's load overlaps this tile's epilogue
+  if (s == 2 && w1 <= 1024) bn = std::min(bn, 128);
   CUtensorMap ma, mb, mc;
   std::string err;
   if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
