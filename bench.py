@@ -163,6 +163,9 @@ def cpu_oracle_sample(A, storage, cols, leaf=64):
     return 2.0 * m * cols * cols / dt / 1e12, dt
 
 
+METRIC = "OOC QR TFLOPS (2mn^2) and % of min(tensor-peak, PCIe roofline)"
+
+
 def run_reference(args, wl, rank):
     if rank != 0:
         return
@@ -180,11 +183,12 @@ def run_reference(args, wl, rank):
     value = float(np.mean(vals))
     sample = (f"oracle O3 (fp64 recursive CGS, numpy/OpenBLAS, leaf 64) on {m}x{cols} "
               f"(first {cols} columns of the {args.workload} input), per step")
-    line = {"impl": "reference", "metric": "OOC QR TFLOPS (2mn^2)", "value": value, "unit": "TFLOPS",
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "TFLOPS",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * float(np.mean(times)), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": wl["desc"], "m": m, "n": n, "sample_cols": cols},
+            "config": {"workload": wl["desc"], "m": m, "n": n, "precision": prec,
+                       "device_budget_bytes": wl["budget"], "sample_cols": cols},
             "cpu_baseline": {"value": value, "unit": "TFLOPS", "cores": cores, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": "TFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -401,7 +405,7 @@ def main():
                          f"of the same input), {dt:.1f} s"}
 
     if rank == 0:
-        line = {"metric": "OOC QR TFLOPS (2mn^2) and % of min(tensor-peak, PCIe roofline)",
+        line = {"metric": METRIC,
                 "value": value, "unit": "TFLOPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": ms_dev, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": DTYPE_NAME[prec], "data": "synthetic",
