@@ -85,10 +85,11 @@ enum rgsqr_option {
                                    left child is being factored (cross-operation overlap,
                                    PAPER.md:231-233; tiles then start at full height instead of
                                    the ramp).  Default 1 */
-  ,RGSQR_OPT_FUSE_SMALL = 14    /* 1 = nodes with w1, w2 <= 64 (fp16/bf16, one GPU) run R12 = Q1^T A2
+  ,RGSQR_OPT_FUSE_SMALL = 14    /* 1 = nodes with w1, w2 <= 128 (fp16/bf16, one GPU) run R12 = Q1^T A2
                                    and A2 -= Q1 R12 (Eq. 2) as one kernel that
                                    reads Q1 and A2 once; 0 = the separate TN / NN products.
-                                   Default 1 */
+                                   Default 1 = nodes with w1, w2 <= 64; 2 = also up to 128 (A2 in
+                                   two halves; measured slower at m = 65536, kept for study) */
   ,RGSQR_OPT_SPLIT_PCT = 15     /* width of an OUT-OF-CORE node's left child in percent of the node
                                    (rounded to 64).  50 = "divide evenly its columns into two halves"
                                    (PAPER.md:115), the default; other values are a scheduling ablation

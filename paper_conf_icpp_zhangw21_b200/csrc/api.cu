@@ -158,8 +158,8 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_d2r, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
-      cudaMalloc(&c->d_sn_partials, sizeof(float) * LEAF_MAX_G * 4096) != cudaSuccess ||
-      cudaMalloc(&c->d_sn_r12op, 64 * 64 * 4) != cudaSuccess ||
+      cudaMalloc(&c->d_sn_partials, sizeof(float) * LEAF_MAX_G * 128 * 128) != cudaSuccess ||
+      cudaMalloc(&c->d_sn_r12op, 128 * 128 * 4) != cudaSuccess ||
       cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess ||
       cudaMalloc(&c->d_xw, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
       cudaMalloc(&c->d_xprev, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||

@@ -82,7 +82,7 @@ struct LeafParams {
   int64_t col_offset;       // global index of the panel's first column
 };
 
-// fused bottom node (small.cu): R12 = Q1^T A2, A2 -= Q1 R12 for w1, w2 <= 64, fp16/bf16
+// fused bottom nodes (small.cu): R12 = Q1^T A2, A2 -= Q1 R12 for w1, w2 <= 128, fp16/bf16
 struct SmallNodeParams {
   const void* Q1;
   int64_t ldq;
@@ -94,14 +94,14 @@ struct SmallNodeParams {
   int vec_ok;               // Q1/A2 16-byte aligned columns
   float* R12;               // fp32 out, ldr
   int64_t ldr;
-  float* partials;          // [grid][4096]
-  void* r12op;              // [64][64] operand copy ([j][i])
+  float* partials;          // [grid][W*W], W = 64 or 128
+  void* r12op;              // [W][W] operand copy ([j][i])
   unsigned* counter;        // zeroed by the launcher
   float* r0_partials;       // non-null: also write the next leaf's round-0 partials of the new A2
                             // ([k][grid]: ||a_k||^2, k < w2, then a_0.a_1) -- leaf r0_mode 3
 };
 constexpr int SN_MAX_RP = 768;  // rows per CTA the fused bottom node holds in shared memory
-size_t small_node_smem(int rp);
+size_t small_node_smem(int rp, int w);
 template <typename T>
 cudaError_t launch_small_node(const SmallNodeParams& p, int grid, cudaStream_t st);
 

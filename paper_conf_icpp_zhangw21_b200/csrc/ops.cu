@@ -449,15 +449,19 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   return RGSQR_OK;
 }
 
-// fused bottom node (small.cu): returns 1 when done, 0 when the shape / precision / context
-// is not covered (the caller then runs the separate products), < 0 on error
+// fused bottom node (small.cu): returns 1 when done (2: and the right child leaf's round-0
+// partials were written), 0 when the shape / precision / context is not covered (the caller
+// then runs the separate products), < 0 on error
 int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64_t lda, int64_t m, int64_t w1,
                   int64_t w2, float* R12, int64_t ldr, cudaStream_t st, bool r0_for_leaf) {
-  if (!c->opt.fuse_small || c->nccl_comm || w1 > 64 || w2 > 64 || w1 < 1 || w2 < 1) return 0;
+  if (!c->opt.fuse_small || c->nccl_comm || w1 > 128 || w2 > 128 || w1 < 1 || w2 < 1) return 0;
   if (prec != RGSQR_FP16 && prec != RGSQR_BF16) return 0;
+  const int W = (w1 <= 64 && w2 <= 64) ? 64 : 128;
+  if (W == 128 && c->opt.fuse_small < 2) return 0;   // measured slower than the separate products
   int G, rp;
   leaf_geometry(c, m, &G, &rp);
-  if (rp > SN_MAX_RP || small_node_smem(rp) > 227 * 1024) return 0;
+  if (rp > SN_MAX_RP || small_node_smem(rp, W) > 227 * 1024) return 0;
+  r0_for_leaf = r0_for_leaf && W == 64;   // the 128-wide instance does not produce them
   SmallNodeParams p{};
   p.Q1 = Q1;
   p.ldq = ldq;
@@ -480,7 +484,7 @@ int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64
   if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("fused node launch: ") + cudaGetErrorString(e));
   c->kend(3, st, kb, 4.0 * m * w1 * w2, 2.0 * m * (w1 + w2) + 2.0 * m * w2 + 4.0 * w1 * w2);
   c->stats.n_other_launches++;
-  return 1;
+  return r0_for_leaf ? 2 : 1;
 }
 
 // ---------------------------------------------------------------------------------
@@ -608,9 +612,9 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
     const bool right_leaf = split_width(w2, k.leaf) == 0;
     rc = op_small_node(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.st, right_leaf);
     if (rc < 0) return rc;
-    if (rc == 1) {   // done by the fused kernel
+    if (rc >= 1) {   // done by the fused kernel (2: it also wrote the right leaf's round 0)
       k.c->stats.n_incore_nodes++;
-      if (right_leaf) {
+      if (rc == 2) {
         k.r0_pre = true;
         rc = incore_rec(k, h, w2);
         k.r0_pre = false;

@@ -19,7 +19,16 @@
 namespace rgsqr {
 
 static constexpr int SN_THREADS = 256;
-static constexpr int SN_RS = 72;   // R12 operand tile stride (halves): 144 B == 16 (mod 128)
+
+// W: the widest w1 / w2 the instance handles (64 or 128).  A2 is processed in NH = W / 64
+// column halves of 64, so the slices fit shared memory; R12 is W x W.
+template <int W>
+struct SNCfg {
+  static constexpr int NH = W / 64;
+  static constexpr int RS = W + 8;       // R12 operand tile stride (halves): 2 RS == 16 (mod 128)
+  static constexpr int E = W * W;        // R12 entries
+  static constexpr int MT = W / 16;      // m-tiles of R12 in phase 1 (= n-tiles per warp)
+};
 
 // shared-memory column stride (halves) of a row slice: >= rows rounded to 16, and
 // 2 * stride == 16 (mod 128) bytes so that ldmatrix row addresses hit distinct banks
@@ -28,7 +37,9 @@ __host__ __device__ inline int sn_stride(int rp) {
   return r16 + ((8 - (r16 % 64)) + 64) % 64;
 }
 
-size_t small_node_smem(int rp) { return (size_t)2 * 64 * sn_stride(rp) * 2 + 64 * SN_RS * 2 + 8 * 65 * 4 + 64; }
+size_t small_node_smem(int rp, int w) {
+  return (size_t)(w + 64) * sn_stride(rp) * 2 + (size_t)64 * (w + 8) * 2 + 8 * 65 * 4 + 64;
+}
 
 template <typename T>
 struct MmaOp;
@@ -79,131 +90,139 @@ __device__ __forceinline__ void sn_grid_barrier(unsigned* counter, unsigned targ
   __syncthreads();
 }
 
+// columns [c0, c0 + ncols) of a column-major m x * operand, rows [r0, r0 + rows), into a
+// [ncols_alloc][S] shared slice (zero-padded): cp.async 16-byte copies + scalar tail
 template <typename T>
+__device__ __forceinline__ void sn_load_cols(T* dst, int S, const T* src, int64_t ld, int64_t r0, int rows, int c0,
+                                             int ncols, int ncols_alloc, bool vec_ok) {
+  const int nv = vec_ok ? rows / 8 : 0;
+  for (int idx = threadIdx.x; idx < ncols_alloc * (S / 8); idx += SN_THREADS) {
+    const int c = idx / (S / 8), v = idx - c * (S / 8);
+    const bool in = v < nv && c < ncols;
+    const T* sp = in ? src + r0 + 8 * v + (int64_t)(c0 + c) * ld : src;
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"((unsigned)__cvta_generic_to_shared(dst + c * S + 8 * v)),
+                 "l"(sp), "r"(in ? 16 : 0)
+                 : "memory");
+  }
+  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+  __syncthreads();
+  const int tl = rows - 8 * nv;
+  for (int idx = threadIdx.x; idx < ncols * tl; idx += SN_THREADS) {
+    const int c = idx / tl, r = 8 * nv + (idx - c * tl);
+    dst[c * S + r] = src[r0 + r + (int64_t)(c0 + c) * ld];
+  }
+  __syncthreads();
+}
+
+template <typename T, int W>
 __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodeParams p) {
+  using C = SNCfg<W>;
   extern __shared__ __align__(16) unsigned char smem[];
   const int RP = p.rows_per_cta;
   const int S = sn_stride(RP);
   const int RP16 = (RP + 15) & ~15;
-  T* qs = reinterpret_cast<T*>(smem);            // [64][S]: column i of the Q1 slice
-  T* as = qs + 64 * S;                           // [64][S]: column j of the A2 slice
-  T* rs = as + 64 * S;                           // [64][SN_RS]: R12 operand as [j][i]
-  float* red = reinterpret_cast<float*>(rs + 64 * SN_RS);   // [8][33] phase 2, [8][65] phase 3
+  T* qs = reinterpret_cast<T*>(smem);            // [W][S]: column i of the Q1 slice
+  T* as = qs + W * S;                            // [64][S]: column j of the current A2 half
+  T* rs = as + 64 * S;                           // [64][RS]: R12 operand of the half as [j][i]
+  float* red = reinterpret_cast<float*>(rs + 64 * C::RS);   // [8][33] phase 2, [8][65] phase 3
   const int G = gridDim.x, g = blockIdx.x;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int q = lane >> 3, l8 = lane & 7;
   const int64_t r0 = (int64_t)g * RP;
   const int64_t rem = p.m - r0;
   const int rows = rem <= 0 ? 0 : (rem < RP ? (int)rem : RP);
   const T* Q1 = static_cast<const T*>(p.Q1);
   T* A2 = static_cast<T*>(p.A2);
+  const bool vec = p.vec_ok != 0;
 
-  // ---- load the slices (zero-padded to 64 columns and RP16 rows): cp.async, all in flight ----
-  {
-    const int nv = p.vec_ok ? rows / 8 : 0;      // 16-byte vectors per column
-    for (int idx = threadIdx.x; idx < 64 * (S / 8); idx += SN_THREADS) {
-      const int c = idx / (S / 8), v = idx - c * (S / 8);
-      const bool inq = v < nv && c < p.w1, ina = v < nv && c < p.w2;
-      const T* srcq = inq ? Q1 + r0 + 8 * v + (int64_t)c * p.ldq : Q1;
-      const T* srca = ina ? A2 + r0 + 8 * v + (int64_t)c * p.lda : A2;
-      asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"((unsigned)__cvta_generic_to_shared(qs + c * S + 8 * v)),
-                   "l"(srcq), "r"(inq ? 16 : 0)
-                   : "memory");
-      asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"((unsigned)__cvta_generic_to_shared(as + c * S + 8 * v)),
-                   "l"(srca), "r"(ina ? 16 : 0)
-                   : "memory");
-    }
-    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
-    __syncthreads();
-    for (int idx = threadIdx.x; idx < 64 * (rows - 8 * nv); idx += SN_THREADS) {
-      const int c = idx / (rows - 8 * nv), r = 8 * nv + (idx - c * (rows - 8 * nv));
-      if (c < p.w1) qs[c * S + r] = Q1[r0 + r + (int64_t)c * p.ldq];
-      if (c < p.w2) as[c * S + r] = A2[r0 + r + (int64_t)c * p.lda];
-    }
-    __syncthreads();
-  }
-
-  // ---- phase 1: partial = Q1_s^T A2_s; warp: m-tile (16 rows of R12) warp & 3, n-tiles
-  //      (warp >> 2) * 4 .. + 3 (8 columns each) ----
-  {
-    const int mt = warp & 3, nt0 = (warp >> 2) * 4;
-    float acc[4][4] = {};
-    const int q = lane >> 3, l8 = lane & 7;
+  // ---- phase 1: partial = Q1_s^T A2_s (W x W); per A2 half: warp = m-tile warp % MT,
+  //      n-tiles (warp / MT) * MT .. + MT - 1 of the half ----
+  sn_load_cols(qs, S, Q1, p.ldq, r0, rows, 0, p.w1, W, vec);
+  float* P = p.partials + (size_t)g * C::E;      // [j][i], i contiguous
+  for (int hh = 0; hh < C::NH; ++hh) {
+    sn_load_cols(as, S, static_cast<const T*>(A2), p.lda, r0, rows, 64 * hh, max(0, min(64, p.w2 - 64 * hh)), 64, vec);
+    const int mt = warp % C::MT, nt0 = (warp / C::MT) * C::MT;
+    float acc[C::MT][4] = {};
     for (int kk = 0; kk < RP16; kk += 16) {
-      uint32_t a[4], b[2][4];
+      uint32_t a[4], b[C::MT / 2][4];
       ldsm_x4(a, qs + (16 * mt + (q & 1) * 8 + l8) * S + kk + (q >> 1) * 8);
 #pragma unroll
-      for (int h = 0; h < 2; ++h)
+      for (int h = 0; h < C::MT / 2; ++h)
         ldsm_x4(b[h], as + (8 * (nt0 + 2 * h + (q >> 1)) + l8) * S + kk + (q & 1) * 8);
 #pragma unroll
-      for (int n = 0; n < 4; ++n) MmaOp<T>::mma(acc[n], a, &b[n >> 1][(n & 1) * 2]);
+      for (int n = 0; n < C::MT; ++n) MmaOp<T>::mma(acc[n], a, &b[n >> 1][(n & 1) * 2]);
     }
-    float* P = p.partials + (size_t)g * 4096;    // [j][i], i contiguous
 #pragma unroll
-    for (int n = 0; n < 4; ++n) {
-      const int i = 16 * mt + (lane >> 2), j = 8 * (nt0 + n) + 2 * (lane & 3);
-      P[j * 64 + i] = acc[n][0];
-      P[(j + 1) * 64 + i] = acc[n][1];
-      P[j * 64 + i + 8] = acc[n][2];
-      P[(j + 1) * 64 + i + 8] = acc[n][3];
+    for (int n = 0; n < C::MT; ++n) {
+      const int i = 16 * mt + (lane >> 2), j = 64 * hh + 8 * (nt0 + n) + 2 * (lane & 3);
+      P[j * W + i] = acc[n][0];
+      P[(j + 1) * W + i] = acc[n][1];
+      P[j * W + i + 8] = acc[n][2];
+      P[(j + 1) * W + i + 8] = acc[n][3];
     }
+    __syncthreads();                               // before the next half overwrites `as`
   }
   sn_grid_barrier(p.counter, (unsigned)G);
 
   // ---- phase 2: entries [g EPC, (g+1) EPC) summed over the G partials in a fixed order:
   //      warp k adds partials k, k+8, ... in order, then warp 0 the 8 groups ----
   {
-    const int EPC = (4096 + G - 1) / G;
-    for (int e0 = g * EPC; e0 < min(4096, (g + 1) * EPC); e0 += 32) {
+    const int EPC = (C::E + G - 1) / G;
+    const int e_end = min(C::E, (g + 1) * EPC);
+    for (int e0 = g * EPC; e0 < e_end; e0 += 32) {
       const int e = e0 + lane;
-      const bool ok = e < min(4096, (g + 1) * EPC);
+      const bool ok = e < e_end;
       // all of this thread's partials in flight at once, then summed in order
       constexpr int PMAX = (LEAF_MAX_G + 7) / 8;
       float v[PMAX];
 #pragma unroll
-      for (int q = 0; q < PMAX; ++q) {
-        const int k = warp + 8 * q;
-        v[q] = (ok && k < G) ? __ldcg(p.partials + (size_t)k * 4096 + e) : 0.0f;
+      for (int qq = 0; qq < PMAX; ++qq) {
+        const int k = warp + 8 * qq;
+        v[qq] = (ok && k < G) ? __ldcg(p.partials + (size_t)k * C::E + e) : 0.0f;
       }
       float s0 = v[0];
 #pragma unroll
-      for (int q = 1; q < PMAX; ++q) s0 += v[q];
+      for (int qq = 1; qq < PMAX; ++qq) s0 += v[qq];
       red[warp * 33 + lane] = s0;
       __syncthreads();
       if (warp == 0 && ok) {
-        float v = red[lane];
+        float vv = red[lane];
 #pragma unroll
-        for (int k = 1; k < 8; ++k) v += red[k * 33 + lane];
-        const int i = e & 63, j = e >> 6;
-        if (i < p.w1 && j < p.w2) p.R12[i + (int64_t)j * p.ldr] = v;
-        static_cast<T*>(p.r12op)[e] = Elem<T>::store(v);    // [j][i]; zero outside w1 x w2
+        for (int k = 1; k < 8; ++k) vv += red[k * 33 + lane];
+        const int i = e % W, j = e / W;
+        if (i < p.w1 && j < p.w2) p.R12[i + (int64_t)j * p.ldr] = vv;
+        static_cast<T*>(p.r12op)[e] = Elem<T>::store(vv);   // [j][i]; zero outside w1 x w2
       }
       __syncthreads();
     }
   }
   sn_grid_barrier(p.counter, (unsigned)(2 * G));
 
-  // ---- phase 3: A2_s -= Q1_s R12; warp: m-tiles warp, warp + 8, ... (16 rows), all 8 n-tiles ----
-  {
-    for (int idx = threadIdx.x; idx < 64 * 8; idx += SN_THREADS) {      // 64 x 64 halves, 16 B each
-      const int j = idx >> 3, v = idx & 7;
-      *reinterpret_cast<uint4*>(rs + j * SN_RS + 8 * v) =
-          __ldcg(reinterpret_cast<const uint4*>(static_cast<const T*>(p.r12op) + j * 64 + 8 * v));
+  // ---- phase 3: A2_s -= Q1_s R12 per half; warp: m-tiles warp, warp + 8, ... (16 rows), all
+  //      8 n-tiles of the half, K = W ----
+  for (int hh = 0; hh < C::NH; ++hh) {
+    const int nc = max(0, min(64, p.w2 - 64 * hh));   // valid columns of this half
+    if (C::NH > 1)
+      sn_load_cols(as, S, static_cast<const T*>(A2), p.lda, r0, rows, 64 * hh, nc, 64, vec);
+    for (int idx = threadIdx.x; idx < 64 * (W / 8); idx += SN_THREADS) {   // 64 x W halves, 16 B each
+      const int j = idx / (W / 8), v = idx - j * (W / 8);
+      *reinterpret_cast<uint4*>(rs + j * C::RS + 8 * v) =
+          __ldcg(reinterpret_cast<const uint4*>(static_cast<const T*>(p.r12op) + (size_t)(64 * hh + j) * W + 8 * v));
     }
     __syncthreads();
-    const int q = lane >> 3, l8 = lane & 7;
-    // the next leaf's round 0 (leaf r0_mode 3): squares of the ROUNDED A2' values per column
-    // (and a_0.a_1), accumulated from the epilogue registers, reduced in a fixed order below
+    // the next leaf's round 0 (leaf r0_mode 3, W == 64): squares of the ROUNDED A2' values per
+    // column (and a_0.a_1), accumulated from the epilogue registers, reduced in a fixed order below
     float nrm[8][2] = {};
     float d01 = 0.f;
     for (int mt = warp; mt < RP16 / 16; mt += SN_THREADS / 32) {
       float acc[8][4] = {};
 #pragma unroll
-      for (int ks = 0; ks < 4; ++ks) {
+      for (int ks = 0; ks < W / 16; ++ks) {
         uint32_t a[4], b[4][4];
         // A[m = row][k = i] lives as qs[i][row]: transposed 8x8 loads
         ldsm_x4_t(a, qs + (16 * ks + (q >> 1) * 8 + l8) * S + 16 * mt + (q & 1) * 8);
 #pragma unroll
-        for (int h = 0; h < 4; ++h) ldsm_x4(b[h], rs + (8 * (2 * h + (q >> 1)) + l8) * SN_RS + 16 * ks + (q & 1) * 8);
+        for (int h = 0; h < 4; ++h) ldsm_x4(b[h], rs + (8 * (2 * h + (q >> 1)) + l8) * C::RS + 16 * ks + (q & 1) * 8);
 #pragma unroll
         for (int n = 0; n < 8; ++n) MmaOp<T>::mma(acc[n], a, &b[n >> 1][(n & 1) * 2]);
       }
@@ -220,14 +239,17 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
         c1[0] = v01;
         c0[8] = v10;
         c1[8] = v11;
-        const float f00 = Elem<T>::load(v00), f01 = Elem<T>::load(v01), f10 = Elem<T>::load(v10),
-                    f11 = Elem<T>::load(v11);
-        nrm[n][0] = fmaf(f00, f00, fmaf(f10, f10, nrm[n][0]));
-        nrm[n][1] = fmaf(f01, f01, fmaf(f11, f11, nrm[n][1]));
-        if (n == 0) d01 = fmaf(f00, f01, fmaf(f10, f11, d01));   // columns 0, 1 on lanes with tig 0
+        if (W == 64) {
+          const float f00 = Elem<T>::load(v00), f01 = Elem<T>::load(v01), f10 = Elem<T>::load(v10),
+                      f11 = Elem<T>::load(v11);
+          nrm[n][0] = fmaf(f00, f00, fmaf(f10, f10, nrm[n][0]));
+          nrm[n][1] = fmaf(f01, f01, fmaf(f11, f11, nrm[n][1]));
+          if (n == 0) d01 = fmaf(f00, f01, fmaf(f10, f11, d01));   // columns 0, 1 on lanes with tig 0
+        }
       }
     }
-    if (p.r0_partials != nullptr) {
+    const bool r0w = W == 64 && p.r0_partials != nullptr;
+    if (r0w) {
       // lanes sharing tig (= lane & 3) hold the same columns: xor tree over the row groups
 #pragma unroll
       for (int n = 0; n < 8; ++n)
@@ -252,7 +274,7 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
       }
     }
     __syncthreads();
-    if (p.r0_partials != nullptr) {
+    if (r0w) {
       const int L = p.w2 + (p.w2 > 1 ? 1 : 0);
       for (int k = threadIdx.x; k < L; k += SN_THREADS) {
         const int col = k < p.w2 ? k : 64;
@@ -262,26 +284,28 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
         p.r0_partials[(size_t)k * G + g] = v;
       }
     }
-    // ---- store A2' (columns < w2, rows < rows) ----
-    const int nv = p.vec_ok ? rows / 8 : 0;
-    for (int idx = threadIdx.x; idx < p.w2 * nv; idx += SN_THREADS) {
+    // ---- store A2' of this half (valid columns, rows < rows) ----
+    const int nv = vec ? rows / 8 : 0;
+    for (int idx = threadIdx.x; idx < nc * nv; idx += SN_THREADS) {
       const int c = idx / nv, v = idx - c * nv;
-      *reinterpret_cast<uint4*>(A2 + r0 + 8 * v + (int64_t)c * p.lda) = *reinterpret_cast<const uint4*>(as + c * S + 8 * v);
+      *reinterpret_cast<uint4*>(A2 + r0 + 8 * v + (int64_t)(64 * hh + c) * p.lda) =
+          *reinterpret_cast<const uint4*>(as + c * S + 8 * v);
     }
-    const int tail = rows - 8 * nv;
-    for (int idx = threadIdx.x; idx < p.w2 * tail; idx += SN_THREADS) {
-      const int c = idx / tail, r = 8 * nv + (idx - c * tail);
-      A2[r0 + r + (int64_t)c * p.lda] = as[c * S + r];
+    const int tl = rows - 8 * nv;
+    for (int idx = threadIdx.x; idx < nc * tl; idx += SN_THREADS) {
+      const int c = idx / tl, r = 8 * nv + (idx - c * tl);
+      A2[r0 + r + (int64_t)(64 * hh + c) * p.lda] = as[c * S + r];
     }
+    __syncthreads();                               // before the next half overwrites `as`, `rs`
   }
 }
 
-template <typename T>
-cudaError_t launch_small_node(const SmallNodeParams& p, int grid, cudaStream_t st) {
-  const size_t smem = small_node_smem(p.rows_per_cta);
+template <typename T, int W>
+static cudaError_t launch_small_node_w(const SmallNodeParams& p, int grid, cudaStream_t st) {
+  const size_t smem = small_node_smem(p.rows_per_cta, W);
   static size_t attr = 0;
   if (smem > attr) {
-    cudaError_t e = cudaFuncSetAttribute(small_node_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(small_node_kernel<T, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr = smem;
   }
@@ -297,7 +321,13 @@ cudaError_t launch_small_node(const SmallNodeParams& p, int grid, cudaStream_t s
   attr1[0].val.cooperative = 1;
   cfg.attrs = attr1;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, small_node_kernel<T>, p);
+  return cudaLaunchKernelEx(&cfg, small_node_kernel<T, W>, p);
+}
+
+template <typename T>
+cudaError_t launch_small_node(const SmallNodeParams& p, int grid, cudaStream_t st) {
+  if (p.w1 <= 64 && p.w2 <= 64) return launch_small_node_w<T, 64>(p, grid, st);
+  return launch_small_node_w<T, 128>(p, grid, st);
 }
 
 template cudaError_t launch_small_node<__half>(const SmallNodeParams&, int, cudaStream_t);

@@ -106,7 +106,7 @@ def test_tf32x3_usv_kappa_1e3(h):
 
 @pytest.mark.parametrize("prec", ["fp16", "bf16"])
 def test_fused_bottom_node_matches_separate_products(h, prec):
-    """The fused bottom-node kernel (small.cu, nodes with w1, w2 <= 64) against the separate
+    """The fused bottom-node kernel (small.cu, nodes with w1, w2 <= 64; 2: also <= 128) against the separate
     TN / NN products: both reach the oracle's R (Eq. 2), they differ only in
     the order of the fp32 sums; a ragged m exercises the partial last row slice."""
     m, n = 12345, 256
@@ -115,7 +115,7 @@ def test_fused_bottom_node_matches_separate_products(h, prec):
     X = gi.to_float64(A, st)
     ref = oracle.rgs(X, leaf=64)
     out = {}
-    for fuse in (0, 1):
+    for fuse in (0, 1, 2):
         h.set_option("fuse_small", fuse)
         rc, Q, R = run(h, A, st, prec, m, n)
         assert rc == 0
@@ -125,3 +125,4 @@ def test_fused_bottom_node_matches_separate_products(h, prec):
         assert be < 5e-3 and re < 5e-3, (fuse, be, re)
     h.set_option("fuse_small", 1)
     assert oracle.r_rel_error(out[1][1], out[0][1]) < 2e-3
+    assert oracle.r_rel_error(out[2][1], out[0][1]) < 2e-3
