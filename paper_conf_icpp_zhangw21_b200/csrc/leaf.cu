@@ -527,7 +527,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
 #pragma unroll
         for (int j = 0; j < NR; ++j)
-          if (vr[j]) ut[rr[j]] = q[j];   // Q goes to global memory at the end
+          if (vr[j]) ut[rr[j]] = q[j];   // (global Q: stored from registers in the exchange wait)
         s0 = s1 = s2 = s3 = s4 = 0.0f;
 #pragma unroll
         for (int j = 0; j < NR; ++j) {
@@ -547,7 +547,13 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           ra3[j] = a4v[j];
         }
       }
-      if (!more) break;
+      if (!more) {
+        // the last column: its rows of Q straight from registers
+#pragma unroll
+        for (int j = 0; j < NR; ++j)
+          if (vr[j]) P[r0 + rr[j] + (int64_t)t * p.ldp] = Elem<T>::store(rq1[j]);
+        break;
+      }
       // the critical reducer's lane 4c (c < 5) adds value c of round t+1: its fixed-point scale now
       const int n_crit = !h2 ? 1 : (!h3 ? 3 : 4);   // critical values of round t+1
       double crit_scale = 0.0;
@@ -596,6 +602,10 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           fx_add(t + 1, 4 + t, v);
         }
       }
+      // q_t of this thread's rows to global memory (rounded once), inside the exchange wait
+#pragma unroll
+      for (int j = 0; j < NR; ++j)
+        if (vr[j]) P[r0 + rr[j] + (int64_t)t * p.ldp] = Elem<T>::store(rq1[j]);
     }
   } else {
     // ---- BULK group: for each round t, after q_t is in smem:
@@ -778,22 +788,6 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   PRO_STAMP(4);
   __syncthreads();
   PRO_STAMP(5);
-  // ---- Q: the panel slice (now q_0..q_{w-1} in fp32) rounded once to the storage type ----
-  {
-    constexpr int V = Vec<T>::N;
-    const int nvec = p.vec_ok ? rows / V : 0;
-    for (int idx = threadIdx.x; idx < w * nvec; idx += LEAF_THREADS) {
-      const int j = idx / nvec, i = (idx - j * nvec) * V;
-#pragma unroll
-      for (int e = 0; e < V; e += 4)
-        store4<T>(P + r0 + i + e + (int64_t)j * p.ldp, *reinterpret_cast<const float4*>(sp + j * LD + i + e));
-    }
-    const int span = rows - nvec * V;
-    for (int idx = threadIdx.x; idx < w * span; idx += LEAF_THREADS) {
-      const int j = idx / span, i = nvec * V + (idx - j * span);
-      P[r0 + i + (int64_t)j * p.ldp] = Elem<T>::store(sp[j * LD + i]);
-    }
-  }
   PRO_STAMP(6);
   // every CTA ends with the same last-seen words; CTA 0 persists them for the next launch
   if (g == 0)
