@@ -37,6 +37,7 @@ struct GemmCfg {
 template <typename T, bool kNN, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                const __grid_constant__ CUtensorMap mapA2, const __grid_constant__ CUtensorMap mapB2,
                 const GemmParams p) {
   using C = GemmCfg<T, kNN, BN>;
   extern __shared__ uint8_t smem_raw[];
@@ -57,6 +58,10 @@ __global__ void __launch_bounds__(128, 1)
   if (warp == 0 && ptx::elect_one()) {
     ptx::tma_prefetch_desc(&mapA);
     ptx::tma_prefetch_desc(&mapB);
+    if (p.kb_seg > 0) {
+      ptx::tma_prefetch_desc(&mapA2);
+      ptx::tma_prefetch_desc(&mapB2);
+    }
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -79,16 +84,27 @@ __global__ void __launch_bounds__(128, 1)
         ptx::mbar_wait(&empty[s], ph ^ 1u);
         uint8_t* sA = smem + s * C::STAGE_BYTES;
         uint8_t* sB = sA + C::A_BYTES;
-        const int32_t k0 = (int32_t)((kb0 + it) * C::BK);
+        // TF32X3 segments (p.kb_seg > 0): k-blocks [0, kb_seg) = (A, B lo), then (A lo, B), then
+        // (A, B): the small cross terms accumulate first -- the tensor core's fp32 accumulation
+        // aligns to the largest addend, so adding them after the big term would drop their low bits
+        int64_t kbg = kb0 + it;
+        int seg = 2;
+        if (p.kb_seg > 0) {
+          seg = (int)(kbg / p.kb_seg);
+          kbg -= (int64_t)seg * p.kb_seg;
+        }
+        const CUtensorMap* ta = seg == 1 ? &mapA2 : &mapA;
+        const CUtensorMap* tb = seg == 0 ? &mapB2 : &mapB;
+        const int32_t k0 = (int32_t)(kbg * C::BK);
         ptx::mbar_arrive_expect_tx(&full[s], C::STAGE_BYTES);
         if constexpr (kNN) {
 #pragma unroll
           for (int mb = 0; mb < C::BM / C::EPB; ++mb)
-            ptx::tma_load_2d(sA + mb * C::BK * 128, &mapA, &full[s], (int32_t)(m0 + mb * C::EPB), k0);
+            ptx::tma_load_2d(sA + mb * C::BK * 128, ta, &full[s], (int32_t)(m0 + mb * C::EPB), k0);
         } else {
-          ptx::tma_load_2d(sA, &mapA, &full[s], k0, (int32_t)m0);
+          ptx::tma_load_2d(sA, ta, &full[s], k0, (int32_t)m0);
         }
-        ptx::tma_load_2d(sB, &mapB, &full[s], k0, (int32_t)n0);
+        ptx::tma_load_2d(sB, tb, &full[s], k0, (int32_t)n0);
       }
     }
   } else if (warp == 1) {
@@ -244,7 +260,8 @@ struct NNCfg {
 template <typename T, int BN>
 __global__ void __launch_bounds__(256, 1)
     nn_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
-              const __grid_constant__ CUtensorMap mapC, const NNParams p) {
+              const __grid_constant__ CUtensorMap mapC, const __grid_constant__ CUtensorMap mapA2,
+              const __grid_constant__ CUtensorMap mapB2, const NNParams p) {
   using C = NNCfg<T, BN>;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = ptx::smem_u32(smem_raw);
@@ -295,12 +312,20 @@ __global__ void __launch_bounds__(256, 1)
           const int s = it % C::STAGES;
           ptx::mbar_wait(&empty[s], ((uint32_t)(it / C::STAGES) & 1u) ^ 1u);
           uint8_t* sA = smem + s * C::STAGE_BYTES;
-          const int32_t k0 = kb * C::BK;
+          // TF32X3 segments (p.kb_seg > 0): (A, B lo), (A lo, B), then (A, B) -- small terms first
+          int seg = 2, kbl = kb;
+          if (p.kb_seg > 0) {
+            seg = kb / (int)p.kb_seg;
+            kbl = kb - seg * (int)p.kb_seg;
+          }
+          const CUtensorMap* ta = seg == 1 ? &mapA2 : &mapA;
+          const CUtensorMap* tb = seg == 0 ? &mapB2 : &mapB;
+          const int32_t k0 = kbl * C::BK;
           ptx::mbar_arrive_expect_tx(&full[s], C::STAGE_BYTES);
 #pragma unroll
           for (int mb = 0; mb < C::BM / C::EPB; ++mb)
-            ptx::tma_load_2d(sA + mb * C::BK * 128, &mapA, &full[s], m0 + mb * C::EPB, k0);
-          ptx::tma_load_2d(sA + C::A_BYTES, &mapB, &full[s], k0, n0);
+            ptx::tma_load_2d(sA + mb * C::BK * 128, ta, &full[s], m0 + mb * C::EPB, k0);
+          ptx::tma_load_2d(sA + C::A_BYTES, tb, &full[s], k0, n0);
         }
       }
     }
@@ -397,7 +422,8 @@ __global__ void __launch_bounds__(256, 1)
 
 template <typename T, int BN>
 static cudaError_t launch_nn_t(const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& mc,
-                               const NNParams& p, int grid, cudaStream_t st) {
+                               const CUtensorMap& ma2, const CUtensorMap& mb2, const NNParams& p, int grid,
+                               cudaStream_t st) {
   using C = NNCfg<T, BN>;
   static bool attr_set = false;
   if (!attr_set) {
@@ -405,36 +431,38 @@ static cudaError_t launch_nn_t(const CUtensorMap& ma, const CUtensorMap& mb, con
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  nn_kernel<T, BN><<<grid, 256, C::SMEM, st>>>(ma, mb, mc, p);
+  nn_kernel<T, BN><<<grid, 256, C::SMEM, st>>>(ma, mb, mc, ma2, mb2, p);
   return cudaGetLastError();
 }
 
 template <typename T>
 cudaError_t launch_nn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& mc,
-                      const NNParams& p, int grid, cudaStream_t st) {
+                      const NNParams& p, int grid, cudaStream_t st, const CUtensorMap* ma2, const CUtensorMap* mb2) {
+  const CUtensorMap& a2 = ma2 ? *ma2 : ma;
+  const CUtensorMap& b2 = mb2 ? *mb2 : mb;
   if constexpr (sizeof(T) == 4) {
-    if (bn >= 128) return launch_nn_t<T, 128>(ma, mb, mc, p, grid, st);
-    return launch_nn_t<T, 64>(ma, mb, mc, p, grid, st);
+    if (bn >= 128) return launch_nn_t<T, 128>(ma, mb, mc, a2, b2, p, grid, st);
+    return launch_nn_t<T, 64>(ma, mb, mc, a2, b2, p, grid, st);
   } else {
-    if (bn == 256) return launch_nn_t<T, 256>(ma, mb, mc, p, grid, st);
-    if (bn == 128) return launch_nn_t<T, 128>(ma, mb, mc, p, grid, st);
-    return launch_nn_t<T, 64>(ma, mb, mc, p, grid, st);
+    if (bn == 256) return launch_nn_t<T, 256>(ma, mb, mc, a2, b2, p, grid, st);
+    if (bn == 128) return launch_nn_t<T, 128>(ma, mb, mc, a2, b2, p, grid, st);
+    return launch_nn_t<T, 64>(ma, mb, mc, a2, b2, p, grid, st);
   }
 }
 
-template cudaError_t launch_nn<__half>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&,
-                                       const NNParams&, int, cudaStream_t);
-template cudaError_t launch_nn<__nv_bfloat16>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&,
-                                              const NNParams&, int, cudaStream_t);
-template cudaError_t launch_nn<float>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&,
-                                      const NNParams&, int, cudaStream_t);
+template cudaError_t launch_nn<__half>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&, const NNParams&,
+                                int, cudaStream_t, const CUtensorMap*, const CUtensorMap*);
+template cudaError_t launch_nn<__nv_bfloat16>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&, const NNParams&,
+                                int, cudaStream_t, const CUtensorMap*, const CUtensorMap*);
+template cudaError_t launch_nn<float>(int, const CUtensorMap&, const CUtensorMap&, const CUtensorMap&, const NNParams&,
+                                int, cudaStream_t, const CUtensorMap*, const CUtensorMap*);
 
 // ---------------------------------------------------------------------------------
 // host-side launch helpers
 // ---------------------------------------------------------------------------------
 template <typename T, bool kNN, int BN>
-static cudaError_t launch_gemm_t(const CUtensorMap& ma, const CUtensorMap& mb, const GemmParams& p,
-                                 int splits, cudaStream_t st) {
+static cudaError_t launch_gemm_t(const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& ma2,
+                                 const CUtensorMap& mb2, const GemmParams& p, int splits, cudaStream_t st) {
   using C = GemmCfg<T, kNN, BN>;
   static bool attr_set = false;
   if (!attr_set) {
@@ -444,21 +472,24 @@ static cudaError_t launch_gemm_t(const CUtensorMap& ma, const CUtensorMap& mb, c
     attr_set = true;
   }
   dim3 grid((unsigned)((p.M + C::BM - 1) / C::BM), (unsigned)((p.N + BN - 1) / BN), (unsigned)splits);
-  gemm_kernel<T, kNN, BN><<<grid, 128, C::SMEM, st>>>(ma, mb, p);
+  gemm_kernel<T, kNN, BN><<<grid, 128, C::SMEM, st>>>(ma, mb, ma2, mb2, p);
   return cudaGetLastError();
 }
 
 template <typename T>
 cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMap& mb,
-                        const GemmParams& p, int splits, cudaStream_t st) {
+                        const GemmParams& p, int splits, cudaStream_t st, const CUtensorMap* ma2,
+                        const CUtensorMap* mb2) {
+  const CUtensorMap& a2 = ma2 ? *ma2 : ma;
+  const CUtensorMap& b2 = mb2 ? *mb2 : mb;
   if (nn) {
-    if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, p, splits, st);
-    if (bn == 128) return launch_gemm_t<T, true, 128>(ma, mb, p, splits, st);
-    return launch_gemm_t<T, true, 64>(ma, mb, p, splits, st);
+    if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, a2, b2, p, splits, st);
+    if (bn == 128) return launch_gemm_t<T, true, 128>(ma, mb, a2, b2, p, splits, st);
+    return launch_gemm_t<T, true, 64>(ma, mb, a2, b2, p, splits, st);
   }
-  if (bn == 256) return launch_gemm_t<T, false, 256>(ma, mb, p, splits, st);
-  if (bn == 128) return launch_gemm_t<T, false, 128>(ma, mb, p, splits, st);
-  return launch_gemm_t<T, false, 64>(ma, mb, p, splits, st);
+  if (bn == 256) return launch_gemm_t<T, false, 256>(ma, mb, a2, b2, p, splits, st);
+  if (bn == 128) return launch_gemm_t<T, false, 128>(ma, mb, a2, b2, p, splits, st);
+  return launch_gemm_t<T, false, 64>(ma, mb, a2, b2, p, splits, st);
 }
 
 // Many splits: a CTA owns 32 consecutive output elements (coalesced 128-byte reads of every
@@ -583,12 +614,12 @@ cudaError_t launch_trmm_upper(const float* S, int64_t lds, float* R, int64_t ldr
   return cudaGetLastError();
 }
 
-template cudaError_t launch_gemm<__half>(bool, int, const CUtensorMap&, const CUtensorMap&,
-                                         const GemmParams&, int, cudaStream_t);
-template cudaError_t launch_gemm<__nv_bfloat16>(bool, int, const CUtensorMap&, const CUtensorMap&,
-                                                const GemmParams&, int, cudaStream_t);
-template cudaError_t launch_gemm<float>(bool, int, const CUtensorMap&, const CUtensorMap&,
-                                        const GemmParams&, int, cudaStream_t);
+template cudaError_t launch_gemm<__half>(bool, int, const CUtensorMap&, const CUtensorMap&, const GemmParams&, int,
+                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*);
+template cudaError_t launch_gemm<__nv_bfloat16>(bool, int, const CUtensorMap&, const CUtensorMap&, const GemmParams&, int,
+                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*);
+template cudaError_t launch_gemm<float>(bool, int, const CUtensorMap&, const CUtensorMap&, const GemmParams&, int,
+                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*);
 template cudaError_t launch_splitk_reduce<__half>(const float*, int64_t, int64_t, int, float*, int64_t,
                                                   int, __half*, int64_t, int64_t, int64_t, cudaStream_t);
 template cudaError_t launch_splitk_reduce<__nv_bfloat16>(const float*, int64_t, int64_t, int, float*,

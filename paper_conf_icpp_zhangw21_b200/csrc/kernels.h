@@ -41,16 +41,20 @@ struct GemmParams {
   // outer product (NN) epilogue: A2 <- A2 - result
   void* A2;
   int64_t lda2;
+  int64_t kb_seg;           // > 0: K blocks per operand segment (TF32X3: hi.lo, lo.hi, hi.hi)
 };
 
 struct NNParams {
   int tiles_m, tiles_n;     // 128-row x BN-column output tiles
-  int64_t kb_total;         // K blocks (K = w1)
+  int64_t kb_total;         // K blocks (K = w1; 3 x that for the TF32X3 segments)
+  int64_t kb_seg;           // > 0: K blocks per operand segment (TF32X3: hi.lo, lo.hi, hi.hi)
 };
 
+// TF32X3: ma2 / mb2 are the lo operands of A / B; segments (A, B lo), (A lo, B), (A, B)
 template <typename T>
 cudaError_t launch_nn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& mc,
-                      const NNParams& p, int grid, cudaStream_t st);
+                      const NNParams& p, int grid, cudaStream_t st, const CUtensorMap* ma2 = nullptr,
+                      const CUtensorMap* mb2 = nullptr);
 
 struct LeafParams {
   void* P;                  // panel m x w (ldp), overwritten by Q
@@ -110,7 +114,8 @@ int leaf_max_smem_rows(int w);
 
 template <typename T>
 cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMap& mb,
-                        const GemmParams& p, int splits, cudaStream_t st);
+                        const GemmParams& p, int splits, cudaStream_t st, const CUtensorMap* ma2 = nullptr,
+                        const CUtensorMap* mb2 = nullptr);
 template <typename T>
 cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t ldp, int splits,
                                  float* C, int64_t ldc, int accumulate, T* Cop, int64_t ldop,

@@ -119,7 +119,7 @@ static int op_inner_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
 template <typename T>
 static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
                          int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
-                         int accumulate, cudaStream_t st);
+                         int accumulate, cudaStream_t st, const void* Q1lo = nullptr, const void* A2lo = nullptr);
 
 // TF32X3 (3-pass split tf32): Q1^T A2 ~= Q1h^T A2h + Q1h^T A2l + Q1l^T A2h, hi = the stored
 // fp32 words read as tf32 (truncated by the MMA), lo = x - trunc_tf32(x); the three
@@ -137,9 +137,8 @@ static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const v
   RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(Q1), ldq, q_lo, m, m, w1, st));
   RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(A2), lda, a_lo, m, m, w2, st));
   c->stats.n_other_launches += 2;
-  int rc = op_inner_once<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, nullptr, 0, accumulate, st);
-  if (rc == 0) rc = op_inner_once<T>(c, prec, Q1, ldq, a_lo, m, m, w1, w2, R12, ldr, nullptr, 0, 1, st);
-  if (rc == 0) rc = op_inner_once<T>(c, prec, q_lo, m, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, 1, st);
+  // one GEMM over the three operand segments (K extended 3x): a single split-K reduction
+  int rc = op_inner_once<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st, q_lo, a_lo);
   c->arena.release(mark);
   return rc;
 }
@@ -147,20 +146,28 @@ static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const v
 template <typename T>
 static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
                          int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
-                         int accumulate, cudaStream_t st) {
+                         int accumulate, cudaStream_t st, const void* Q1lo, const void* A2lo) {
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
   const int bn = pick_bn(w2);
-  CUtensorMap ma, mb;
+  CUtensorMap ma, mb, ma2, mb2;
   std::string err;
   if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, BK, 128, &err) ||
       !encode_tmap_2d(&mb, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, BK, bn, &err))
     return fail(c, RGSQR_ERR_INVALID_ARG, "inner: " + err);
+  const bool x3 = Q1lo != nullptr && A2lo != nullptr;
+  if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)m * s, BK, 128, &err) ||
+             !encode_tmap_2d(&mb2, prec, A2lo, (uint64_t)m, (uint64_t)w2, (uint64_t)m * s, BK, bn, &err)))
+    return fail(c, RGSQR_ERR_INVALID_ARG, "inner (tf32x3): " + err);
   GemmParams p{};
   p.M = w1;
   p.N = w2;
   p.K = m;
   p.kb_total = (m + BK - 1) / BK;
+  if (x3) {   // TF32X3: k-blocks of (Q1, A2 lo), (Q1 lo, A2), (Q1, A2): small terms first
+    p.kb_seg = p.kb_total;
+    p.kb_total *= 3;
+  }
   const int64_t tiles = ((w1 + 127) / 128) * ((w2 + bn - 1) / bn);
   int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : (c->num_sms + tiles - 1) / tiles);
   splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.kb_total / 4));
@@ -180,7 +187,7 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
     p.P = P;
     p.ldp = w1;
     p.split_stride = w1 * w2;
-    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, (int)splits, st));
+    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, (int)splits, st, x3 ? &ma2 : nullptr, x3 ? &mb2 : nullptr));
     RGSQR_CUDA(c, launch_splitk_reduce<T>(P, w1 * w2, w1, (int)splits, R12, ldr, accumulate,
                                           static_cast<T*>(R12op), ldop, w1, w2, st));
     c->stats.n_other_launches++;
@@ -190,9 +197,9 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
     p.accumulate = accumulate;
     p.Cop = R12op;
     p.ldop = ldop;
-    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, 1, st));
+    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, 1, st, x3 ? &ma2 : nullptr, x3 ? &mb2 : nullptr));
   }
-  c->kend(1, st, kb, 2.0 * m * w1 * w2, (double)m * (w1 + w2) * s + 4.0 * w1 * w2);
+  c->kend(1, st, kb, (x3 ? 6.0 : 2.0) * m * w1 * w2, (double)m * (w1 + w2) * s * (x3 ? 2 : 1) + 4.0 * w1 * w2);
   c->arena.release(mark);
   c->stats.n_tn_launches++;
   return RGSQR_OK;
@@ -200,7 +207,8 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
 
 template <typename T>
 static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, int64_t ldr, void* A2,
-                      int64_t lda, int64_t m, int64_t w1, int64_t w2, cudaStream_t st) {
+                      int64_t lda, int64_t m, int64_t w1, int64_t w2, cudaStream_t st, const void* Q1lo = nullptr,
+                      const void* R12lo = nullptr) {
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
   const int EPB = 128 / s;
@@ -215,14 +223,24 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
       !encode_tmap_2d(&mb, prec, R12op, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err) ||
       !encode_tmap_2d(&mc, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, 128, 64, &err, 2))
     return fail(c, RGSQR_ERR_INVALID_ARG, "outer: " + err);
+  const bool x3 = Q1lo != nullptr && R12lo != nullptr;
+  CUtensorMap ma2, mb2;
+  if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)m * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
+             !encode_tmap_2d(&mb2, prec, R12lo, (uint64_t)w1, (uint64_t)w2, (uint64_t)w1 * s, BK, bn, &err)))
+    return fail(c, RGSQR_ERR_INVALID_ARG, "outer (tf32x3): " + err);
   NNParams p{};
   p.tiles_m = (int)((m + 127) / 128);
   p.tiles_n = (int)((w2 + bn - 1) / bn);
   p.kb_total = (w1 + BK - 1) / BK;
+  if (x3) {   // TF32X3: k-blocks of (Q1, R12 lo), (Q1 lo, R12), (Q1, R12) into one accumulator
+    p.kb_seg = p.kb_total;
+    p.kb_total *= 3;
+  }
   const int grid = (int)std::min<int64_t>((int64_t)p.tiles_m * p.tiles_n, c->num_sms);
   cudaEvent_t kb = c->kbegin(st);
-  RGSQR_CUDA(c, launch_nn<T>(bn, ma, mb, mc, p, grid, st));
-  c->kend(2, st, kb, 2.0 * m * w1 * w2, (double)m * w1 * s + (double)w1 * w2 * s + 2.0 * m * w2 * s);
+  RGSQR_CUDA(c, launch_nn<T>(bn, ma, mb, mc, p, grid, st, x3 ? &ma2 : nullptr, x3 ? &mb2 : nullptr));
+  c->kend(2, st, kb, (x3 ? 6.0 : 2.0) * m * w1 * w2,
+          (double)m * w1 * s * (x3 ? 2 : 1) + (double)w1 * w2 * s * (x3 ? 2 : 1) + 2.0 * m * w2 * s);
   c->stats.n_nn_launches++;
   return RGSQR_OK;
 }
@@ -275,7 +293,7 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
     case RGSQR_BF16: return op_outer_t<__nv_bfloat16>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
     case RGSQR_TF32: return op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
     case RGSQR_TF32X3: {
-      // A2 <- ((A2 - Q1h R12h) - Q1h R12l) - Q1l R12h  (three in-place tf32 updates)
+      // A2 <- A2 - (Q1h R12h + Q1h R12l + Q1l R12h): one NN pass over the three segments
       const size_t mark = c->arena.mark();
       float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
       float* r_lo = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
@@ -283,9 +301,7 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
       RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(Q1), ldq, q_lo, m, m, w1, st));
       RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(R12op), ldr, r_lo, w1, w1, w2, st));
       c->stats.n_other_launches += 2;
-      int rc = op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
-      if (rc == 0) rc = op_outer_t<float>(c, prec, Q1, ldq, r_lo, w1, A2, lda, m, w1, w2, st);
-      if (rc == 0) rc = op_outer_t<float>(c, prec, q_lo, m, R12op, ldr, A2, lda, m, w1, w2, st);
+      int rc = op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st, q_lo, r_lo);
       c->arena.release(mark);
       return rc;
     }
