@@ -180,7 +180,9 @@ struct Exec {
       }
     };
     hk.pending = [&](int64_t col_end) { return next < chunks.size() && chunks[next].first < col_end; };
-    hk.chunk = cw;
+    // deferred products are applied in pieces of >= 256 columns (a multiple of the upload
+    // chunk): narrower products (tall m makes cw small) would run at a fraction of the MMA rate
+    hk.chunk = cw * std::max<int64_t>(1, (256 + cw - 1) / cw);
     // Q columns and the matching R columns (full height: entries below the diagonal are zero
     // and stay zero) go out as soon as a chunk of leaves is final
     hk.leaf_done = [&](int64_t col_end) {
