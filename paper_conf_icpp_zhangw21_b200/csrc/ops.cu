@@ -169,7 +169,9 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
     p.kb_total *= 3;
   }
   const int64_t tiles = ((w1 + 127) / 128) * ((w2 + bn - 1) / bn);
-  int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : (c->num_sms + tiles - 1) / tiles);
+  // One wave: tiles x splits <= SMs (rounding up put 152 CTAs on 148 SMs at w1 = w2 = 512 and
+  // doubled the kernel time: 57 vs 37 us, profiles/r1_splitk_scan.txt).
+  int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : c->num_sms / tiles);
   splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.kb_total / 4));
   const size_t cap = std::min<size_t>((size_t)64 << 20, c->arena.free_bytes());
   while (splits > 1 && (size_t)splits * w1 * w2 * 4 + 256 > cap) --splits;
