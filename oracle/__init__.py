@@ -19,9 +19,12 @@ Contents (each function cites the PAPER.md passage it follows):
 Pins (tests/test_oracle_*.py, `-m "not gpu"`): Householder QR with sign
 normalisation, Cholesky of X^T X, closed forms for n <= 2, Hadamard (R = I),
 diagonal scaling (R = D), exact dyadic mixing (R = R0), invariants, and the
-paper's printed shape / byte formulas (tests/golden/).  Parity status per
-function is listed in DESIGN.md section 4 ("parity unpinned" where applicable:
-O5 -- an emulation whose only pin is agreement with O3 in the fp64 limit).
+paper's printed shape / byte formulas (tests/golden/).  O5 is pinned two-sided
+(tests/test_oracle_emulation_pins.py): the closed-form backward error of RN storage
+rounding, 0.4247 u sqrt(1 + L/2), and the independent emulation table of SURVEY.md:618-626.
+The executor-shaped byte splits of model.py are tied to PAPER.md:141/145 and to the
+reading-R11 count by exact identities (tests/test_model_pins.py).  Parity status per
+function: DESIGN.md section 4.
 """
 from .cgs import cgs, cgs2, rgs, rgs2, blocked_cgs, rgs_emulated, QRResult  # noqa: F401
 from .checks import (backward_error, orthogonality, r_rel_error, is_upper_triangular,  # noqa: F401

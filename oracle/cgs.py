@@ -228,6 +228,8 @@ def rgs_emulated(X: np.ndarray, mode: str, leaf: int = 32, reorth: bool = False)
     R = np.zeros((n, n), dtype=np.float64)
 
     def panel_cgs(P):
+        # Eq. (1) in fp32 on the stored panel; the q_j are used in fp32 inside the leaf
+        # and rounded to storage once, when the panel is written back (R20)
         P = P.astype(np.float32)
         Q = np.zeros_like(P)
         Rp = np.zeros((P.shape[1], P.shape[1]), dtype=np.float64)
@@ -236,10 +238,10 @@ def rgs_emulated(X: np.ndarray, mode: str, leaf: int = 32, reorth: bool = False)
             r = Q[:, :j].T @ a
             u = a - Q[:, :j] @ r
             rjj = np.float32(np.sqrt(np.float32(u @ u)))
-            Q[:, j] = _store(u / rjj, mode)
+            Q[:, j] = u / rjj
             Rp[:j, j] = r
             Rp[j, j] = rjj
-        return Q, Rp
+        return _store(Q, mode), Rp
 
     def leaf_cgs(c0, c1):
         Q, Rp = panel_cgs(Xs[:, c0:c1])

@@ -78,3 +78,33 @@ def test_recursive_moves_less_than_blocked():
         rh, rd = model.recursive_noreuse_words_closed(m, n, b)
         bh, bd = model.blocked_total_words(m, n, b)
         assert rh < bh and rd < bd
+
+
+def _r12_words(m, n, b):
+    """Sum of w1*w2 over the recursion's inner products (the R12 words the paper's outer
+    product re-reads: 'outer reads Q1 + R12 + A2')."""
+    return sum(w1 * w2 for w1, _, w2 in model.recursion_inner_products(m, n, b))
+
+
+@pytest.mark.parametrize("m,n,b", [(1000, 64, 8), (4096, 256, 32), (65536, 8192, 64), (7, 12, 3), (100, 96, 32)])
+def test_recursive_split_words_identity(m, n, b):
+    """The executor-shaped split (GPU byte-counter target, tests/test_gpu_factor_host.py)
+    differs from the paper-accounting count (reading R11 of PAPER.md:147-153, itself pinned
+    to its closed form above) by exactly the R12 re-reads of the outer product, which the
+    executor does not do because R12 stays resident."""
+    sp = model.recursive_noreuse_split_words(m, n, b)
+    h, d = model.recursive_noreuse_words_count(m, n, b)
+    assert sp["h2d_matrix"] + _r12_words(m, n, b) == h
+    assert sp["d2h_matrix"] + sp["d2h_r"] == d
+
+
+@pytest.mark.parametrize("m,n,b", [(1000, 64, 8), (4096, 256, 32), (65536, 8192, 1024), (131072, 131072, 8192)])
+def test_blocked_split_words_identity(m, n, b):
+    """blocked split + the R12 re-reads sum_i b(n - ib) + the last panel's 2mb (PAPER.md:139
+    counts mb + mb + mb for it although there is no trailing matrix) == PAPER.md:141 exactly;
+    its D2H == PAPER.md:145 exactly."""
+    k = n // b
+    sp = model.blocked_noreuse_split_words(m, n, b)
+    H, D = model.blocked_total_words(m, n, b)
+    assert sp["h2d_matrix"] + sum(b * (n - i * b) for i in range(1, k + 1)) + 2 * m * b == H
+    assert sp["d2h_matrix"] + sp["d2h_r"] == D
