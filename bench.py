@@ -5,17 +5,22 @@ and the fraction of the min(tensor-peak, host-link) roofline).
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2] [--impl ours|reference]
 
 Workload (N = 1): BASELINE.json configs[1] -- fp16 A 65536 x 8192 Gaussian with the device
-budget capped at 1 GiB (out-of-core).  Two measurements of the same metric:
+budget capped at 1 GiB (out-of-core).
 
-* ``value``: rgsqr_factor_device, A / Q / R already resident in HBM (the library's own
-  workspace still capped at the 1 GiB budget), timed with CUDA events on the library's
-  stream, barrier + synchronize on both sides, max over ranks.
-* ``e2e``: rgsqr_factor with the matrix in pinned HOST memory -- the paper's
-  out-of-core setting: every host->device tile upload and Q / R download is inside
-  the timed region (h2d/d2h bytes per step are the library's own counters).
+* ``value`` (the metric): rgsqr_factor through the C ABI with A, Q and R in pinned HOST
+  memory -- the paper's out-of-core setting: every host->device tile
+  upload and Q / R download is inside the timed region (h2d/d2h bytes per step are the
+  library's own counters).  CUDA events on the library's compute stream around K
+  host-synchronous calls, barrier + synchronize on both sides, max over ranks.
+* ``e2e``: the same measurement (the value path already starts from host buffers).
+* ``roofline``: the binding host-link term of the north-star roofline (bytes the schedule
+  moves over the 2D-tile link bandwidth the library's own copies reach, probed live), i.e.
+  max(T_tensor, T_link) / T_wall.
+* ``device_resident``: rgsqr_factor_device with A / Q / R already in HBM (workspace <= the
+  budget) and its per-kernel-class breakdown; ``kernel_roofline``: the dominant kernel.
 
-N > 1: each rank factors its own independent matrix (rows of the global Philox stream
-at offset rank*m): "replicas" until the row-sharded NCCL path lands.
+N > 1: rows of ONE global (N*65536) x 8192 matrix are sharded over the ranks (row-sharded
+NCCL path); the bench fails instead of silently falling back to replicas.
 ``--impl reference`` times the CPU oracle (fp64 recursive CGS, numpy/OpenBLAS) on a
 bounded sample of the same workload; it is a baseline, not the target.
 """
@@ -202,7 +207,7 @@ def main():
     ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--skip-e2e", action="store_true")
+    ap.add_argument("--skip-device", action="store_true", help="skip the HBM-resident secondary measurement")
     ap.add_argument("--no-ablation", action="store_true", help="skip the split-ratio e2e ablation")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
@@ -237,162 +242,156 @@ def main():
 
     m, n, prec, budget = wl["m"], wl["n"], wl["prec"], wl["budget"]
     st_name = STORAGE[prec]
+    s_bytes = 2 if st_name != "fp32" else 4
     peaks, peak_src = load_peaks()
     parallelism = "single"
     if world > 1:
-        # row-sharded: each rank holds m rows of ONE global (m*world) x n factorization
-        try:
-            from paper_conf_icpp_zhangw21_b200 import dist as rdist
-            h = rdist.create_handle(local, rank, world)
-            parallelism = f"rows sharded over {world} GPUs (R12 ncclAllReduce + in-kernel leaf exchange)"
-        except Exception as ex:  # pragma: no cover - fallback keeps the bench alive
-            print(f"[bench] distributed context unavailable ({ex}); running replicas", file=sys.stderr)
-            h = Handle(local)
-            parallelism = "replicas"
+        # row-sharded: each rank holds m rows of ONE global (m*world) x n factorization; no
+        # silent fallback to replicas (a failure to build the distributed context is fatal)
+        from paper_conf_icpp_zhangw21_b200 import dist as rdist
+        h = rdist.create_handle(local, rank, world)
+        parallelism = f"rows sharded over {world} GPUs (R12 ncclAllReduce + in-kernel leaf exchange)"
     else:
         h = Handle(local)
-    sharded = parallelism.startswith("rows")
-    # flops of the work all ranks do together (2 m_global n^2 if sharded, world x 2 m n^2 if replicas)
-    flops = 2.0 * m * n * n
+    flops = 2.0 * m * n * n          # per rank's rows; the job's flops are world x this
     stream = torch.cuda.current_stream()
     h.set_stream(stream.cuda_stream)
+    tensor_peak = peaks["bf16_tflops_sustained"] * (0.5 if prec == "tf32" else 1.0)
 
-    # ---- input (host, seeded; replicas use their own global rows) ----
+    # ---- input (host, seeded; rank r holds global rows [r m, (r+1) m)) ----
     A = gi.gaussian(m, n, seed=2, dtype=st_name, row0=rank * ((m + gi.ROW_BLOCK - 1) // gi.ROW_BLOCK) * gi.ROW_BLOCK)
-    tdt = {"fp16": torch.float16, "bf16": torch.bfloat16, "fp32": torch.float32}[st_name]
-    at_host = torch.from_numpy(np.ascontiguousarray(A.T).view(np.int16 if st_name == "bf16" else A.dtype))
-    if st_name == "bf16":
-        at_host = at_host.view(torch.bfloat16)
-    Ad = at_host.to("cuda")
-    Qd = torch.empty_like(Ad)
-    Rd = torch.empty((n, n), dtype=torch.float32, device="cuda")
-
     clocks = ClockSampler(local)
     clocks.start()
+    import ctypes
+    nbytes = A.nbytes
+    pa, pq, pr = h.host_alloc(nbytes), h.host_alloc(nbytes), h.host_alloc(n * n * 4)
+    np.ctypeslib.as_array((ctypes.c_uint8 * nbytes).from_address(pa))[:] = A.reshape(-1, order="F").view(np.uint8)
+    lda = m
 
-    # ---- value: device-resident factorization ----
+    # ---- host link: the executor's own 2D copies (in-core column chunks and ring row tiles) ----
+    link_geoms = {"columns": h.probe_link(pq, lda, m, min(n, (64 << 20) // (m * s_bytes)), s_bytes),
+                  "tile_16384": h.probe_link(pq, lda, min(m, 16384), min(n, 2048), s_bytes)}
+    link = {k: max(g[k] for g in link_geoms.values()) for k in ("h2d", "d2h", "duplex_total")}
+
+    # ---- value: host-resident (out-of-core) through rgsqr_factor, pinned host buffers ----
     for _ in range(args.warmup):
-        h.factor_device(Ad, m, m, n, Qd, Rd, precision=prec, budget=budget)
-    st_dev = h.stats()
-    launches_per_step = sum(st_dev[k] for k in ("n_leaf_launches", "n_tn_launches", "n_nn_launches",
-                                                "n_other_launches"))
+        h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
     barrier()
     torch.cuda.synchronize()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     clocks.active = True
-    ev0.record(stream)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
     for _ in range(args.steps):
-        h.factor_device(Ad, m, m, n, Qd, Rd, precision=prec, budget=budget)
-    ev1.record(stream)
+        h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
+    e1.record(stream)
     torch.cuda.synchronize()
     clocks.active = False
     barrier()
-    ms_dev = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
-    value = world * flops / (ms_dev / 1e3) / 1e12
-
-    # ---- per-kernel roofline (a profiled pass with CUDA events around every launch) ----
-    h.set_option("profile", 1)
-    h.factor_device(Ad, m, m, n, Qd, Rd, precision=prec, budget=budget)
-    prof = h.stats()
-    h.set_option("profile", 0)
-    kms = prof["kern_ms"]
-    dom = int(np.argmax(kms))
-    dom_name = KERNEL_CLASSES[dom]
-    tensor_peak = peaks["bf16_tflops_sustained"] * (0.5 if prec == "tf32" else 1.0)
-    if dom_name in ("inner", "outer"):
-        achieved = prof["kern_flops"][dom] / (kms[dom] / 1e3) / 1e12
-        roof = {"bound": "tensor", "achieved": achieved, "peak": tensor_peak, "unit": "TFLOP/s"}
-    else:
-        achieved = prof["kern_bytes"][dom] / (kms[dom] / 1e3) / 1e9
-        roof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s"}
-    roof["frac"] = roof["achieved"] / roof["peak"]
-    roof["kernel"] = dom_name
-    roof["peak_source"] = f"{peak_src} (MEASURED_PEAKS.json" + (", bf16 sustained x 0.5 for tf32)" if prec == "tf32" else ", bf16 sustained; fp16 dense rate = bf16)")
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tp):
-        t = json.load(open(tp)).get(args.workload, {}).get(dom_name)
-        if t is not None:
-            traffic = t
-    roof["traffic"] = traffic
-    roof["share_of_step"] = kms[dom] / sum(kms) if sum(kms) else None
-    if dom_name == "leaf":
-        # the leaf is bound by the latency of its dependent grid-wide reductions (one per
-        # column), not by a throughput: its per-column time against the measured floor of that
-        # exchange alone (profiles/r1_leaf_latency.md, scripts/crit_bench.cu variant V12)
-        us_col = kms[dom] * 1e3 / n
-        floor = 0.914
-        roof["latency"] = {"unit": "us per column", "achieved": us_col, "floor": floor, "frac": floor / us_col,
-                           "floor_source": "exchange-only round of 148 CTAs, measured on B200 (crit_bench V12)"}
-    kernels = {KERNEL_CLASSES[i]: {"ms": kms[i], "launches": prof["kern_launches"][i],
-                                   "tflops": (prof["kern_flops"][i] / (kms[i] / 1e3) / 1e12) if kms[i] else None,
-                                   "gbps": (prof["kern_bytes"][i] / (kms[i] / 1e3) / 1e9) if kms[i] else None}
-               for i in range(4)}
-
-    # ---- e2e: host-resident (out-of-core) through rgsqr_factor, pinned host buffers ----
-    e2e = None
-    if not args.skip_e2e:
-        link = link_bandwidth(torch)
-        nbytes = A.nbytes
-        pa, pq, pr = h.host_alloc(nbytes), h.host_alloc(nbytes), h.host_alloc(n * n * 4)
-        import ctypes
-        np.ctypeslib.as_array((ctypes.c_uint8 * nbytes).from_address(pa))[:] = A.reshape(-1, order="F").view(np.uint8)
-        lda = m
-        for _ in range(min(args.warmup, 2)):
+    ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+    so = h.stats()
+    value = world * flops / (ms / 1e3) / 1e12
+    launches_per_step = sum(so[k] for k in ("n_leaf_launches", "n_tn_launches", "n_nn_launches", "n_other_launches"))
+    t_tensor = flops / (tensor_peak * 1e12)
+    terms = {"h2d": (so["h2d_bytes"], link["h2d"]), "d2h": (so["d2h_bytes"], link["d2h"]),
+             "duplex": (so["h2d_bytes"] + so["d2h_bytes"], link["duplex_total"])}
+    bind = max(terms, key=lambda k: terms[k][0] / terms[k][1])
+    t_link = terms[bind][0] / (terms[bind][1] * 1e9)
+    roof = {"bound": "pcie" if t_link >= t_tensor else "tensor",
+            "achieved": terms[bind][0] / (ms / 1e3) / 1e9, "peak": terms[bind][1], "unit": "GB/s",
+            "frac": max(t_tensor, t_link) / (ms / 1e3),
+            "traffic": so["h2d_bytes"] + so["d2h_bytes"],
+            "binding_term": bind, "t_link_ms": 1e3 * t_link, "t_tensor_ms": 1e3 * t_tensor,
+            "peak_source": "host link probed live with the library's own cudaMemcpy2DAsync tile copies "
+                           "(rgsqr_probe_link; best of the in-core column-chunk and 16384-row ring-tile "
+                           "geometries); T_tensor against MEASURED_PEAKS.json bf16 sustained",
+            "link_gbps_measured": link_geoms,
+            "compulsory_bytes": {"h2d": m * n * s_bytes, "d2h": m * n * s_bytes + 2 * n * (n + 1)},
+            "frac_vs_compulsory": max(t_tensor, max(m * n * s_bytes / (link["h2d"] * 1e9),
+                                                    (m * n * s_bytes + 2 * n * (n + 1)) / (link["d2h"] * 1e9),
+                                                    (2 * m * n * s_bytes + 2 * n * (n + 1)) /
+                                                    (link["duplex_total"] * 1e9))) / (ms / 1e3)}
+    e2e = {"value": value, "unit": "TFLOPS", "ms_per_step": ms,
+           "h2d_bytes_per_step": so["h2d_bytes"], "d2h_bytes_per_step": so["d2h_bytes"],
+           "path": "rgsqr_factor (C ABI), A/Q/R in pinned host memory, budget %d MiB (same run as value)"
+                   % (budget // MiB),
+           "overlap_ratio": so["overlap_ratio"],
+           "busy_ms": {"h2d": so["h2d_busy_ms"], "d2h": so["d2h_busy_ms"], "compute": so["compute_busy_ms"]},
+           "ooc_nodes": so["n_ooc_nodes"], "arena_bytes": so["arena_bytes"],
+           "arena_high_water": so["arena_high_water"]}
+    # ablation (not the headline): OOC left child 62.5% of the columns instead of the paper's halves
+    if world == 1 and not args.no_ablation:
+        h.set_option("split_pct", 62)
+        h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
+        torch.cuda.synchronize()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        for _ in range(2):
             h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
+        a1.record(stream)
+        torch.cuda.synchronize()
+        ms_ab = a0.elapsed_time(a1) / 2
+        e2e["ablation_split_pct_62"] = {"value": flops / (ms_ab / 1e3) / 1e12, "ms_per_step": ms_ab}
+        h.set_option("split_pct", 50)
+
+    # ---- secondary: device-resident factorization (A / Q / R in HBM) and its kernels ----
+    dev = None
+    kroof = None
+    if not args.skip_device:
+        tdt = {"fp16": torch.float16, "bf16": torch.bfloat16, "fp32": torch.float32}[st_name]
+        at_host = torch.from_numpy(np.ascontiguousarray(A.T).view(np.int16 if st_name == "bf16" else A.dtype))
+        if st_name == "bf16":
+            at_host = at_host.view(torch.bfloat16)
+        Ad = at_host.to("cuda")
+        Qd = torch.empty_like(Ad)
+        Rd = torch.empty((n, n), dtype=torch.float32, device="cuda")
+        for _ in range(args.warmup):
+            h.factor_device(Ad, m, m, n, Qd, Rd, precision=prec, budget=budget)
         barrier()
         torch.cuda.synchronize()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         clocks.active = True
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
+        ev0.record(stream)
         for _ in range(args.steps):
-            h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
-        e1.record(stream)
+            h.factor_device(Ad, m, m, n, Qd, Rd, precision=prec, budget=budget)
+        ev1.record(stream)
         torch.cuda.synchronize()
         clocks.active = False
         barrier()
-        ms_e2e = max_over_ranks(e0.elapsed_time(e1) / args.steps)
-        so = h.stats()
-        t_tensor = flops / (tensor_peak * 1e12)
-        t_link = max(so["h2d_bytes"] / (link["h2d"] * 1e9), so["d2h_bytes"] / (link["d2h"] * 1e9),
-                     (so["h2d_bytes"] + so["d2h_bytes"]) / (link["duplex_total"] * 1e9))
-        t_min = m * n * (2 if st_name != "fp32" else 4)
-        e2e = {"value": world * flops / (ms_e2e / 1e3) / 1e12, "unit": "TFLOPS", "ms_per_step": ms_e2e,
-               "h2d_bytes_per_step": so["h2d_bytes"], "d2h_bytes_per_step": so["d2h_bytes"],
-               "path": "rgsqr_factor (C ABI), A/Q/R in pinned host memory, budget %d MiB" % (budget // MiB),
-               "roofline_frac": max(t_tensor, t_link) / (ms_e2e / 1e3),
-               "roofline_bound": "pcie" if t_link > t_tensor else "tensor",
-               "t_link_ms": 1e3 * t_link, "t_tensor_ms": 1e3 * t_tensor,
-               "link_gbps_measured": link, "compulsory_bytes": {"h2d": t_min, "d2h": t_min + n * n * 4},
-               "overlap_ratio": so["overlap_ratio"], "busy_ms": {"h2d": so["h2d_busy_ms"], "d2h": so["d2h_busy_ms"],
-                                                               "compute": so["compute_busy_ms"]},
-               "ooc_nodes": so["n_ooc_nodes"], "arena_bytes": so["arena_bytes"],
-               "gpu_launches": args.steps * sum(so[k] for k in ("n_leaf_launches", "n_tn_launches",
-                                                                  "n_nn_launches", "n_other_launches"))}
-        # ablation (not the headline): OOC left child 62.5% of the columns instead of the paper's
-        # halves -- the right child's in-core factorization is the one phase that cannot overlap
-        # host transfers (RGSQR_OPT_SPLIT_PCT)
-        if world == 1 and not args.no_ablation:
-            h.set_option("split_pct", 62)
-            h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
-            torch.cuda.synchronize()
-            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a0.record(stream)
-            for _ in range(2):
-                h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
-            a1.record(stream)
-            torch.cuda.synchronize()
-            ms_ab = a0.elapsed_time(a1) / 2
-            sa = h.stats()
-            tl_ab = max(sa["h2d_bytes"] / (link["h2d"] * 1e9), sa["d2h_bytes"] / (link["d2h"] * 1e9),
-                        (sa["h2d_bytes"] + sa["d2h_bytes"]) / (link["duplex_total"] * 1e9))
-            e2e["ablation_split_pct_62"] = {"value": flops / (ms_ab / 1e3) / 1e12, "ms_per_step": ms_ab,
-                                            "h2d_bytes_per_step": sa["h2d_bytes"],
-                                            "d2h_bytes_per_step": sa["d2h_bytes"],
-                                            "roofline_frac": max(t_tensor, tl_ab) / (ms_ab / 1e3)}
-            h.set_option("split_pct", 50)
-        for p in (pa, pq, pr):
-            h.host_free(p)
+        ms_dev = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
+        h.set_option("profile", 1)
+        h.factor_device(Ad, m, m, n, Qd, Rd, precision=prec, budget=budget)
+        prof = h.stats()
+        h.set_option("profile", 0)
+        kms = prof["kern_ms"]
+        dom = int(np.argmax(kms))
+        dom_name = KERNEL_CLASSES[dom]
+        if dom_name in ("inner", "outer"):
+            achieved = prof["kern_flops"][dom] / (kms[dom] / 1e3) / 1e12
+            kroof = {"bound": "tensor", "achieved": achieved, "peak": tensor_peak, "unit": "TFLOP/s"}
+        else:
+            achieved = prof["kern_bytes"][dom] / (kms[dom] / 1e3) / 1e9
+            kroof = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s"}
+        kroof["frac"] = kroof["achieved"] / kroof["peak"]
+        kroof["kernel"] = dom_name
+        kroof["peak_source"] = f"{peak_src} (MEASURED_PEAKS.json)"
+        tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+        kroof["traffic"] = json.load(open(tp)).get(args.workload, {}).get(dom_name) if os.path.exists(tp) else None
+        kroof["share_of_step"] = kms[dom] / sum(kms) if sum(kms) else None
+        if dom_name == "leaf":
+            us_col = kms[dom] * 1e3 / n
+            floor = 0.914
+            kroof["latency"] = {"unit": "us per column", "achieved": us_col, "floor": floor, "frac": floor / us_col,
+                                "floor_source": "exchange-only round of 148 CTAs, measured on B200 (crit_bench V12)"}
+        kernels = {KERNEL_CLASSES[i]: {"ms": kms[i], "launches": prof["kern_launches"][i],
+                                       "tflops": (prof["kern_flops"][i] / (kms[i] / 1e3) / 1e12) if kms[i] else None,
+                                       "gbps": (prof["kern_bytes"][i] / (kms[i] / 1e3) / 1e9) if kms[i] else None}
+                   for i in range(4)}
+        dev = {"value": world * flops / (ms_dev / 1e3) / 1e12, "unit": "TFLOPS", "ms_per_step": ms_dev,
+               "path": "rgsqr_factor_device: A/Q/R resident in HBM, library workspace <= budget",
+               "kernels": kernels, "kernel_timing": "per-kernel CUDA events in one profiled step after the timed region"}
+        del Ad, Qd, Rd
+    for p_ in (pa, pq, pr):
+        h.host_free(p_)
     clocks.stop()
 
     # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1) ----
@@ -402,21 +401,24 @@ def main():
         v, dt = cpu_oracle_sample(A, st_name, cols)
         cpu = {"value": v, "unit": "TFLOPS", "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
                "sample": f"oracle O3 (fp64 recursive CGS, numpy/OpenBLAS) on {m}x{cols} (first {cols} columns "
-                         f"of the same input), {dt:.1f} s"}
+                         f"of the same input), {dt:.1f} s; extrapolated to the full {m}x{n} at this rate: "
+                         f"{2.0 * m * n * n / (v * 1e12):.0f} s (the rate grows with n, so this over-states "
+                         f"the CPU time)"}
+        full = os.path.join(ROOT, "profiles", "r2_cpu_oracle_c2.json")
+        if os.path.exists(full) and args.workload == "c2":
+            cpu["full_c2_measured"] = json.load(open(full))
 
     if rank == 0:
         line = {"metric": METRIC,
                 "value": value, "unit": "TFLOPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-                "ms_per_step": ms_dev, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": DTYPE_NAME[prec], "data": "synthetic",
                 "config": {"workload": wl["desc"], "m": m, "n": n, "precision": prec, "device_budget_bytes": budget,
-                           "value_path": "rgsqr_factor_device: A/Q/R resident in HBM, library workspace <= budget",
+                           "value_path": "rgsqr_factor: A/Q/R in pinned host memory, out-of-core under the budget",
                            "l2": "inputs (>= 1 GiB) larger than L2 (126 MB); no flush needed",
-                           "parallelism": parallelism,
-                           "m_global": m * world if sharded else m},
-                "roofline": roof, "kernels": kernels, "e2e": e2e, "cpu_baseline": cpu,
-                "gpu_launches": args.steps * launches_per_step, "clocks": clocks.summary(),
-                "kernel_timing": "per-kernel CUDA events in one profiled step after the timed region"}
+                           "parallelism": parallelism, "m_global": m * world},
+                "roofline": roof, "e2e": e2e, "device_resident": dev, "kernel_roofline": kroof,
+                "cpu_baseline": cpu, "gpu_launches": args.steps * launches_per_step, "clocks": clocks.summary()}
         print(json.dumps(line), flush=True)
     h.close()
     if world > 1:

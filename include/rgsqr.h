@@ -94,6 +94,10 @@ enum rgsqr_option {
                                    (rounded to 64).  50 = "divide evenly its columns into two halves"
                                    (PAPER.md:115), the default; other values are a scheduling ablation
                                    (same factorization in exact arithmetic).  In-core nodes always halve */
+  ,RGSQR_OPT_X3_CHAIN = 16      /* TF32X3 inner products: at most this many k-blocks (32 rows each, per
+                                   operand segment) accumulate in one tensor-core fp32 chain; longer K is
+                                   split and the partials summed in fixed order on the CUDA cores
+                                   (R25).  0 = the automatic one-wave split */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */
@@ -182,6 +186,13 @@ int rgsqr_host_free(rgsqr_handle h, void* p);
 int rgsqr_set_option(rgsqr_handle h, int key, int64_t value);
 int rgsqr_get_option(rgsqr_handle h, int key, int64_t* value);
 int rgsqr_get_stats(rgsqr_handle h, rgsqr_stats* out);
+/* Host-link probe with the executor's own copy calls (cudaMemcpy2DAsync on the library's H2D and
+ * D2H streams): `reps` copies of a rows x cols tile of elem_bytes-sized elements whose columns are
+ * ld elements apart in the caller's pinned host buffer `host` (>= ld * cols elements), H2D alone,
+ * D2H alone, then both directions concurrently.  gbps[0..2] = H2D, D2H and duplex-total GB/s
+ * (10^9 B/s), CUDA-event timed.  The device tile is a temporary allocation outside any budget. */
+int rgsqr_probe_link(rgsqr_handle h, void* host, int64_t ld, int64_t rows, int64_t cols, int elem_bytes,
+                     int reps, double* gbps);
 int rgsqr_version(void);                                        /* 100 * major + minor */
 const char* rgsqr_status_string(int status);
 const char* rgsqr_last_error(rgsqr_handle h);

@@ -96,7 +96,10 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   c->stats.arena_bytes = (int64_t)c->arena.size;
   c->stats.arena_high_water = (int64_t)c->arena.high;
   c->stats.flops = (int64_t)(2.0 * m * (double)n * n);
-  if (brk == -2) return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
+  if (brk == -2) {
+    c->broken = true;
+    return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
+  }
   c->stats.first_breakdown_col = brk == 0x7f7f7f7f || brk == INT_MAX ? -1 : brk;
   c->collect_kernel_stats();
   return c->stats.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;
@@ -235,11 +238,25 @@ int rgsqr_get_unique_id(unsigned char id[128]) {
   return g_nccl.getUniqueId(id) == 0 ? RGSQR_OK : RGSQR_ERR_NCCL;
 }
 
+static int create_dist_impl(Ctx* c, int rank, int nranks, const unsigned char id[128]);
+
 int rgsqr_create_dist(rgsqr_handle* h, int device, int rank, int nranks, const unsigned char id[128]) {
+  if (!h) return RGSQR_ERR_INVALID_ARG;
+  *h = nullptr;
   if (nranks < 1 || rank < 0 || rank >= nranks || !id) return RGSQR_ERR_INVALID_ARG;
+  if (nranks > 64) return RGSQR_ERR_UNSUPPORTED;
   int rc = create_impl(h, device);
   if (rc < 0) return rc;
-  Ctx* c = C(*h);
+  rc = create_dist_impl(C(*h), rank, nranks, id);
+  if (rc < 0) {
+    // release the streams, device buffers, IPC mappings and communicator created so far
+    rgsqr_destroy(*h);
+    *h = nullptr;
+  }
+  return rc;
+}
+
+static int create_dist_impl(Ctx* c, int rank, int nranks, const unsigned char id[128]) {
   c->rank = rank;
   c->nranks = nranks;
   // A distributed context always has an NCCL communicator (also for nranks == 1, which runs
@@ -247,8 +264,10 @@ int rgsqr_create_dist(rgsqr_handle* h, int device, int rank, int nranks, const u
   if (!g_nccl.load()) return fail(c, RGSQR_ERR_NCCL, "libnccl.so.2 not loadable");
   NcclApi::UniqueId uid;
   std::memcpy(uid.internal, id, sizeof(uid.internal));
-  if (g_nccl.commInitRank(&c->nccl_comm, nranks, uid, rank) != 0)
+  if (g_nccl.commInitRank(&c->nccl_comm, nranks, uid, rank) != 0) {
+    c->nccl_comm = nullptr;
     return fail(c, RGSQR_ERR_NCCL, "ncclCommInitRank failed");
+  }
   // Map every rank's leaf exchange words (CUDA IPC handles exchanged with ncclAllGather),
   // so the leaf kernel can red.add its partials into all GPUs' words over NVLink.
   std::vector<unsigned long long*> peers(nranks, nullptr);
@@ -260,8 +279,10 @@ int rgsqr_create_dist(rgsqr_handle* h, int device, int rank, int nranks, const u
     const size_t hs = sizeof(cudaIpcMemHandle_t);
     if (cudaMalloc(&dbuf, hs * (nranks + 1)) != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, "cudaMalloc");
     cudaMemcpy(dbuf + hs * nranks, &mine, hs, cudaMemcpyHostToDevice);
-    if (g_nccl.allGather(dbuf + hs * nranks, dbuf, hs, /*ncclChar*/ 0, c->nccl_comm, c->st_own) != 0)
+    if (g_nccl.allGather(dbuf + hs * nranks, dbuf, hs, /*ncclChar*/ 0, c->nccl_comm, c->st_own) != 0) {
+      cudaFree(dbuf);
       return fail(c, RGSQR_ERR_NCCL, "ncclAllGather of IPC handles");
+    }
     std::vector<cudaIpcMemHandle_t> all(nranks);
     cudaMemcpyAsync(all.data(), dbuf, hs * nranks, cudaMemcpyDeviceToHost, c->st_own);
     cudaStreamSynchronize(c->st_own);
@@ -275,7 +296,6 @@ int rgsqr_create_dist(rgsqr_handle* h, int device, int rank, int nranks, const u
       c->ipc_opened.push_back(ptr);
     }
   }
-  if (nranks > 64) return fail(c, RGSQR_ERR_UNSUPPORTED, "more than 64 ranks");
   cudaMemcpy(c->d_peers, peers.data(), sizeof(void*) * nranks, cudaMemcpyHostToDevice);
   // every rank has zeroed its words (create_impl) before anyone may add into them
   float one = 0.f;
@@ -316,6 +336,7 @@ int rgsqr_factor(rgsqr_handle h, const void* A_host, int64_t lda, int64_t m, int
   Ctx* c = C(h);
   if (!c) return RGSQR_ERR_INVALID_ARG;
   cudaSetDevice(c->device);
+  if (c->broken) return fail(c, RGSQR_ERR_CUDA, "handle unusable after a leaf exchange timeout: destroy it");
   return factor_host(c, A_host, lda, m, n, Q_out, R_out, precision, device_mem_budget);
 }
 
@@ -324,6 +345,7 @@ int rgsqr_factor_device(rgsqr_handle h, const void* A_dev, int64_t lda, int64_t 
   Ctx* c = C(h);
   if (!c) return RGSQR_ERR_INVALID_ARG;
   cudaSetDevice(c->device);
+  if (c->broken) return fail(c, RGSQR_ERR_CUDA, "handle unusable after a leaf exchange timeout: destroy it");
   return factor_device(c, A_dev, lda, m, n, Q_dev, R_dev, precision, device_mem_budget);
 }
 
@@ -332,6 +354,7 @@ int rgsqr_op_leaf(rgsqr_handle h, void* P, int64_t ldp, int64_t m, int64_t w, fl
   Ctx* c = C(h);
   if (!c || !P || !R11 || m < 1 || w < 1 || ldp < m || ldr < w) return RGSQR_ERR_INVALID_ARG;
   cudaSetDevice(c->device);
+  if (c->broken) return fail(c, RGSQR_ERR_CUDA, "handle unusable after a leaf exchange timeout: destroy it");
   cudaStream_t st = c->compute();
   RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), st));
   int rc = op_leaf(c, precision, P, ldp, m, w, R11, ldr, 0, st);
@@ -339,7 +362,10 @@ int rgsqr_op_leaf(rgsqr_handle h, void* P, int64_t ldp, int64_t m, int64_t w, fl
   int brk = INT_MAX;
   RGSQR_CUDA(c, cudaMemcpyAsync(&brk, c->d_breakdown, sizeof(int), cudaMemcpyDeviceToHost, st));
   RGSQR_CUDA(c, cudaStreamSynchronize(st));
-  if (brk == -2) return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
+  if (brk == -2) {
+    c->broken = true;
+    return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
+  }
   if (breakdown) *breakdown = (brk == 0x7f7f7f7f) ? -1 : brk;
   return brk == 0x7f7f7f7f ? RGSQR_OK : RGSQR_WARN_RANK_DEFICIENT;
 }
@@ -414,6 +440,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_PREFETCH: return &o.prefetch;
     case RGSQR_OPT_FUSE_SMALL: return &o.fuse_small;
     case RGSQR_OPT_SPLIT_PCT: return &o.split_pct;
+    case RGSQR_OPT_X3_CHAIN: return &o.x3_chain;
   }
   return nullptr;
 }
@@ -450,6 +477,60 @@ int rgsqr_get_stats(rgsqr_handle h, rgsqr_stats* out) {
   Ctx* c = C(h);
   if (!c || !out) return RGSQR_ERR_INVALID_ARG;
   *out = c->stats;
+  return RGSQR_OK;
+}
+
+int rgsqr_probe_link(rgsqr_handle h, void* host, int64_t ld, int64_t rows, int64_t cols, int elem_bytes, int reps,
+                     double* gbps) {
+  Ctx* c = C(h);
+  if (!c || !host || !gbps || rows < 1 || cols < 1 || ld < rows || elem_bytes < 1 || reps < 1)
+    return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  const size_t pitch = (size_t)ld * elem_bytes, wb = (size_t)rows * elem_bytes;
+  const size_t tile = wb * cols;
+  char* d = nullptr;
+  RGSQR_CUDA(c, cudaMalloc(&d, 2 * tile));
+  cudaEvent_t e[6];
+  for (auto& x : e) cudaEventCreate(&x);
+  auto up = [&](int r) { return cudaMemcpy2DAsync(d, wb, host, pitch, wb, cols, cudaMemcpyHostToDevice, c->st_h2d); };
+  auto down = [&](int r) { return cudaMemcpy2DAsync(host, pitch, d + tile, wb, wb, cols, cudaMemcpyDeviceToHost, c->st_d2h); };
+  cudaError_t err = cudaSuccess;
+  // warm-up, then H2D alone, D2H alone, duplex (both streams, joined)
+  err = up(0) == cudaSuccess && down(0) == cudaSuccess ? cudaSuccess : cudaErrorUnknown;
+  cudaStreamSynchronize(c->st_h2d);
+  cudaStreamSynchronize(c->st_d2h);
+  cudaEventRecord(e[0], c->st_h2d);
+  for (int r = 0; r < reps; ++r) up(r);
+  cudaEventRecord(e[1], c->st_h2d);
+  cudaStreamSynchronize(c->st_h2d);
+  cudaEventRecord(e[2], c->st_d2h);
+  for (int r = 0; r < reps; ++r) down(r);
+  cudaEventRecord(e[3], c->st_d2h);
+  cudaStreamSynchronize(c->st_d2h);
+  cudaEventRecord(e[4], c->st_h2d);
+  cudaStreamWaitEvent(c->st_d2h, e[4], 0);
+  for (int r = 0; r < reps; ++r) {
+    up(r);
+    down(r);
+  }
+  cudaEvent_t j;
+  cudaEventCreate(&j);
+  cudaEventRecord(j, c->st_d2h);
+  cudaStreamWaitEvent(c->st_h2d, j, 0);
+  cudaEventRecord(e[5], c->st_h2d);
+  cudaError_t e2 = cudaStreamSynchronize(c->st_h2d);
+  float ms[3] = {0, 0, 0};
+  cudaEventElapsedTime(&ms[0], e[0], e[1]);
+  cudaEventElapsedTime(&ms[1], e[2], e[3]);
+  cudaEventElapsedTime(&ms[2], e[4], e[5]);
+  for (auto& x : e) cudaEventDestroy(x);
+  cudaEventDestroy(j);
+  cudaFree(d);
+  if (err != cudaSuccess || e2 != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, "probe_link copies failed");
+  const double bytes = (double)tile * reps;
+  gbps[0] = bytes / (ms[0] * 1e-3) / 1e9;
+  gbps[1] = bytes / (ms[1] * 1e-3) / 1e9;
+  gbps[2] = 2.0 * bytes / (ms[2] * 1e-3) / 1e9;
   return RGSQR_OK;
 }
 

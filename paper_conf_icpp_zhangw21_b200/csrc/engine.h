@@ -30,6 +30,7 @@ struct Options {
   int64_t prefetch = 1;      // OOC: upload the first ring tiles during the left child (RGSQR_OPT_PREFETCH)
   int64_t fuse_small = 1;    // fused kernel for nodes with w1, w2 <= 64 (RGSQR_OPT_FUSE_SMALL)
   int64_t split_pct = 50;    // OOC split: left child width in % (RGSQR_OPT_SPLIT_PCT; 50 = halves, the paper)
+  int64_t x3_chain = 0;      // TF32X3: max k-blocks per split-K chain (RGSQR_OPT_X3_CHAIN; 0 = one-wave rule)
 };
 
 struct KernSeg {
@@ -94,6 +95,9 @@ struct Ctx {
   std::vector<cudaEvent_t> event_pool;
   size_t event_next = 0;
   bool timing = false;
+  // a leaf exchange timed out (a rank did not arrive): late contributions may still land in the
+  // never-reset exchange words, so the handle refuses further factorizations (rgsqr_destroy it)
+  bool broken = false;
 
   cudaStream_t compute() const { return st_user ? st_user : st_own; }
   cudaEvent_t ev();

@@ -13,6 +13,8 @@
 // in NN the Q1 operand is MN-major (its rows are the output rows) -- legal for
 // f16/bf16/tf32 UMMA.  The subtraction A2 - Q1 R12 is fused into the epilogue, so A2'
 // is written exactly once, rounded RN-even to the storage type (R5).
+#include <algorithm>
+
 #include "dtype.cuh"
 #include "kernels.h"
 #include "ptx.cuh"
@@ -561,23 +563,52 @@ cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t l
 
 int gemm_block_k(int elem_bytes) { return 128 / elem_bytes; }
 
-// TF32X3 operand split: lo = x - trunc_tf32(x) (exact in fp32).  The hi part is the
-// original array: tcgen05 kind::tf32 reads only the top 19 bits of each fp32 word.
-__global__ void tf32_lo_kernel(const float* __restrict__ src, int64_t lds, float* __restrict__ dst, int64_t ldd,
-                               int64_t M, int64_t N) {
-  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= M * N) return;
-  const int64_t i = idx % M, j = idx / M;
-  const float x = src[i + j * lds];
-  const float hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
-  dst[i + j * ldd] = x - hi;
+// TF32X3 operand split (R25): hi = RN_tf32(x), lo = RN_tf32(x - hi),
+// both written as fp32 words whose low 13 mantissa bits are zero, so tcgen05 kind::tf32 (which
+// reads the top 19 bits) consumes them exactly.  |x - hi - lo| <= 2^-22 |x| and the dropped
+// lo*lo term is <= 2^-22 |x||y| (truncated parts would give 2^-20 for both).  x - hi is exact in
+// fp32.  RN-even by integer rounding of the bit pattern (finite inputs).
+__device__ __forceinline__ float rn_tf32(float x) {
+  const uint32_t u = __float_as_uint(x);
+  return __uint_as_float((u + 0xFFFu + ((u >> 13) & 1u)) & 0xFFFFE000u);
 }
 
-cudaError_t launch_tf32_lo(const float* src, int64_t lds, float* dst, int64_t ldd, int64_t M, int64_t N,
-                           cudaStream_t st) {
-  const int64_t total = M * N;
-  if (total == 0) return cudaSuccess;
-  tf32_lo_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(src, lds, dst, ldd, M, N);
+__global__ void tf32_split_kernel(const float* __restrict__ src, int64_t lds, float* __restrict__ hi, int64_t ldh,
+                                  float* __restrict__ lo, int64_t ldl, int64_t M, int64_t N, int vec) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  if (vec) {   // M, lds, ldh, ldl multiples of 4, 16-byte aligned bases
+    const int64_t M4 = M / 4, total = M4 * N;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += stride) {
+      const int64_t i = (idx % M4) * 4, j = idx / M4;
+      const float4 x = *reinterpret_cast<const float4*>(src + i + j * lds);
+      float4 h, l;
+      h.x = rn_tf32(x.x); l.x = rn_tf32(x.x - h.x);
+      h.y = rn_tf32(x.y); l.y = rn_tf32(x.y - h.y);
+      h.z = rn_tf32(x.z); l.z = rn_tf32(x.z - h.z);
+      h.w = rn_tf32(x.w); l.w = rn_tf32(x.w - h.w);
+      *reinterpret_cast<float4*>(hi + i + j * ldh) = h;
+      *reinterpret_cast<float4*>(lo + i + j * ldl) = l;
+    }
+    return;
+  }
+  for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < M * N; idx += stride) {
+    const int64_t i = idx % M, j = idx / M;
+    const float x = src[i + j * lds];
+    const float h = rn_tf32(x);
+    hi[i + j * ldh] = h;
+    lo[i + j * ldl] = rn_tf32(x - h);
+  }
+}
+
+cudaError_t launch_tf32_split(const float* src, int64_t lds, float* hi, int64_t ldh, float* lo, int64_t ldl,
+                              int64_t M, int64_t N, int num_sms, cudaStream_t st) {
+  if (M * N == 0) return cudaSuccess;
+  const bool vec = M % 4 == 0 && lds % 4 == 0 && ldh % 4 == 0 && ldl % 4 == 0 &&
+                   ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(hi) |
+                     reinterpret_cast<uintptr_t>(lo)) & 15) == 0;
+  const int64_t work = vec ? (M / 4) * N : M * N;
+  const int64_t blocks = std::min<int64_t>((work + 255) / 256, (int64_t)num_sms * 8);
+  tf32_split_kernel<<<(unsigned)blocks, 256, 0, st>>>(src, lds, hi, ldh, lo, ldl, M, N, vec ? 1 : 0);
   return cudaGetLastError();
 }
 

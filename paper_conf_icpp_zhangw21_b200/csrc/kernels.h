@@ -8,6 +8,9 @@ namespace rgsqr {
 
 constexpr int LEAF_MAX_W = 64;
 constexpr int LEAF_MAX_G = 160;       // leaf grid size cap (>= SM count)
+// arrivals one exchange word can count (11-bit field, leaf.cu FX_CNT_SHIFT = 53): the leaf grid
+// of a row-sharded run is capped at LEAF_MAX_ARRIVALS / nranks CTAs per GPU
+constexpr int LEAF_MAX_ARRIVALS = 2047;
 constexpr int LEAF_PARTS = 4;         // row quarters of the per-CTA partial sums
 // leaf exchange words: [LEAF_XW_SETS round sets][LEAF_MAX_W+2 values], word i at
 // xw[i * LEAF_XW_STRIDE] (one 256-byte line each: concurrent atomics and polls of different
@@ -123,9 +126,9 @@ cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t l
 template <typename T>
 cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st);
 
-// TF32X3: dst = src - trunc_tf32(src), M x N
-cudaError_t launch_tf32_lo(const float* src, int64_t lds, float* dst, int64_t ldd, int64_t M, int64_t N,
-                           cudaStream_t st);
+// TF32X3 operand split: hi = RN_tf32(src), lo = RN_tf32(src - hi), M x N (R25)
+cudaError_t launch_tf32_split(const float* src, int64_t lds, float* hi, int64_t ldh, float* lo, int64_t ldl,
+                              int64_t M, int64_t N, int num_sms, cudaStream_t st);
 // dst_f[i,j] = src[i,j] (optional) and dst_op[i,j] = RN(src[i,j]) (optional), M x N
 template <typename T>
 cudaError_t launch_copy_cast(const float* src, int64_t lds, float* dst_f, int64_t ldf, T* dst_op, int64_t ldo,

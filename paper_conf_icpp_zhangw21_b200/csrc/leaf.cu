@@ -53,6 +53,8 @@ __device__ __forceinline__ unsigned long long ld_word(const unsigned long long* 
 // bits [0,53) accumulate (v + 2^41) with |v| <= 2^41 per arrival (no carry into the count).
 static constexpr int FX_CNT_SHIFT = 53;
 static constexpr int FX_VBITS = 41;
+static_assert((1 << (64 - FX_CNT_SHIFT)) - 1 == LEAF_MAX_ARRIVALS, "arrival count field width");
+static_assert(LEAF_MAX_G <= LEAF_MAX_ARRIVALS, "one GPU's grid must fit the count field");
 
 __device__ __forceinline__ void st_release_shared(int* p, int v) {
   asm volatile("st.release.cta.shared.b32 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(p)), "r"(v) : "memory");

@@ -135,8 +135,13 @@ struct Exec {
     }
     return v;
   }
-  int64_t pick_tile(size_t avail, int64_t cols_per_slot, bool uncapped = false) const {
-    if (prec == RGSQR_TF32X3) avail /= 2;  // leave room for the per-tile lo operands
+  int64_t pick_tile(size_t avail, int64_t cols_per_slot, bool uncapped = false, int64_t w1w2 = 0) const {
+    if (prec == RGSQR_TF32X3) {
+      // leave room for the per-call hi/lo operands: 2 x (tile of Q1 + tile of A2) and the hi/lo
+      // copies of R12 of the outer product
+      const size_t r = (size_t)w1w2 * 8 + 4096;
+      avail = avail > r ? (avail - r) / 3 : 0;
+    }
     int64_t t = (int64_t)(avail / ((size_t)K * cols_per_slot * s));
     // the ramp's cap bounds streamed tiles; prefetched (flat) rings hold as
     // much of A2 as the budget allows
@@ -367,7 +372,7 @@ struct Exec {
     if (q1_res) {
       char* D = static_cast<char*>(c->arena.alloc(dB));
       const size_t avail = c->arena.free_bytes() > scratch ? c->arena.free_bytes() - scratch : 0;
-      const int64_t t = D ? pick_tile(avail, w2, c->opt.prefetch != 0) : 0;
+      const int64_t t = D ? pick_tile(avail, w2, c->opt.prefetch != 0, w1 * w2) : 0;
       char* ring = t >= 128 ? static_cast<char*>(c->arena.alloc((size_t)K * t * w2 * s)) : nullptr;
       const size_t mark_s = c->arena.mark();
       float* Rs1 = ring ? static_cast<float*>(c->arena.alloc(rsb)) : nullptr;
@@ -437,7 +442,7 @@ struct Exec {
     void* R12op = c->arena.alloc(r12ob);
     float* S = reorth ? static_cast<float*>(c->arena.alloc(r12b)) : R12;
     if (!R12 || !R12op || !S) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: no space for R12");
-    const int64_t t = pick_tile(c->arena.free_bytes() > 4096 ? c->arena.free_bytes() - 4096 : 0, w1 + w2);
+    const int64_t t = pick_tile(c->arena.free_bytes() > 4096 ? c->arena.free_bytes() - 4096 : 0, w1 + w2, false, w1 * w2);
     if (t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "OOC node: ring does not fit the budget");
     char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
     std::vector<cudaEvent_t> ev_free(K);
@@ -638,7 +643,10 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   st.arena_bytes = (int64_t)c->arena.size;
   st.arena_high_water = (int64_t)c->arena.high;
   st.flops = (int64_t)(2.0 * m * (double)n * n);
-  if (brk == -2) return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
+  if (brk == -2) {
+    c->broken = true;
+    return fail(c, RGSQR_ERR_CUDA, "leaf exchange timed out (a rank did not arrive)");
+  }
   st.first_breakdown_col = (brk == 0x7f7f7f7f || brk == INT_MAX) ? -1 : brk;
   c->collect_kernel_stats();
   return st.first_breakdown_col >= 0 ? RGSQR_WARN_RANK_DEFICIENT : RGSQR_OK;

@@ -121,9 +121,9 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
                          int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
                          int accumulate, cudaStream_t st, const void* Q1lo = nullptr, const void* A2lo = nullptr);
 
-// TF32X3 (3-pass split tf32): Q1^T A2 ~= Q1h^T A2h + Q1h^T A2l + Q1l^T A2h, hi = the stored
-// fp32 words read as tf32 (truncated by the MMA), lo = x - trunc_tf32(x); the three
-// products accumulate into R12 in this fixed order.  Error ~ |Q1l||A2l| ~ 2^-22 relative.
+// TF32X3 (3-pass split tf32): Q1^T A2 ~= Q1h^T A2h + Q1h^T A2l + Q1l^T A2h with hi = RN_tf32(x),
+// lo = RN_tf32(x - hi) (R25); the three products accumulate into R12 in one GEMM over
+// three K segments, small terms first.  Error ~ |Q1l||A2l| <= 2^-22 relative per product.
 template <typename T>
 static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
                           int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop,
@@ -131,14 +131,17 @@ static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const v
   if (prec != RGSQR_TF32X3)
     return op_inner_once<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
   const size_t mark = c->arena.mark();
+  float* q_hi = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
   float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
+  float* a_hi = static_cast<float*>(c->arena.alloc((size_t)m * w2 * 4));
   float* a_lo = static_cast<float*>(c->arena.alloc((size_t)m * w2 * 4));
-  if (!q_lo || !a_lo) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner (tf32x3): no space for the lo operands");
-  RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(Q1), ldq, q_lo, m, m, w1, st));
-  RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(A2), lda, a_lo, m, m, w2, st));
+  if (!q_hi || !q_lo || !a_hi || !a_lo)
+    return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner (tf32x3): no space for the hi/lo operands");
+  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, m, q_lo, m, m, w1, c->num_sms, st));
+  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(A2), lda, a_hi, m, a_lo, m, m, w2, c->num_sms, st));
   c->stats.n_other_launches += 2;
   // one GEMM over the three operand segments (K extended 3x): a single split-K reduction
-  int rc = op_inner_once<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st, q_lo, a_lo);
+  int rc = op_inner_once<T>(c, prec, q_hi, m, a_hi, m, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st, q_lo, a_lo);
   c->arena.release(mark);
   return rc;
 }
@@ -173,6 +176,10 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
   // doubled the kernel time: 57 vs 37 us, profiles/r1_splitk_scan.txt).
   int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : c->num_sms / tiles);
   splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.kb_total / 4));
+  // TF32X3: bound the tensor-core accumulation chain (RGSQR_OPT_X3_CHAIN k-blocks per split):
+  // its fp32 accumulator error grows with the chain length, the fixed-order split-K sum is RN
+  if (x3 && c->opt.splitk <= 0 && c->opt.x3_chain > 0)
+    splits = std::max<int64_t>(splits, (p.kb_total + c->opt.x3_chain - 1) / c->opt.x3_chain);
   const size_t cap = std::min<size_t>((size_t)64 << 20, c->arena.free_bytes());
   while (splits > 1 && (size_t)splits * w1 * w2 * 4 + 256 > cap) --splits;
   p.kb_per_split = (p.kb_total + splits - 1) / splits;
@@ -295,15 +302,19 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
     case RGSQR_BF16: return op_outer_t<__nv_bfloat16>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
     case RGSQR_TF32: return op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st);
     case RGSQR_TF32X3: {
-      // A2 <- A2 - (Q1h R12h + Q1h R12l + Q1l R12h): one NN pass over the three segments
+      // A2 <- A2 - (Q1h R12l + Q1l R12h + Q1h R12h): one NN pass over the three segments,
+      // hi = RN_tf32(x), lo = RN_tf32(x - hi) (R25)
       const size_t mark = c->arena.mark();
+      float* q_hi = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
       float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
+      float* r_hi = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
       float* r_lo = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
-      if (!q_lo || !r_lo) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "outer (tf32x3): no space for lo operands");
-      RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(Q1), ldq, q_lo, m, m, w1, st));
-      RGSQR_CUDA(c, launch_tf32_lo(static_cast<const float*>(R12op), ldr, r_lo, w1, w1, w2, st));
+      if (!q_hi || !q_lo || !r_hi || !r_lo)
+        return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "outer (tf32x3): no space for hi/lo operands");
+      RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, m, q_lo, m, m, w1, c->num_sms, st));
+      RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(R12op), ldr, r_hi, w1, r_lo, w1, w1, w2, c->num_sms, st));
       c->stats.n_other_launches += 2;
-      int rc = op_outer_t<float>(c, prec, Q1, ldq, R12op, ldr, A2, lda, m, w1, w2, st, q_lo, r_lo);
+      int rc = op_outer_t<float>(c, prec, q_hi, m, r_hi, w1, A2, lda, m, w1, w2, st, q_lo, r_lo);
       c->arena.release(mark);
       return rc;
     }
@@ -314,6 +325,8 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
 static void leaf_geometry(Ctx* c, int64_t m, int* grid, int* rp) {
   int G = c->opt.leaf_ctas > 0 ? (int)c->opt.leaf_ctas : c->num_sms;
   G = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)G, (int64_t)LEAF_MAX_G, (m + 31) / 32}));
+  // the exchange word counts nranks x G arrivals in its top 11 bits (leaf.cu FX_CNT_SHIFT)
+  G = std::max(1, std::min(G, LEAF_MAX_ARRIVALS / std::max(1, c->nranks)));
   int64_t r = (m + G - 1) / G;
   r = (r + 7) & ~int64_t(7);  // 16-byte aligned row slices for the vector loads
   *grid = G;
@@ -523,7 +536,7 @@ size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n) {
   size_t b = 0;
   if (w1 > 0) b += (size_t)w1 * (n - w1) * elem_bytes(prec) + 1024;  // R12 operand copy
   if (w1 > 0 && c->nccl_comm) b += (size_t)w1 * (n - w1) * 4 + 1024;  // R12 rank-reduction buffer
-  if (prec == RGSQR_TF32X3) b += (size_t)m * n * 4 + 4096;              // lo operands of the top node
+  if (prec == RGSQR_TF32X3) b += (size_t)2 * m * n * 4 + 8192;          // hi/lo operands of the top node
   if (c->opt.reorth) {                                                   // CGS2: S (fp32) + leaf S block
     if (w1 > 0) b += (size_t)w1 * (n - w1) * 4 + 1024;
     b += (size_t)LEAF_MAX_W * LEAF_MAX_W * 4 + 1024;

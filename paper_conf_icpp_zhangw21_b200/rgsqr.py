@@ -23,12 +23,13 @@ STORAGE = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32", "tf32x3": "fp32"}
 OK, WARN_RANK_DEFICIENT = 0, 1
 OPTIONS = {"leaf_width": 1, "tile_rows_min": 2, "tile_rows_max": 3, "ring_depth": 4, "algo": 5,
            "block_cols": 6, "serialize": 7, "reuse": 8, "leaf_ctas": 9, "splitk": 10, "profile": 11,
-           "reorth": 12, "prefetch": 13, "fuse_small": 14, "split_pct": 15}
+           "reorth": 12, "prefetch": 13, "fuse_small": 14, "split_pct": 15,
+           "x3_chain": 16}
 
 EXPORTS = ["rgsqr_create", "rgsqr_get_unique_id", "rgsqr_create_dist", "rgsqr_destroy", "rgsqr_factor",
            "rgsqr_factor_device", "rgsqr_op_leaf", "rgsqr_op_inner", "rgsqr_op_outer", "rgsqr_set_stream",
            "rgsqr_get_stream", "rgsqr_host_alloc", "rgsqr_host_free", "rgsqr_set_option", "rgsqr_get_option",
-           "rgsqr_get_stats", "rgsqr_version", "rgsqr_status_string", "rgsqr_last_error"]
+           "rgsqr_get_stats", "rgsqr_version", "rgsqr_status_string", "rgsqr_last_error", "rgsqr_probe_link"]
 
 
 class Stats(C.Structure):
@@ -93,6 +94,7 @@ def load_library(path: str = LIB_PATH):
         "rgsqr_version": ([], i32),
         "rgsqr_status_string": ([i32], C.c_char_p),
         "rgsqr_last_error": ([vp], C.c_char_p),
+        "rgsqr_probe_link": ([vp, vp, i64, i64, i64, i32, i32, C.POINTER(C.c_double)], i32),
     }
     del fp
     for name, (args, res) in sig.items():
@@ -183,6 +185,13 @@ class Handle:
 
     def host_free(self, p: int):
         self._check(self.lib.rgsqr_host_free(self.h, p), "host_free")
+
+    def probe_link(self, host, ld: int, rows: int, cols: int, elem_bytes: int, reps: int = 4) -> dict:
+        """Host-link GB/s of the executor's 2D tile copies (H2D, D2H, duplex total)."""
+        out = (C.c_double * 3)()
+        self._check(self.lib.rgsqr_probe_link(self.h, _ptr(host), ld, rows, cols, elem_bytes, reps, out),
+                    "probe_link")
+        return {"h2d": out[0], "d2h": out[1], "duplex_total": out[2]}
 
     # ---- factorizations ----
     def factor(self, A, lda: int, m: int, n: int, Q, R, precision: str = "fp16", budget: int = 0) -> int:

@@ -174,6 +174,43 @@ def dyadic_mixed(m: int, n: int, seed: int = 0) -> tuple[np.ndarray, np.ndarray]
     return a, r0
 
 
+def hadamard_cols(m: int, c0: int, c1: int) -> np.ndarray:
+    """Columns [c0, c1) of hadamard(m, .) (float64, Fortran order), via popcount of i & k."""
+    j = int(round(np.log(m) / np.log(4)))
+    if 4 ** j != m:
+        raise ValueError("m must be a power of 4")
+    i = np.arange(m, dtype=np.uint64)[:, None]
+    k = np.arange(c0, c1, dtype=np.uint64)[None, :]
+    par = (np.bitwise_count(i & k) & 1).astype(np.float64)
+    return np.asfortranarray((1.0 - 2.0 * par) * 2.0 ** (-j))
+
+
+def dyadic_mixed_storage(m: int, n: int, seed: int = 0, dtype: str = "fp16",
+                         chunk: int = 256) -> tuple[np.ndarray, np.ndarray]:
+    """(A, R0) of dyadic_mixed, written column chunk by column chunk straight into the storage
+    type (every entry is exact there), in parallel: for configs[2]-sized inputs whose fp64
+    copy would not fit host memory.  Bit-identical to to_storage(dyadic_mixed(m, n, seed))."""
+    r0 = dyadic_r0(n, seed)
+    out = np.empty((m, n), dtype=storage_numpy_dtype(dtype), order="F")
+
+    def fill(c0):
+        c1 = min(n, c0 + chunk)
+        lo0 = max(0, c0 - 4)
+        h = hadamard_cols(m, lo0, c1)
+        blk = np.empty((m, c1 - c0), order="F")
+        for j in range(c0, c1):
+            lo = max(0, j - 4)
+            blk[:, j - c0] = h[:, lo - lo0:j + 1 - lo0] @ r0[lo:j + 1, j]
+        out[:, c0:c1] = to_storage(blk, dtype)
+
+    from concurrent.futures import ThreadPoolExecutor
+    import os
+    # (each worker holds ~ 2 m chunk fp64 temporaries: at most 8 workers)
+    with ThreadPoolExecutor(max_workers=min(8, len(os.sched_getaffinity(0)))) as ex:
+        list(ex.map(fill, range(0, n, chunk)))
+    return out, r0
+
+
 # ----------------------------------------------------------------------------------
 # G2: dense U diag(sigma) V^T, prescribed condition number
 # ----------------------------------------------------------------------------------

@@ -162,3 +162,25 @@ def test_ooc_split_ratio_ablation(h, gauss, split_pct):
     assert oracle.is_upper_triangular(Rg)
     assert oracle.backward_error(X, gi.to_float64(Q, "fp16"), Rg) < 5e-3
     assert oracle.r_rel_error(Rg, ref.R) < 5e-3
+
+
+@pytest.mark.parametrize("prec,lda_pad", [("fp16", 8), ("bf16", 120), ("tf32", 4)])
+def test_host_path_lda_greater_than_m(h, prec, lda_pad):
+    """lda > m (LAPACK convention, include/rgsqr.h): A and Q live in a taller host buffer; the
+    rows [m, lda) of Q_out must not be touched, and the result equals the lda = m run bitwise
+    (same tiles, same kernels), out-of-core under a small budget."""
+    st = STOR[prec]
+    m, n = 8192, 512
+    lda = m + lda_pad
+    A = gi.gaussian(m, n, seed=21, dtype=st)
+    big = np.zeros((lda, n), dtype=A.dtype, order="F")
+    big[:m] = A
+    Qb = np.full_like(big, 7, order="F")
+    Rb = np.full((n, n), np.nan, dtype=np.float32, order="F")
+    budget = 6 * MiB if st != "fp32" else 12 * MiB
+    rc = h.factor(big, lda, m, n, Qb, Rb, precision=prec, budget=budget)
+    assert rc == 0 and h.stats()["n_ooc_nodes"] >= 1
+    assert np.all(Qb[m:] == 7)
+    rc, Q, R, _ = factor(h, np.asfortranarray(A), prec, budget)
+    np.testing.assert_array_equal(Rb, R)
+    np.testing.assert_array_equal(Qb[:m], Q)
