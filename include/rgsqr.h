@@ -98,6 +98,16 @@ enum rgsqr_option {
                                    operand segment) accumulate in one tensor-core fp32 chain; longer K is
                                    split and the partials summed in fixed order on the CUDA cores
                                    (R25).  0 = the automatic one-wave split */
+  ,RGSQR_OPT_COLCHUNK = 17      /* 1 = column-chunked out-of-core node (DAG lookahead across the OOC
+                                   boundary; R26): when the left child is
+                                   in-core and resident, A2 is uploaded in the column order the right
+                                   child consumes, R12 = Q1^T A2 and A2 -= Q1 R12 are applied per column
+                                   chunk, and the right child starts while later columns are still in
+                                   flight; the columns that do not fit beside Q1 are projected first
+                                   from the host and re-uploaded once Q1's memory is free.  0 = the
+                                   row-tile streamed node.  Default 1 */
+  ,RGSQR_OPT_EAGER_PCT = 18     /* column-chunked node: complete the Q1 projection when the right child's
+                                   leaves reach this percentage of its left half (default 75) */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

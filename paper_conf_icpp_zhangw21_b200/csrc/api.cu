@@ -160,6 +160,7 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaStreamCreateWithFlags(&c->st_h2d, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_d2h, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_d2r, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->st_h2d2, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
       cudaMalloc(&c->d_sn_partials, sizeof(float) * LEAF_MAX_G * 128 * 128) != cudaSuccess ||
       cudaMalloc(&c->d_sn_r12op, 128 * 128 * 4) != cudaSuccess ||
@@ -327,6 +328,7 @@ int rgsqr_destroy(rgsqr_handle h) {
   cudaStreamDestroy(c->st_h2d);
   cudaStreamDestroy(c->st_d2h);
   cudaStreamDestroy(c->st_d2r);
+  cudaStreamDestroy(c->st_h2d2);
   delete c;
   return RGSQR_OK;
 }
@@ -441,6 +443,8 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_FUSE_SMALL: return &o.fuse_small;
     case RGSQR_OPT_SPLIT_PCT: return &o.split_pct;
     case RGSQR_OPT_X3_CHAIN: return &o.x3_chain;
+    case RGSQR_OPT_COLCHUNK: return &o.colchunk;
+    case RGSQR_OPT_EAGER_PCT: return &o.eager_pct;
   }
   return nullptr;
 }

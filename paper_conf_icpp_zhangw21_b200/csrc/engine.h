@@ -31,6 +31,9 @@ struct Options {
   int64_t fuse_small = 1;    // fused kernel for nodes with w1, w2 <= 64 (RGSQR_OPT_FUSE_SMALL)
   int64_t split_pct = 50;    // OOC split: left child width in % (RGSQR_OPT_SPLIT_PCT; 50 = halves, the paper)
   int64_t x3_chain = 0;      // TF32X3: max k-blocks per split-K chain (RGSQR_OPT_X3_CHAIN; 0 = one-wave rule)
+  int64_t colchunk = 1;      // column-chunked OOC node (RGSQR_OPT_COLCHUNK, R26)
+  int64_t eager_pct = 75;    // column-chunked node: the external projection is completed once the right
+                             // child's leaves reach this % of its left half (RGSQR_OPT_EAGER_PCT)
 };
 
 struct KernSeg {
@@ -70,6 +73,7 @@ struct Ctx {
   cudaStream_t st_user = nullptr;   // set by rgsqr_set_stream
   cudaStream_t st_own = nullptr;
   cudaStream_t st_h2d = nullptr, st_d2h = nullptr, st_d2r = nullptr;   // copies: in, Q out, R out
+  cudaStream_t st_h2d2 = nullptr;   // second upload queue (small uploads that must not queue behind prefetches)
   Options opt;
   rgsqr_stats stats{};
   std::string last_error;
@@ -162,12 +166,31 @@ size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n);
 // overlap a node's column upload / Q download with its factorization:
 //   need(c)      -- called before any op that reads columns [0, c) of the node
 //   leaf_done(c) -- called after the leaf ending at column c (Q[:, 0:c) is final)
+// A deferred projection against a Q1 that is NOT part of the node (the left child of an
+// out-of-core parent, resident in HBM): for node columns [0, end), R12 = Q1^T A2 and
+// A2 -= Q1 R12 (Eq. 2), applied chunk by chunk before the node's own deferred
+// products (ancestor first), R12 handed to r_out (downloaded to the host R) per chunk.
+struct ExtProduct {
+  const void* Q1 = nullptr;
+  int64_t ldq = 0, w1 = 0;
+  int64_t end = 0;                            // node columns [0, end) receive the product
+  int64_t applied = 0;
+  float* R12[2] = {nullptr, nullptr};         // w1 x chunk fp32, alternating
+  cudaEvent_t free_ev[2] = {nullptr, nullptr};  // R12[i] may be overwritten after this event
+  void* R12op = nullptr;                      // w1 x chunk, operand type
+  int n_done = 0;
+  std::function<cudaEvent_t(int64_t a, int64_t b, const float* R12)> r_out;  // download; event after it
+  std::function<void()> done;                 // after the last chunk: Q1 is dead once sc gets there
+};
+
 struct IncoreHooks {
   std::function<void(int64_t)> need;          // make the compute stream wait for columns < col_end
   std::function<void(int64_t)> leaf_done;     // columns < col_end are final
   std::function<bool(int64_t)> pending;       // need(col_end) would still wait on an upload
   int64_t chunk = 0;                          // upload chunk width (columns)
+  ExtProduct* ext = nullptr;                  // optional projection against an external Q1
 };
+int apply_ext(Ctx* c, int prec, char* A, int64_t lda, int64_t m, IncoreHooks* hk, int64_t upto, cudaStream_t st);
 int incore_factor(Ctx* c, int prec, void* A, int64_t lda, int64_t m, int64_t n, float* R, int64_t ldr,
                   int64_t col_offset, cudaStream_t st, IncoreHooks* hooks = nullptr);
 int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* Q, float* R, int prec,

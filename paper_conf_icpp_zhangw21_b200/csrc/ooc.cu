@@ -56,6 +56,7 @@ struct Exec {
   int64_t tmin, tmax;
   bool reuse;
   bool reorth;
+  cudaStream_t sh2 = nullptr;    // second upload queue (column-chunked node's late tail piece)
 
   // ---- timing / accounting helpers ----
   cudaEvent_t seg_begin(cudaStream_t st) {
@@ -78,18 +79,27 @@ struct Exec {
     wait(sc, sh);
     wait(sc, sd);
     wait(sc, sr);
+    if (sh2) wait(sc, sh2);
     wait(sh, sc);
     wait(sd, sc);
     wait(sr, sc);
+    if (sh2) wait(sh2, sc);
+  }
+  cudaEvent_t mark_ev(cudaStream_t st) {
+    cudaEvent_t e = c->ev();
+    cudaEventRecord(e, st);
+    return e;
   }
   const char* hsrc(bool q) const { return q ? Q : A; }
   const char* hptr(const char* base, int64_t r0, int64_t col) const { return base + (r0 + col * lda) * s; }
 
-  int h2d(void* dst, int64_t ldd, const char* base, int64_t r0, int64_t rows, int64_t c0, int64_t cols) {
-    cudaEvent_t a = seg_begin(sh);
+  int h2d(void* dst, int64_t ldd, const char* base, int64_t r0, int64_t rows, int64_t c0, int64_t cols,
+          cudaStream_t on = nullptr) {
+    if (!on) on = sh;
+    cudaEvent_t a = seg_begin(on);
     RGSQR_CUDA(c, cudaMemcpy2DAsync(dst, ldd * s, hptr(base, r0, c0), lda * s, rows * s, cols,
-                                    cudaMemcpyHostToDevice, sh));
-    seg_end(0, sh, a);
+                                    cudaMemcpyHostToDevice, on));
+    seg_end(0, on, a);
     c->stats.h2d_bytes += rows * cols * s;
     c->stats.h2d_matrix_bytes += rows * cols * s;
     return RGSQR_OK;
@@ -154,8 +164,18 @@ struct Exec {
   // ---- in-core node: upload (unless resident), factor, stream Q and R out ----
   // Rs_ext: caller-owned R block (kept alive by the caller, so no stream has to wait for
   // its download here); nullptr = allocate it from the arena and fence its reuse.
+  // Feed of a node whose columns arrive from elsewhere (column-chunked OOC node, f4): uploads
+  // already issued (column offset, completion event), one LATE chunk issued by the caller once
+  // its memory is free (event filled in then), and a projection against an external Q1.
+  struct Feed {
+    std::vector<std::pair<int64_t, cudaEvent_t>> chunks;   // sorted by column; late one last
+    int64_t late_col = -1;                                 // first column of the late chunk
+    ExtProduct* ext = nullptr;
+    int64_t eager_col = -1;   // leaf_done(col >= eager_col): apply the whole ext product now
+  };
+
   int incore_node(int64_t c0, int64_t w, bool src_q, char* D, bool resident, cudaEvent_t* q_done,
-                  float* Rs_ext = nullptr) {
+                  float* Rs_ext = nullptr, Feed* feed = nullptr) {
     const size_t mark = c->arena.mark();
     float* Rs = Rs_ext ? Rs_ext : static_cast<float*>(c->arena.alloc((size_t)w * w * 4));
     if (!Rs) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core node: no space for R block");
@@ -163,8 +183,9 @@ struct Exec {
     const int64_t leaf = std::max(1, leaf_width_for(c, m));
     int64_t cw = ((int64_t)32 << 20) / std::max<int64_t>(1, m * s);
     cw = std::max<int64_t>(leaf, cw / 64 * 64);
-    std::vector<std::pair<int64_t, cudaEvent_t>> chunks;
-    if (!resident) {
+    std::vector<std::pair<int64_t, cudaEvent_t>> own;
+    std::vector<std::pair<int64_t, cudaEvent_t>>& chunks = feed ? feed->chunks : own;
+    if (!resident && !feed) {
       for (int64_t a = 0; a < w; a += cw) {
         const int64_t cols = std::min(cw, w - a);
         int rc = h2d(D + a * m * s, m, hsrc(src_q), 0, m, c0 + a, cols);
@@ -180,17 +201,34 @@ struct Exec {
     IncoreHooks hk;
     hk.need = [&](int64_t col_end) {
       while (next < chunks.size() && chunks[next].first < col_end) {
+        if (!chunks[next].second) {   // a late chunk must be issued before anyone waits for it
+          err = fail(c, RGSQR_ERR_CUDA, "column-chunked node: late chunk awaited before it was issued");
+          return;
+        }
         cudaStreamWaitEvent(sc, chunks[next].second, 0);
         ++next;
       }
     };
-    hk.pending = [&](int64_t col_end) { return next < chunks.size() && chunks[next].first < col_end; };
+    // (a late chunk counts as pending only until it is issued: afterwards the recursion waits
+    // for it instead of deferring whole products into column pieces)
+    hk.pending = [&](int64_t col_end) {
+      if (next >= chunks.size() || chunks[next].first >= col_end) return false;
+      return !(feed && chunks[next].first == feed->late_col && chunks[next].second);
+    };
+    if (feed) hk.ext = feed->ext;
     // deferred products are applied in pieces of >= 256 columns (a multiple of the upload
     // chunk): narrower products (tall m makes cw small) would run at a fraction of the MMA rate
     hk.chunk = cw * std::max<int64_t>(1, (256 + cw - 1) / cw);
     // Q columns and the matching R columns (full height: entries below the diagonal are zero
     // and stay zero) go out as soon as a chunk of leaves is final
     hk.leaf_done = [&](int64_t col_end) {
+      if (feed && feed->ext && feed->eager_col >= 0 && col_end >= feed->eager_col &&
+          feed->ext->applied < feed->ext->end) {
+        // apply the rest of the external projection now, so that Q1's memory frees (and the late
+        // chunk uploads) while the recursion still works on earlier columns
+        int rc = apply_ext(c, prec, D, m, m, &hk, feed->ext->end, sc);
+        if (rc < 0) err = rc;
+      }
       if (col_end - flushed < cw && col_end < w) return;
       wait(sd, sc);
       int rc = d2h(Q, 0, m, c0 + flushed, col_end - flushed, D + flushed * m * s, m);
@@ -508,6 +546,210 @@ struct Exec {
     return RGSQR_OK;
   }
 
+  // ---- column-chunked out-of-core node (f4, R26) ----------------------------------
+  // The left child fits in-core: Q1 stays resident (rule 1).  A2 is split by COLUMNS into a head
+  // [0, wh) that fits beside Q1 and a tail [wh, w2) that does not.  Arena layout:
+  //     [ H : m x wh  (head; its top part first hosts the left child's workspace) ]
+  //     [ D : m x w1  (Q1; after Q1 is dead its first wt columns receive the tail) ]
+  //     [ X :         (tail piece T1 while prefetched, then the right child's workspace) ]
+  // so that [H | D[:, :wt]] is the right child's contiguous m x w2 matrix (ld m).
+  //   1. left child in-core in D (its columns uploaded in chunks, Q1 downloaded as leaves end);
+  //      uploads queue behind it: the tail piece T1 (into X), then the head columns (into H).
+  //   2. tail: R12_t = Q1^T A2_t, A2_t -= Q1 R12_t (Eq. 2) on the resident tail
+  //      pieces, R12_t and A2_t' downloaded (A2_t' parked in the host Q columns it will occupy).
+  //   3. right child in-core on [H | D[:, :wt]] at once: the head's R12 = Q1^T A2 and
+  //      A2 -= Q1 R12 are applied column chunk by column chunk as the recursion reaches the
+  //      columns (ExtProduct, ancestor first), completed eagerly part-way through; then Q1 is
+  //      dead and A2_t' is uploaded into D while the recursion continues on earlier columns.
+  // Same arithmetic per output element as the streamed node: every R12 column is Q1^T a_j over
+  // all m rows and every A2' column is a_j - Q1 r_j (the column split only regroups the GEMMs).
+  struct CCPlan {
+    int64_t wh = 0, wt1 = 0, wt2 = 0;
+    size_t htop = 0;                 // bytes at the top of H used as scratch (left child, tail phase)
+    int64_t ch = 0;                  // upload / product chunk width
+  };
+  bool plan_cc(int64_t w1, int64_t w2, size_t free0, CCPlan* P) const {
+    if (w2 > w1 || (m * s * 64) % 256 != 0) return false;
+    const int64_t leaf = std::max(1, leaf_width_for(c, m));
+    int64_t cw = ((int64_t)32 << 20) / std::max<int64_t>(1, m * s);
+    cw = std::max<int64_t>(leaf, cw / 64 * 64);
+    const int64_t ch = cw * std::max<int64_t>(1, (256 + cw - 1) / cw);
+    const size_t colb = (size_t)m * s, dB = (size_t)m * w1 * s;
+    const size_t left_ws = incore_need(w1) - dB + 4096;
+    const size_t ext_b = 2 * ((size_t)w1 * ch * 4 + 256) + (size_t)w1 * ch * s + 256;
+    const size_t right_ws = (size_t)w2 * w2 * 4 + 256 + incore_workspace_bytes(c, prec, m, w2) + ext_b + 16384;
+    for (int64_t wh = (w2 - 1) / 64 * 64; wh >= std::max<int64_t>(64, w2 / 4); wh -= 64) {
+      const size_t H = colb * wh;
+      if (H + dB + right_ws > free0) continue;
+      const int64_t wt = w2 - wh;
+      const size_t X = free0 - H - dB;
+      const int64_t wt1 = std::min<int64_t>(wt, (int64_t)(X / colb) / 8 * 8);
+      const int64_t wt2 = wt - wt1;
+      const size_t tail_ws = (size_t)w1 * wt * (4 + s) + 1024 + (size_t)wt2 * colb + 256;
+      const size_t htop = (std::max(left_ws, tail_ws) + 4095) / 4096 * 4096;
+      if (htop > H || wt > w1) continue;
+      P->wh = wh;
+      P->wt1 = wt1;
+      P->wt2 = wt2;
+      P->htop = htop;
+      P->ch = ch;
+      return true;
+    }
+    return false;
+  }
+
+  // sets the arena's bump window to [lo, hi) (allocations of a phase that lives inside a region
+  // reserved by an earlier allocation); returns the previous (top, size)
+  std::pair<size_t, size_t> window(char* lo, char* hi) {
+    std::pair<size_t, size_t> w{c->arena.top, c->arena.size};
+    c->arena.top = (size_t)(lo - c->arena.base);
+    c->arena.size = (size_t)(hi - c->arena.base);
+    return w;
+  }
+  void unwindow(std::pair<size_t, size_t> w) {
+    c->arena.top = w.first;
+    c->arena.size = w.second;
+  }
+
+  int ooc_node_cc(int64_t c0, int64_t w1, int64_t w2, bool src_q, const CCPlan& P) {
+    const int64_t h = c0 + w1, wh = P.wh, wt1 = P.wt1, wt2 = P.wt2, wt = wt1 + wt2, ch = P.ch;
+    const size_t colb = (size_t)m * s;
+    const size_t mark0 = c->arena.mark();
+    char* H = static_cast<char*>(c->arena.alloc(colb * wh));
+    char* D = static_cast<char*>(c->arena.alloc(colb * w1));
+    if (!H || !D || D != H + colb * wh) {
+      c->arena.release(mark0);
+      return 1;   // layout not contiguous: caller falls back to the streamed node
+    }
+    c->stats.n_ooc_nodes++;
+    char* T1 = wt1 > 0 ? static_cast<char*>(c->arena.alloc(colb * wt1)) : nullptr;
+    if (wt1 > 0 && !T1) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the tail");
+    const size_t x_mark = c->arena.mark();   // (X holds T1 until the right child starts)
+    char* Hend = H + colb * wh;
+    char* Htop = Hend - P.htop;
+    const int64_t htop_col = (int64_t)((size_t)(Htop - H) / colb);   // head columns clear of the scratch
+    // ---- 1. left child in-core in D; its workspace lives in the top of H ----
+    auto wsave = window(Htop, Hend);
+    float* Rs1 = static_cast<float*>(c->arena.alloc((size_t)w1 * w1 * 4));
+    if (!Rs1) {
+      unwindow(wsave);
+      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the left R block");
+    }
+    cudaEvent_t q1_done = nullptr;
+    int rc = incore_node(c0, w1, src_q, D, false, &q1_done, Rs1);
+    unwindow(wsave);
+    if (rc < 0) return rc;
+    cudaEvent_t left_done = mark_ev(sc);
+    cudaEvent_t left_r = r_done;
+    // ---- uploads queued behind the left child's: tail piece 1, then the head clear of H's top ----
+    cudaEvent_t ev_t1 = nullptr, ev_t2 = nullptr;
+    if (wt1 > 0) {
+      rc = h2d(T1, m, hsrc(src_q), 0, m, h + wh, wt1);
+      if (rc < 0) return rc;
+      ev_t1 = mark_ev(sh);
+    }
+    Feed feed;
+    for (int64_t a = 0; a < htop_col; a += ch) {
+      const int64_t cols = std::min(ch, htop_col - a);
+      rc = h2d(H + a * colb, m, hsrc(src_q), 0, m, h + a, cols);
+      if (rc < 0) return rc;
+      feed.chunks.push_back({a, mark_ev(sh)});
+    }
+    // ---- 2. the tail: its workspace and second piece in the top of H (free after the left child) ----
+    if (left_r) cudaStreamWaitEvent(sc, left_r, 0);
+    wsave = window(Htop, Hend);
+    float* R12t = static_cast<float*>(c->arena.alloc((size_t)w1 * wt * 4));
+    char* R12top = static_cast<char*>(c->arena.alloc((size_t)w1 * wt * s));
+    char* T2 = wt2 > 0 ? static_cast<char*>(c->arena.alloc(colb * wt2)) : nullptr;
+    unwindow(wsave);
+    if (!R12t || !R12top || (wt2 > 0 && !T2))
+      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the tail products");
+    if (wt2 > 0) {
+      // a second queue: this piece must not wait behind the head prefetch
+      cudaStreamWaitEvent(sh2, left_done, 0);
+      if (left_r) cudaStreamWaitEvent(sh2, left_r, 0);
+      rc = h2d(T2, m, hsrc(src_q), 0, m, h + wh + wt1, wt2, sh2);
+      if (rc < 0) return rc;
+      ev_t2 = mark_ev(sh2);
+    }
+    cudaEvent_t a_seg = seg_begin(sc);
+    struct Piece { char* T; int64_t col, w; cudaEvent_t ev; };
+    const Piece pieces[2] = {{T1, 0, wt1, ev_t1}, {T2, wt1, wt2, ev_t2}};
+    for (const Piece& pc : pieces) {
+      if (pc.w == 0) continue;
+      cudaStreamWaitEvent(sc, pc.ev, 0);
+      rc = op_inner(c, prec, D, m, pc.T, m, m, w1, pc.w, R12t + pc.col * w1, w1, R12top + pc.col * w1 * s, w1, 0, sc);
+      if (rc < 0) return rc;
+    }
+    wait(sd, sc);
+    rc = d2h_r(c0, h + wh, w1, wt, R12t, w1);
+    if (rc < 0) return rc;
+    cudaEvent_t r12t_out = r_done;
+    for (const Piece& pc : pieces) {
+      if (pc.w == 0) continue;
+      rc = op_outer(c, prec, D, m, R12top + pc.col * w1 * s, w1, pc.T, m, m, w1, pc.w, sc);
+      if (rc < 0) return rc;
+    }
+    seg_end(2, sc, a_seg);
+    wait(sd, sc);
+    for (const Piece& pc : pieces) {
+      if (pc.w == 0) continue;
+      rc = d2h(Q, 0, m, h + wh + pc.col, pc.w, pc.T, m);   // A2_t' parked in its host Q columns
+      if (rc < 0) return rc;
+    }
+    cudaEvent_t tail_out = mark_ev(sd);
+    cudaEvent_t tail_done = mark_ev(sc);
+    // the rest of the head goes into H's top once the tail phase has released it
+    cudaStreamWaitEvent(sh, tail_done, 0);
+    cudaStreamWaitEvent(sh, tail_out, 0);
+    if (r12t_out) cudaStreamWaitEvent(sh, r12t_out, 0);
+    for (int64_t a = htop_col; a < wh;) {
+      const int64_t end = std::min(wh, (a / ch + 1) * ch);
+      rc = h2d(H + a * colb, m, hsrc(src_q), 0, m, h + a, end - a);
+      if (rc < 0) return rc;
+      feed.chunks.push_back({a, mark_ev(sh)});
+      a = end;
+    }
+    // ---- 3. the right child, with the head's Q1 projection applied as its columns are reached ----
+    cudaStreamWaitEvent(sc, tail_out, 0);          // X (T1) becomes the right child's workspace
+    c->arena.release(T1 ? (size_t)(T1 - c->arena.base) : x_mark);
+    ExtProduct ext;
+    ext.Q1 = D;
+    ext.ldq = m;
+    ext.w1 = w1;
+    ext.end = wh;
+    ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * ch * 4));
+    ext.R12[1] = static_cast<float*>(c->arena.alloc((size_t)w1 * ch * 4));
+    ext.R12op = c->arena.alloc((size_t)w1 * ch * s);
+    if (!ext.R12[0] || !ext.R12[1] || !ext.R12op)
+      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the projection chunks");
+    ext.r_out = [&](int64_t a, int64_t b, const float* R12) -> cudaEvent_t {
+      wait(sd, sc);
+      if (d2h_r(c0, h + a, w1, b - a, R12, w1) < 0) return nullptr;
+      return r_done;
+    };
+    feed.late_col = wh;
+    feed.chunks.push_back({wh, nullptr});
+    ext.done = [&]() {
+      // Q1 is dead once the compute stream gets here: the tail goes into D's first columns
+      cudaEvent_t q1_dead = mark_ev(sc);
+      cudaStreamWaitEvent(sh, q1_dead, 0);
+      cudaStreamWaitEvent(sh, tail_out, 0);
+      if (h2d(D, m, Q, 0, m, h + wh, wt) < 0) return;
+      feed.chunks.back().second = mark_ev(sh);
+    };
+    feed.ext = &ext;
+    const int64_t leaf = std::max(1, leaf_width_for(c, m));
+    const int64_t hw = split_width(w2, leaf);
+    feed.eager_col = hw > 0 ? std::max<int64_t>(leaf, hw * c->opt.eager_pct / 100) : -1;
+    rc = incore_node(h, w2, true, H, true, nullptr, nullptr, &feed);
+    if (rc < 0) return rc;
+    if (ext.applied < ext.end) return fail(c, RGSQR_ERR_CUDA, "column-chunked node: projection incomplete");
+    join_all();
+    c->arena.release(mark0);
+    return RGSQR_OK;
+  }
+
   // recursive algorithm (Eq. 2)
   int node(int64_t c0, int64_t w, bool src_q) {
     if (incore_need(w) <= c->arena.free_bytes()) return panel(c0, w, src_q);
@@ -518,6 +760,12 @@ struct Exec {
       // busy anyway, leaves a shorter right child -- the one phase that cannot overlap transfers
       const int64_t t = (w * c->opt.split_pct / 100 + 63) / 64 * 64;
       if (t >= 64 && t <= w - 64) w1 = t;
+    }
+    CCPlan P;
+    if (c->opt.colchunk && reuse && !reorth && prec != RGSQR_TF32X3 && sh2 != nullptr &&
+        plan_cc(w1, w - w1, c->arena.free_bytes(), &P)) {
+      int rc = ooc_node_cc(c0, w1, w - w1, src_q, P);
+      if (rc != 1) return rc;
     }
     return ooc_node(c0, w1, w - w1, src_q, true);
   }
@@ -586,7 +834,8 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   Exec x{c, prec, s, static_cast<const char*>(A), static_cast<char*>(Q), lda, m, n, R,
          c->compute(), c->st_h2d, c->st_d2h, c->st_d2r, (int)c->opt.ring_depth, c->opt.tile_rows_min,
          c->opt.tile_rows_max, c->opt.reuse != 0, c->opt.reorth != 0};
-  if (c->opt.serialize) x.sh = x.sd = x.sr = x.sc;
+  x.sh2 = c->st_h2d2;
+  if (c->opt.serialize) x.sh = x.sd = x.sr = x.sh2 = x.sc;
   // make the copy streams start after prior work of the compute stream
   x.join_all();
   cudaEvent_t t_ref = c->ev();

@@ -573,9 +573,39 @@ struct IncoreCtx {
   std::vector<Deferred> deferred;
 };
 
+// external projection (ExtProduct) of node columns [applied, upto): chunk by chunk, each
+// chunk's upload awaited first
+int apply_ext(Ctx* c, int prec, char* A, int64_t lda, int64_t m, IncoreHooks* hk, int64_t upto, cudaStream_t st) {
+  ExtProduct* e = hk->ext;
+  if (!e) return RGSQR_OK;
+  const int64_t s = elem_bytes(prec);
+  upto = std::min(upto, e->end);
+  const int64_t ch = std::max<int64_t>(hk->chunk, 64);
+  while (e->applied < upto) {
+    const int64_t a = e->applied, b = std::min(e->end, (a / ch + 1) * ch);
+    hk->need(b);
+    const int slot = e->n_done & 1;
+    if (e->free_ev[slot]) cudaStreamWaitEvent(st, e->free_ev[slot], 0);
+    char* A2 = A + a * lda * s;
+    int rc = op_inner(c, prec, e->Q1, e->ldq, A2, lda, m, e->w1, b - a, e->R12[slot], e->w1, e->R12op, e->w1, 0, st);
+    if (rc < 0) return rc;
+    rc = op_outer(c, prec, e->Q1, e->ldq, e->R12op, e->w1, A2, lda, m, e->w1, b - a, st);
+    if (rc < 0) return rc;
+    e->free_ev[slot] = e->r_out ? e->r_out(a, b, e->R12[slot]) : nullptr;
+    e->n_done++;
+    e->applied = b;
+    if (e->applied >= e->end && e->done) e->done();
+  }
+  return RGSQR_OK;
+}
+
 // columns < col_end: wait for their upload, then apply the deferred products to them
 static int incore_need(IncoreCtx& k, int64_t col_end) {
   if (!k.hooks || !k.hooks->need) return RGSQR_OK;
+  if (k.hooks->ext) {
+    int rc = apply_ext(k.c, k.prec, k.A, k.lda, k.m, k.hooks, col_end, k.st);
+    if (rc < 0) return rc;
+  }
   for (auto& d : k.deferred) {
     while (d.applied < std::min(col_end, d.end)) {
       const int64_t a = d.applied;
