@@ -144,6 +144,9 @@ typedef struct rgsqr_stats {
   int64_t kern_launches[4];
   double  kern_flops[4];
   double  kern_bytes[4];
+  int64_t n_colchunk_nodes;     /* out-of-core nodes run column-chunked (RGSQR_OPT_COLCHUNK) */
+  int64_t colchunk_tail_cols;   /* columns of those nodes projected from the host before the right
+                                   child (they did not fit beside Q1) */
 } rgsqr_stats;
 
 /* ---- lifetime -------------------------------------------------------------------- */

@@ -622,6 +622,8 @@ struct Exec {
       return 1;   // layout not contiguous: caller falls back to the streamed node
     }
     c->stats.n_ooc_nodes++;
+    c->stats.n_colchunk_nodes++;
+    c->stats.colchunk_tail_cols += wt;
     char* T1 = wt1 > 0 ? static_cast<char*>(c->arena.alloc(colb * wt1)) : nullptr;
     if (wt1 > 0 && !T1) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the tail");
     const size_t x_mark = c->arena.mark();   // (X holds T1 until the right child starts)
@@ -681,7 +683,6 @@ struct Exec {
       rc = op_inner(c, prec, D, m, pc.T, m, m, w1, pc.w, R12t + pc.col * w1, w1, R12top + pc.col * w1 * s, w1, 0, sc);
       if (rc < 0) return rc;
     }
-    wait(sd, sc);
     rc = d2h_r(c0, h + wh, w1, wt, R12t, w1);
     if (rc < 0) return rc;
     cudaEvent_t r12t_out = r_done;
@@ -724,7 +725,6 @@ struct Exec {
     if (!ext.R12[0] || !ext.R12[1] || !ext.R12op)
       return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the projection chunks");
     ext.r_out = [&](int64_t a, int64_t b, const float* R12) -> cudaEvent_t {
-      wait(sd, sc);
       if (d2h_r(c0, h + a, w1, b - a, R12, w1) < 0) return nullptr;
       return r_done;
     };

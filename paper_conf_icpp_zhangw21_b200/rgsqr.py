@@ -42,7 +42,8 @@ class Stats(C.Structure):
                 ("n_other_launches", C.c_int64), ("n_ooc_nodes", C.c_int64), ("n_incore_nodes", C.c_int64),
                 ("first_breakdown_col", C.c_int64), ("flops", C.c_int64),
                 ("kern_ms", C.c_double * 4), ("kern_launches", C.c_int64 * 4),
-                ("kern_flops", C.c_double * 4), ("kern_bytes", C.c_double * 4)]
+                ("kern_flops", C.c_double * 4), ("kern_bytes", C.c_double * 4),
+                ("n_colchunk_nodes", C.c_int64), ("colchunk_tail_cols", C.c_int64)]
 
     def as_dict(self):
         out = {}

@@ -184,3 +184,60 @@ def test_host_path_lda_greater_than_m(h, prec, lda_pad):
     rc, Q, R, _ = factor(h, np.asfortranarray(A), prec, budget)
     np.testing.assert_array_equal(Rb, R)
     np.testing.assert_array_equal(Qb[:m], Q)
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+@pytest.mark.parametrize("budget_mib", [34, 38, 40])
+def test_colchunk_node_vs_streamed_node(h, prec, budget_mib):
+    """Column-chunked OOC node (RGSQR_OPT_COLCHUNK, R26; PAPER.md:231-233 cross-operation
+    overlap): the right child starts while A2's later columns are in flight, the tail that does not
+    fit beside Q1 is projected from the host first.  Same factorization as the row-tile streamed
+    node (Eq. 2): both against the oracle, and against each other."""
+    st = STOR[prec]
+    m, n = 16384, 1024
+    A = gi.gaussian(m, n, seed=31, dtype=st)
+    X = gi.to_float64(A, st)
+    ref = oracle.rgs(X, leaf=64)
+    budget = budget_mib * MiB * (2 if st == "fp32" else 1)
+    out = {}
+    for cc in (1, 0):
+        rc, Q, R, stt = factor(h, A, prec, budget, colchunk=cc)
+        assert rc == 0 and stt["n_ooc_nodes"] >= 1 and stt["arena_bytes"] <= budget
+        if cc:
+            assert stt["n_colchunk_nodes"] >= 1, stt
+        else:
+            assert stt["n_colchunk_nodes"] == 0
+        Rg = R.astype(np.float64)
+        assert oracle.is_upper_triangular(Rg)
+        be = oracle.backward_error(X, gi.to_float64(Q, st), Rg)
+        re = oracle.r_rel_error(Rg, ref.R)
+        assert be < 5e-3 and re < 5e-3, (cc, be, re, stt)
+        out[cc] = Rg
+    h.set_option("colchunk", 1)
+    assert oracle.r_rel_error(out[1], out[0]) < 2e-3
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+def test_colchunk_node_dyadic_bitwise(h, prec):
+    """Exact-dyadic input through the column-chunked node: R == R0 and Q == H
+    bitwise, whatever the column split, the tail's host round trip and the chunked projections."""
+    st = STOR[prec]
+    m, n = 16384, 1024
+    A64, R0 = gi.dyadic_mixed(m, n, seed=9)
+    A = gi.to_storage(A64, st)
+    for budget_mib in (34, 40):
+        budget = budget_mib * MiB * (2 if st == "fp32" else 1)
+        rc, Q, R, stt = factor(h, A, prec, budget, colchunk=1)
+        assert rc == 0 and stt["n_colchunk_nodes"] >= 1, stt
+        np.testing.assert_array_equal(R.astype(np.float64), R0)
+        np.testing.assert_array_equal(gi.to_float64(Q, st), gi.hadamard(m, n))
+
+
+def test_colchunk_serialized_equals_overlapped(h):
+    """Race check of the column-chunked node: one stream (RGSQR_OPT_SERIALIZE) == overlapped, bitwise."""
+    A = gi.gaussian(16384, 1024, seed=33, dtype="fp16")
+    _, Q1, R1, s1 = factor(h, A, "fp16", 40 * MiB, colchunk=1, serialize=1)
+    _, Q2, R2, s2 = factor(h, A, "fp16", 40 * MiB, colchunk=1, serialize=0)
+    assert s1["n_colchunk_nodes"] >= 1 and s2["n_colchunk_nodes"] >= 1
+    np.testing.assert_array_equal(R1, R2)
+    np.testing.assert_array_equal(Q1, Q2)
