@@ -94,10 +94,12 @@ enum rgsqr_option {
                                    (rounded to 64).  50 = "divide evenly its columns into two halves"
                                    (PAPER.md:115), the default; other values are a scheduling ablation
                                    (same factorization in exact arithmetic).  In-core nodes always halve */
-  ,RGSQR_OPT_X3_CHAIN = 16      /* TF32X3 inner products: at most this many k-blocks (32 rows each, per
-                                   operand segment) accumulate in one tensor-core fp32 chain; longer K is
-                                   split and the partials summed in fixed order on the CUDA cores
-                                   (R25).  0 = the automatic one-wave split */
+  ,RGSQR_OPT_X3_CHAIN = 16      /* TF32X3 products: at most this many k-blocks (32 rows / columns each,
+                                   per operand segment) accumulate in one tensor-core fp32 chain in TMEM;
+                                   the chains are summed with round-to-nearest fp32 adds (registers for
+                                   the inner product, the shared-memory C tile for the outer product),
+                                   because the tensor core's accumulation error grows with the chain
+                                   length (R25).  Default 4; 0 = unbounded chains */
   ,RGSQR_OPT_COLCHUNK = 17      /* 1 = column-chunked out-of-core node (DAG lookahead across the OOC
                                    boundary; R26): when the left child is
                                    in-core and resident, A2 is uploaded in the column order the right
@@ -107,7 +109,10 @@ enum rgsqr_option {
                                    from the host and re-uploaded once Q1's memory is free.  0 = the
                                    row-tile streamed node.  Default 1 */
   ,RGSQR_OPT_EAGER_PCT = 18     /* column-chunked node: complete the Q1 projection when the right child's
-                                   leaves reach this percentage of its left half (default 75) */
+                                   leaves reach this percentage of its left half (default 50) */
+  ,RGSQR_OPT_CHUNK_MIB = 19     /* host path: MiB per column-chunk upload of an in-core or column-chunked
+                                   node (the granularity at which the recursion waits for its columns and
+                                   applies deferred products; >= 256 columns per product piece).  Default 32 */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

@@ -445,6 +445,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_X3_CHAIN: return &o.x3_chain;
     case RGSQR_OPT_COLCHUNK: return &o.colchunk;
     case RGSQR_OPT_EAGER_PCT: return &o.eager_pct;
+    case RGSQR_OPT_CHUNK_MIB: return &o.chunk_mib;
   }
   return nullptr;
 }
@@ -461,6 +462,9 @@ int rgsqr_set_option(rgsqr_handle h, int key, int64_t value) {
     case RGSQR_OPT_RING_DEPTH: if (value < 2 || value > 16) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_ALGO: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_REORTH: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_COLCHUNK: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_EAGER_PCT: if (value < 0 || value > 100) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_CHUNK_MIB: if (value < 1 || value > 1024) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_BLOCK_COLS: if (value < 8) return RGSQR_ERR_INVALID_ARG; break;
     default: if (value < 0) return RGSQR_ERR_INVALID_ARG;
   }

@@ -30,9 +30,10 @@ struct Options {
   int64_t prefetch = 1;      // OOC: upload the first ring tiles during the left child (RGSQR_OPT_PREFETCH)
   int64_t fuse_small = 1;    // fused kernel for nodes with w1, w2 <= 64 (RGSQR_OPT_FUSE_SMALL)
   int64_t split_pct = 50;    // OOC split: left child width in % (RGSQR_OPT_SPLIT_PCT; 50 = halves, the paper)
-  int64_t x3_chain = 0;      // TF32X3: max k-blocks per split-K chain (RGSQR_OPT_X3_CHAIN; 0 = one-wave rule)
+  int64_t x3_chain = 4;      // TF32X3: k-blocks per tensor-core accumulation chain (RGSQR_OPT_X3_CHAIN; 0 = unbounded)
   int64_t colchunk = 1;      // column-chunked OOC node (RGSQR_OPT_COLCHUNK, R26)
-  int64_t eager_pct = 75;    // column-chunked node: the external projection is completed once the right
+  int64_t chunk_mib = 32;    // host-path column upload chunk (RGSQR_OPT_CHUNK_MIB)
+  int64_t eager_pct = 50;    // column-chunked node: the external projection is completed once the right
                              // child's leaves reach this % of its left half (RGSQR_OPT_EAGER_PCT)
 };
 
@@ -175,9 +176,10 @@ struct ExtProduct {
   int64_t ldq = 0, w1 = 0;
   int64_t end = 0;                            // node columns [0, end) receive the product
   int64_t applied = 0;
-  float* R12[2] = {nullptr, nullptr};         // w1 x chunk fp32, alternating
+  int64_t piece = 0;                          // columns per application (0: the upload chunk)
+  float* R12[2] = {nullptr, nullptr};         // w1 x piece fp32, alternating (R12[1] may be null)
   cudaEvent_t free_ev[2] = {nullptr, nullptr};  // R12[i] may be overwritten after this event
-  void* R12op = nullptr;                      // w1 x chunk, operand type
+  void* R12op = nullptr;                      // w1 x piece, operand type
   int n_done = 0;
   std::function<cudaEvent_t(int64_t a, int64_t b, const float* R12)> r_out;  // download; event after it
   std::function<void()> done;                 // after the last chunk: Q1 is dead once sc gets there

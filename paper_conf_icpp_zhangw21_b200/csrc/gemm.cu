@@ -207,6 +207,156 @@ __global__ void __launch_bounds__(128, 1)
 }
 
 // ---------------------------------------------------------------------------------
+// Inner product with a bounded tensor-core accumulation chain (TF32X3, fp32 operands;
+// DESIGN.md R25).  The tcgen05 fp32 accumulation drops low bits at every add, so its error grows
+// linearly with the number of k-blocks summed in TMEM (measured: ~1.5e-7 relative per k-block,
+// profiles/r2_x3_chain_before_promotion.json).  Here the MMA warp accumulates units of
+// p.kb_per_unit k-blocks into one of TWO TMEM accumulators, and the epilogue warps fold every unit
+// into fp32 registers (round-to-nearest adds) while the next unit is being accumulated.
+// Warp roles (256 threads): 0 TMA, 1 MMA, 2 TMEM allocator, 4..7 accumulate + epilogue (warp w
+// owns TMEM lanes [32 (w-4), 32 (w-4) + 32)).  Output as gemm_kernel's TN epilogue.
+// ---------------------------------------------------------------------------------
+template <int BN>
+__global__ void __launch_bounds__(256, 1)
+    tn_promote_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                      const __grid_constant__ CUtensorMap mapA2, const __grid_constant__ CUtensorMap mapB2,
+                      const GemmParams p) {
+  using C = GemmCfg<float, false, BN>;
+  static_assert(2 * BN <= 512, "two accumulators must fit TMEM");
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = ptx::smem_u32(smem_raw);
+  uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;   // [2]
+  uint64_t* tempty = tfull + 2;          // [2]
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x >> 5;
+  const int64_t m0 = (int64_t)blockIdx.x * C::BM;
+  const int64_t n0 = (int64_t)blockIdx.y * BN;
+  const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;
+  const int64_t kb1 = min(p.kb_total, kb0 + p.kb_per_split);
+  const int nkb = kb1 > kb0 ? (int)(kb1 - kb0) : 0;
+  const int pk = p.kb_per_unit > 0 ? (int)p.kb_per_unit : max(nkb, 1);
+  const int nunits = nkb > 0 ? (nkb + pk - 1) / pk : 0;
+
+  if (warp == 0 && ptx::elect_one()) {
+    ptx::tma_prefetch_desc(&mapA);
+    ptx::tma_prefetch_desc(&mapB);
+    ptx::tma_prefetch_desc(&mapA2);
+    ptx::tma_prefetch_desc(&mapB2);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      ptx::mbar_init(&tfull[b], 1);
+      ptx::mbar_init(&tempty[b], 4);
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 2) ptx::tmem_alloc<2 * BN>(tslot);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0) {
+    if (ptx::elect_one()) {
+      for (int it = 0; it < nkb; ++it) {
+        const int s = it % C::STAGES;
+        const uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
+        ptx::mbar_wait(&empty[s], ph ^ 1u);
+        uint8_t* sA = smem + s * C::STAGE_BYTES;
+        uint8_t* sB = sA + C::A_BYTES;
+        int64_t kbg = kb0 + it;
+        int seg = 2;
+        if (p.kb_seg > 0) {
+          seg = (int)(kbg / p.kb_seg);
+          kbg -= (int64_t)seg * p.kb_seg;
+        }
+        const CUtensorMap* ta = seg == 1 ? &mapA2 : &mapA;
+        const CUtensorMap* tb = seg == 0 ? &mapB2 : &mapB;
+        const int32_t k0 = (int32_t)(kbg * C::BK);
+        ptx::mbar_arrive_expect_tx(&full[s], C::STAGE_BYTES);
+        ptx::tma_load_2d(sA, ta, &full[s], k0, (int32_t)m0);
+        ptx::tma_load_2d(sB, tb, &full[s], k0, (int32_t)n0);
+      }
+    }
+  } else if (warp == 1) {
+    if (ptx::elect_one()) {
+      int it = 0;
+      for (int u = 0; u < nunits; ++u) {
+        const int b = u & 1;
+        ptx::mbar_wait(&tempty[b], ((uint32_t)(u >> 1) & 1u) ^ 1u);
+        ptx::tc_fence_after();
+        const uint32_t acc = tmem + (uint32_t)(b * BN);
+        const int q1 = min(nkb, (u + 1) * pk);
+        for (; it < q1; ++it) {
+          const int s = it % C::STAGES;
+          ptx::mbar_wait(&full[s], (uint32_t)(it / C::STAGES) & 1u);
+          ptx::tc_fence_after();
+          const uint32_t aBase = ptx::smem_u32(smem + s * C::STAGE_BYTES);
+          const uint32_t bBase = aBase + C::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < C::BK / C::UK; ++kk) {
+            const uint64_t ad = ptx::sdesc_sw128(aBase + kk * C::UK * 4, 16, 1024);
+            const uint64_t bd = ptx::sdesc_sw128(bBase + kk * C::UK * 4, 16, 1024);
+            ptx::umma<true>(acc, ad, bd, C::IDESC, (it != u * pk || kk != 0) ? 1u : 0u);
+          }
+          ptx::umma_commit(&empty[s]);
+        }
+        ptx::umma_commit(&tfull[b]);
+      }
+    }
+  } else if (warp >= 4) {
+    const int ew = warp - 4, lane = threadIdx.x & 31;
+    float sum[BN];
+#pragma unroll
+    for (int j = 0; j < BN; ++j) sum[j] = 0.0f;
+    for (int u = 0; u < nunits; ++u) {
+      const int b = u & 1;
+      ptx::mbar_wait(&tfull[b], (uint32_t)(u >> 1) & 1u);
+      ptx::tc_fence_after();
+#pragma unroll
+      for (int cc = 0; cc < BN / 32; ++cc) {
+        uint32_t v[32];
+        ptx::tmem_ld_32x32b_x32(tmem + (uint32_t)(b * BN) + ((uint32_t)(ew * 32) << 16) + (uint32_t)(cc * 32), v);
+        ptx::tmem_ld_wait();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) sum[cc * 32 + j] += __uint_as_float(v[j]);
+      }
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&tempty[b]);
+    }
+    const int64_t i = m0 + ew * 32 + lane;
+    if (i < p.M) {
+#pragma unroll
+      for (int j = 0; j < BN; ++j) {
+        const int64_t n = n0 + j;
+        if (n < p.N) {
+          if (p.P != nullptr) {
+            p.P[blockIdx.z * p.split_stride + i + n * p.ldp] = sum[j];
+          } else {
+            const float y = p.accumulate ? p.C[i + n * p.ldc] + sum[j] : sum[j];
+            p.C[i + n * p.ldc] = y;
+            if (p.Cop != nullptr) reinterpret_cast<float*>(p.Cop)[i + n * p.ldop] = y;
+          }
+        }
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<2 * BN>(tmem);
+  }
+}
+
+// ---------------------------------------------------------------------------------
 // Deterministic split-K reduction: C = (accumulate ? C : 0) + sum_{s=0..S-1} P[s] in
 // a fixed order (no float atomics; R10), plus the optional operand copy.
 // ---------------------------------------------------------------------------------
@@ -280,6 +430,7 @@ __global__ void __launch_bounds__(256, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_tiles = p.tiles_m * p.tiles_n;
   const int nkb = (int)p.kb_total;
+  const int pk = p.promote_kb > 0 ? (int)p.promote_kb : max(nkb, 1);   // k-blocks per accumulation unit
 
   if (warp == 0 && ptx::elect_one()) {
     ptx::tma_prefetch_desc(&mapA);
@@ -333,31 +484,38 @@ __global__ void __launch_bounds__(256, 1)
     }
   } else if (warp == 1) {
     if (ptx::elect_one()) {
-      int it = 0, lt = 0;
-      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++lt) {
-        const int b = lt & 1;
-        ptx::mbar_wait(&tempty[b], ((uint32_t)(lt >> 1) & 1u) ^ 1u);
-        ptx::tc_fence_after();
-        const uint32_t acc = tmem + (uint32_t)(b * BN);
-        for (int kb = 0; kb < nkb; ++kb, ++it) {
-          const int s = it % C::STAGES;
-          ptx::mbar_wait(&full[s], (uint32_t)(it / C::STAGES) & 1u);
+      // accumulation units: a tile's K range in chains of `pk` k-blocks (p.promote_kb; the whole K
+      // when 0), alternating between the two TMEM accumulators; the epilogue folds each unit into
+      // the fp32 C tile in shared memory (RN), bounding the tensor core's accumulation chain
+      int it = 0, u = 0;
+      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+        for (int q0 = 0; q0 < nkb || q0 == 0; q0 += pk, ++u) {
+          const int b = u & 1;
+          ptx::mbar_wait(&tempty[b], ((uint32_t)(u >> 1) & 1u) ^ 1u);
           ptx::tc_fence_after();
-          const uint32_t aBase = ptx::smem_u32(smem + s * C::STAGE_BYTES);
-          const uint32_t bBase = aBase + C::A_BYTES;
+          const uint32_t acc = tmem + (uint32_t)(b * BN);
+          const int q1 = min(nkb, q0 + pk);
+          for (int kb = q0; kb < q1; ++kb, ++it) {
+            const int s = it % C::STAGES;
+            ptx::mbar_wait(&full[s], (uint32_t)(it / C::STAGES) & 1u);
+            ptx::tc_fence_after();
+            const uint32_t aBase = ptx::smem_u32(smem + s * C::STAGE_BYTES);
+            const uint32_t bBase = aBase + C::A_BYTES;
 #pragma unroll
-          for (int kk = 0; kk < C::BK / C::UK; ++kk) {
-            uint64_t ad;
-            if constexpr (Elem<T>::kTF32)
-              ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 512, 1);
-            else
-              ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 1024);
-            const uint64_t bd = ptx::sdesc_sw128(bBase + kk * C::UK * (int)sizeof(T), 16, 1024);
-            ptx::umma<Elem<T>::kTF32>(acc, ad, bd, C::IDESC, (kb | kk) != 0 ? 1u : 0u);
+            for (int kk = 0; kk < C::BK / C::UK; ++kk) {
+              uint64_t ad;
+              if constexpr (Elem<T>::kTF32)
+                ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 512, 1);
+              else
+                ad = ptx::sdesc_sw128(aBase + kk * C::UK * 128, C::BK * 128, 1024);
+              const uint64_t bd = ptx::sdesc_sw128(bBase + kk * C::UK * (int)sizeof(T), 16, 1024);
+              ptx::umma<Elem<T>::kTF32>(acc, ad, bd, C::IDESC, (kb != q0 || kk != 0) ? 1u : 0u);
+            }
+            ptx::umma_commit(&empty[s]);
           }
-          ptx::umma_commit(&empty[s]);
+          ptx::umma_commit(&tfull[b]);
+          if (nkb == 0) break;
         }
-        ptx::umma_commit(&tfull[b]);
       }
     }
   } else if (warp == 2) {
@@ -378,29 +536,32 @@ __global__ void __launch_bounds__(256, 1)
   } else if (warp >= 4) {
     const int ew = warp - 4;                 // == warp % 4: TMEM lanes [32 ew, 32 ew + 32)
     const int r = ew * 32 + lane;            // row within the tile
-    int lt = 0;
+    int lt = 0, u = 0;
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++lt) {
       const int32_t m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * BN;
-      const int b = lt & 1;
       const int cbuf = lt % C::C_BUFS;
       T* Cs = Cs0 + cbuf * (C::C_BYTES / (int)sizeof(T));
-      ptx::mbar_wait(&tfull[b], (uint32_t)(lt >> 1) & 1u);
-      ptx::tc_fence_after();
       ptx::mbar_wait(&cfull[cbuf], (uint32_t)(lt / C::C_BUFS) & 1u);
+      for (int q0 = 0; q0 < nkb || q0 == 0; q0 += pk, ++u) {
+        const int b = u & 1;
+        ptx::mbar_wait(&tfull[b], (uint32_t)(u >> 1) & 1u);
+        ptx::tc_fence_after();
 #pragma unroll 1
-      for (int cc = 0; cc < BN / 32; ++cc) {
-        uint32_t v[32];
-        ptx::tmem_ld_32x32b_x32(tmem + (uint32_t)(b * BN) + ((uint32_t)(ew * 32) << 16) + (uint32_t)(cc * 32), v);
-        ptx::tmem_ld_wait();
+        for (int cc = 0; cc < BN / 32; ++cc) {
+          uint32_t v[32];
+          ptx::tmem_ld_32x32b_x32(tmem + (uint32_t)(b * BN) + ((uint32_t)(ew * 32) << 16) + (uint32_t)(cc * 32), v);
+          ptx::tmem_ld_wait();
 #pragma unroll
-        for (int j = 0; j < 32; ++j) {
-          T* cp = Cs + (cc * 32 + j) * C::BM + r;
-          *cp = Elem<T>::store(Elem<T>::load(*cp) - __uint_as_float(v[j]));
+          for (int j = 0; j < 32; ++j) {
+            T* cp = Cs + (cc * 32 + j) * C::BM + r;
+            *cp = Elem<T>::store(Elem<T>::load(*cp) - __uint_as_float(v[j]));
+          }
         }
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&tempty[b]);
+        if (nkb == 0) break;
       }
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&tempty[b]);
       ptx::fence_proxy_async();              // generic smem writes -> visible to the TMA store
       ptx::named_bar_sync(1, 128);
       if (ew == 0 && lane == 0) {
@@ -478,12 +639,34 @@ static cudaError_t launch_gemm_t(const CUtensorMap& ma, const CUtensorMap& mb, c
   return cudaGetLastError();
 }
 
+template <int BN>
+static cudaError_t launch_tn_promote_t(const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& ma2,
+                                       const CUtensorMap& mb2, const GemmParams& p, int splits, cudaStream_t st) {
+  using C = GemmCfg<float, false, BN>;
+  constexpr int SMEM = C::SMEM + 64;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(tn_promote_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  dim3 grid((unsigned)((p.M + C::BM - 1) / C::BM), (unsigned)((p.N + BN - 1) / BN), (unsigned)splits);
+  tn_promote_kernel<BN><<<grid, 256, SMEM, st>>>(ma, mb, ma2, mb2, p);
+  return cudaGetLastError();
+}
+
 template <typename T>
 cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMap& mb,
                         const GemmParams& p, int splits, cudaStream_t st, const CUtensorMap* ma2,
                         const CUtensorMap* mb2) {
   const CUtensorMap& a2 = ma2 ? *ma2 : ma;
   const CUtensorMap& b2 = mb2 ? *mb2 : mb;
+  if constexpr (sizeof(T) == 4) {
+    if (!nn && p.kb_per_unit > 0) {   // bounded accumulation chain (TF32X3)
+      if (bn >= 128) return launch_tn_promote_t<128>(ma, mb, a2, b2, p, splits, st);
+      return launch_tn_promote_t<64>(ma, mb, a2, b2, p, splits, st);
+    }
+  }
   if (nn) {
     if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, a2, b2, p, splits, st);
     if (bn == 128) return launch_gemm_t<T, true, 128>(ma, mb, a2, b2, p, splits, st);

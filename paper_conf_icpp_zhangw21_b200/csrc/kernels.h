@@ -45,12 +45,16 @@ struct GemmParams {
   void* A2;
   int64_t lda2;
   int64_t kb_seg;           // > 0: K blocks per operand segment (TF32X3: hi.lo, lo.hi, hi.hi)
+  int64_t kb_per_unit;      // > 0 (fp32 TN only): k-blocks per tensor-core accumulation chain, the
+                            // chains summed in fp32 registers (tn_promote_kernel, R25)
 };
 
 struct NNParams {
   int tiles_m, tiles_n;     // 128-row x BN-column output tiles
   int64_t kb_total;         // K blocks (K = w1; 3 x that for the TF32X3 segments)
   int64_t kb_seg;           // > 0: K blocks per operand segment (TF32X3: hi.lo, lo.hi, hi.hi)
+  int64_t promote_kb;       // > 0: k-blocks per tensor-core accumulation chain, folded into the fp32
+                            // C tile in between (fp32 storage only; R25)
 };
 
 // TF32X3: ma2 / mb2 are the lo operands of A / B; segments (A, B lo), (A lo, B), (A, B)

@@ -172,6 +172,7 @@ struct Exec {
     int64_t late_col = -1;                                 // first column of the late chunk
     ExtProduct* ext = nullptr;
     int64_t eager_col = -1;   // leaf_done(col >= eager_col): apply the whole ext product now
+    size_t next0 = 0;         // chunks before this index were already awaited by the compute stream
   };
 
   int incore_node(int64_t c0, int64_t w, bool src_q, char* D, bool resident, cudaEvent_t* q_done,
@@ -181,7 +182,7 @@ struct Exec {
     if (!Rs) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core node: no space for R block");
     RGSQR_CUDA(c, cudaMemsetAsync(Rs, 0, (size_t)w * w * 4, sc));
     const int64_t leaf = std::max(1, leaf_width_for(c, m));
-    int64_t cw = ((int64_t)32 << 20) / std::max<int64_t>(1, m * s);
+    int64_t cw = (c->opt.chunk_mib << 20) / std::max<int64_t>(1, m * s);
     cw = std::max<int64_t>(leaf, cw / 64 * 64);
     std::vector<std::pair<int64_t, cudaEvent_t>> own;
     std::vector<std::pair<int64_t, cudaEvent_t>>& chunks = feed ? feed->chunks : own;
@@ -195,7 +196,7 @@ struct Exec {
         chunks.push_back({a, e});
       }
     }
-    size_t next = 0;
+    size_t next = feed ? feed->next0 : 0;
     int64_t flushed = 0;
     int err = 0;
     IncoreHooks hk;
@@ -567,17 +568,22 @@ struct Exec {
     int64_t wh = 0, wt1 = 0, wt2 = 0;
     size_t htop = 0;                 // bytes at the top of H used as scratch (left child, tail phase)
     int64_t ch = 0;                  // upload / product chunk width
+    int64_t E1 = 0;                  // head columns projected before the right child (phase A)
+    int64_t pB = 0;                  // piece width of the remaining projection (phase B)
   };
   bool plan_cc(int64_t w1, int64_t w2, size_t free0, CCPlan* P) const {
     if (w2 > w1 || (m * s * 64) % 256 != 0) return false;
     const int64_t leaf = std::max(1, leaf_width_for(c, m));
-    int64_t cw = ((int64_t)32 << 20) / std::max<int64_t>(1, m * s);
+    int64_t cw = (c->opt.chunk_mib << 20) / std::max<int64_t>(1, m * s);
     cw = std::max<int64_t>(leaf, cw / 64 * 64);
     const int64_t ch = cw * std::max<int64_t>(1, (256 + cw - 1) / cw);
     const size_t colb = (size_t)m * s, dB = (size_t)m * w1 * s;
     const size_t left_ws = incore_need(w1) - dB + 4096;
-    const size_t ext_b = 2 * ((size_t)w1 * ch * 4 + 256) + (size_t)w1 * ch * s + 256;
+    const int64_t hw = split_width(w2, leaf);
+    const int64_t pB = std::min<int64_t>(w2, 2 * ch);                 // phase-B piece (in X)
+    const size_t ext_b = (size_t)w1 * pB * (4 + s) + 512;
     const size_t right_ws = (size_t)w2 * w2 * 4 + 256 + incore_workspace_bytes(c, prec, m, w2) + ext_b + 16384;
+    const size_t rs1 = ((size_t)w1 * w1 * 4 + 255) / 256 * 256;
     for (int64_t wh = (w2 - 1) / 64 * 64; wh >= std::max<int64_t>(64, w2 / 4); wh -= 64) {
       const size_t H = colb * wh;
       if (H + dB + right_ws > free0) continue;
@@ -586,13 +592,18 @@ struct Exec {
       const int64_t wt1 = std::min<int64_t>(wt, (int64_t)(X / colb) / 8 * 8);
       const int64_t wt2 = wt - wt1;
       const size_t tail_ws = (size_t)w1 * wt * (4 + s) + 1024 + (size_t)wt2 * colb + 256;
-      const size_t htop = (std::max(left_ws, tail_ws) + 4095) / 4096 * 4096;
+      // phase A: the first E1 head columns projected in one piece before the right child starts
+      const int64_t E1 = std::min<int64_t>(wh, std::max<int64_t>(ch, (hw / 2) / ch * ch));
+      const size_t phaseA = (size_t)w1 * E1 * (4 + s) + 512;
+      const size_t htop = (std::max({left_ws, rs1 + tail_ws, phaseA}) + 4095) / 4096 * 4096;
       if (htop > H || wt > w1) continue;
       P->wh = wh;
       P->wt1 = wt1;
       P->wt2 = wt2;
       P->htop = htop;
       P->ch = ch;
+      P->E1 = E1;
+      P->pB = pB;
       return true;
     }
     return false;
@@ -650,29 +661,41 @@ struct Exec {
       if (rc < 0) return rc;
       ev_t1 = mark_ev(sh);
     }
+    // head chunks clear of H's top; the tail's second piece goes in after the first two (it waits for
+    // the left child, and a copy queued behind the whole head would arrive long after it is needed:
+    // uploads from all streams share the copy engine in submission order)
     Feed feed;
-    for (int64_t a = 0; a < htop_col; a += ch) {
-      const int64_t cols = std::min(ch, htop_col - a);
-      rc = h2d(H + a * colb, m, hsrc(src_q), 0, m, h + a, cols);
-      if (rc < 0) return rc;
+    auto head_chunk = [&](int64_t a, int64_t end) -> int {
+      int r = h2d(H + a * colb, m, hsrc(src_q), 0, m, h + a, end - a);
+      if (r < 0) return r;
       feed.chunks.push_back({a, mark_ev(sh)});
-    }
-    // ---- 2. the tail: its workspace and second piece in the top of H (free after the left child) ----
-    if (left_r) cudaStreamWaitEvent(sc, left_r, 0);
-    wsave = window(Htop, Hend);
+      return RGSQR_OK;
+    };
+    // ---- 2. the tail: workspace and second piece in the top of H, above the left R block (so that
+    //      nothing waits for that block's download) ----
+    wsave = window(Htop + ((size_t)w1 * w1 * 4 + 255) / 256 * 256, Hend);
     float* R12t = static_cast<float*>(c->arena.alloc((size_t)w1 * wt * 4));
     char* R12top = static_cast<char*>(c->arena.alloc((size_t)w1 * wt * s));
     char* T2 = wt2 > 0 ? static_cast<char*>(c->arena.alloc(colb * wt2)) : nullptr;
     unwindow(wsave);
     if (!R12t || !R12top || (wt2 > 0 && !T2))
       return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the tail products");
+    int64_t a_head = 0;
+    for (int k = 0; k < 2 && a_head < htop_col; ++k) {
+      const int64_t e = std::min(htop_col, a_head + ch);
+      if ((rc = head_chunk(a_head, e)) < 0) return rc;
+      a_head = e;
+    }
     if (wt2 > 0) {
-      // a second queue: this piece must not wait behind the head prefetch
-      cudaStreamWaitEvent(sh2, left_done, 0);
-      if (left_r) cudaStreamWaitEvent(sh2, left_r, 0);
-      rc = h2d(T2, m, hsrc(src_q), 0, m, h + wh + wt1, wt2, sh2);
+      cudaStreamWaitEvent(sh, left_done, 0);
+      rc = h2d(T2, m, hsrc(src_q), 0, m, h + wh + wt1, wt2);
       if (rc < 0) return rc;
-      ev_t2 = mark_ev(sh2);
+      ev_t2 = mark_ev(sh);
+    }
+    for (; a_head < htop_col;) {
+      const int64_t e = std::min(htop_col, a_head + ch);
+      if ((rc = head_chunk(a_head, e)) < 0) return rc;
+      a_head = e;
     }
     cudaEvent_t a_seg = seg_begin(sc);
     struct Piece { char* T; int64_t col, w; cudaEvent_t ev; };
@@ -691,7 +714,6 @@ struct Exec {
       rc = op_outer(c, prec, D, m, R12top + pc.col * w1 * s, w1, pc.T, m, m, w1, pc.w, sc);
       if (rc < 0) return rc;
     }
-    seg_end(2, sc, a_seg);
     wait(sd, sc);
     for (const Piece& pc : pieces) {
       if (pc.w == 0) continue;
@@ -699,37 +721,65 @@ struct Exec {
       if (rc < 0) return rc;
     }
     cudaEvent_t tail_out = mark_ev(sd);
-    cudaEvent_t tail_done = mark_ev(sc);
-    // the rest of the head goes into H's top once the tail phase has released it
-    cudaStreamWaitEvent(sh, tail_done, 0);
-    cudaStreamWaitEvent(sh, tail_out, 0);
-    if (r12t_out) cudaStreamWaitEvent(sh, r12t_out, 0);
-    for (int64_t a = htop_col; a < wh;) {
-      const int64_t end = std::min(wh, (a / ch + 1) * ch);
-      rc = h2d(H + a * colb, m, hsrc(src_q), 0, m, h + a, end - a);
-      if (rc < 0) return rc;
-      feed.chunks.push_back({a, mark_ev(sh)});
-      a = end;
-    }
-    // ---- 3. the right child, with the head's Q1 projection applied as its columns are reached ----
-    cudaStreamWaitEvent(sc, tail_out, 0);          // X (T1) becomes the right child's workspace
-    c->arena.release(T1 ? (size_t)(T1 - c->arena.base) : x_mark);
+    // ---- phase A: the first E1 head columns' projection in one piece (buffers at the bottom of H's
+    //      top, once the left R block is downloaded), while the tail goes out ----
     ExtProduct ext;
     ext.Q1 = D;
     ext.ldq = m;
     ext.w1 = w1;
     ext.end = wh;
-    ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * ch * 4));
-    ext.R12[1] = static_cast<float*>(c->arena.alloc((size_t)w1 * ch * 4));
-    ext.R12op = c->arena.alloc((size_t)w1 * ch * s);
-    if (!ext.R12[0] || !ext.R12[1] || !ext.R12op)
-      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the projection chunks");
     ext.r_out = [&](int64_t a, int64_t b, const float* R12) -> cudaEvent_t {
       if (d2h_r(c0, h + a, w1, b - a, R12, w1) < 0) return nullptr;
       return r_done;
     };
+    size_t waited = 0;
+    IncoreHooks hkA;
+    hkA.chunk = ch;
+    hkA.ext = &ext;
+    hkA.need = [&](int64_t col_end) {
+      while (waited < feed.chunks.size() && feed.chunks[waited].first < col_end)
+        cudaStreamWaitEvent(sc, feed.chunks[waited++].second, 0);
+    };
+    const int64_t E1 = std::min<int64_t>(P.E1, htop_col / ch * ch);   // (its columns must be uploaded)
+    if (E1 > 0) {
+      if (left_r) cudaStreamWaitEvent(sc, left_r, 0);
+      wsave = window(Htop, Hend);
+      ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * E1 * 4));
+      ext.R12op = c->arena.alloc((size_t)w1 * E1 * s);
+      unwindow(wsave);
+      if (!ext.R12[0] || !ext.R12op)
+        return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the first projection");
+      ext.piece = E1;
+      rc = apply_ext(c, prec, H, m, m, &hkA, E1, sc);
+      if (rc < 0) return rc;
+    }
+    seg_end(2, sc, a_seg);
+    cudaEvent_t phaseA_done = mark_ev(sc);
+    cudaEvent_t phaseA_r = ext.free_ev[0];
+    // the rest of the head goes into H's top once the tail phase and phase A have released it
+    cudaStreamWaitEvent(sh, phaseA_done, 0);
+    cudaStreamWaitEvent(sh, tail_out, 0);
+    if (r12t_out) cudaStreamWaitEvent(sh, r12t_out, 0);
+    if (phaseA_r) cudaStreamWaitEvent(sh, phaseA_r, 0);
+    for (int64_t a = htop_col; a < wh;) {
+      const int64_t end = std::min(wh, (a / ch + 1) * ch);
+      if ((rc = head_chunk(a, end)) < 0) return rc;
+      a = end;
+    }
+    // ---- 3. the right child, with the rest of the head's projection applied as its columns are
+    //      reached and completed eagerly part-way through ----
+    cudaStreamWaitEvent(sc, tail_out, 0);          // X (T1) becomes the right child's workspace
+    c->arena.release(T1 ? (size_t)(T1 - c->arena.base) : x_mark);
+    ext.piece = P.pB;
+    ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * P.pB * 4));
+    ext.R12[1] = nullptr;
+    ext.R12op = c->arena.alloc((size_t)w1 * P.pB * s);
+    ext.free_ev[0] = ext.free_ev[1] = nullptr;
+    if (!ext.R12[0] || !ext.R12op)
+      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the projection pieces");
     feed.late_col = wh;
     feed.chunks.push_back({wh, nullptr});
+    feed.next0 = waited;
     ext.done = [&]() {
       // Q1 is dead once the compute stream gets here: the tail goes into D's first columns
       cudaEvent_t q1_dead = mark_ev(sc);

@@ -152,7 +152,8 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
                          int accumulate, cudaStream_t st, const void* Q1lo, const void* A2lo) {
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
-  const int bn = pick_bn(w2);
+  const bool promote = Q1lo != nullptr && A2lo != nullptr && c->opt.x3_chain > 0;
+  const int bn = promote ? std::min(pick_bn(w2), 128) : pick_bn(w2);   // (register accumulators)
   CUtensorMap ma, mb, ma2, mb2;
   std::string err;
   if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, BK, 128, &err) ||
@@ -176,10 +177,9 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
   // doubled the kernel time: 57 vs 37 us, profiles/r1_splitk_scan.txt).
   int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : c->num_sms / tiles);
   splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.kb_total / 4));
-  // TF32X3: bound the tensor-core accumulation chain (RGSQR_OPT_X3_CHAIN k-blocks per split):
-  // its fp32 accumulator error grows with the chain length, the fixed-order split-K sum is RN
-  if (x3 && c->opt.splitk <= 0 && c->opt.x3_chain > 0)
-    splits = std::max<int64_t>(splits, (p.kb_total + c->opt.x3_chain - 1) / c->opt.x3_chain);
+  // TF32X3: the tensor-core accumulation chain is bounded in-kernel (RGSQR_OPT_X3_CHAIN k-blocks per
+  // TMEM chain, the chains summed in fp32 registers: tn_promote_kernel, R25)
+  if (x3) p.kb_per_unit = c->opt.x3_chain;
   const size_t cap = std::min<size_t>((size_t)64 << 20, c->arena.free_bytes());
   while (splits > 1 && (size_t)splits * w1 * w2 * 4 + 256 > cap) --splits;
   p.kb_per_split = (p.kb_total + splits - 1) / splits;
@@ -244,6 +244,7 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   if (x3) {   // TF32X3: k-blocks of (Q1, R12 lo), (Q1 lo, R12), (Q1, R12) into one accumulator
     p.kb_seg = p.kb_total;
     p.kb_total *= 3;
+    p.promote_kb = c->opt.x3_chain;   // chains folded into the fp32 C tile (R25)
   }
   const int grid = (int)std::min<int64_t>((int64_t)p.tiles_m * p.tiles_n, c->num_sms);
   cudaEvent_t kb = c->kbegin(st);
@@ -580,11 +581,11 @@ int apply_ext(Ctx* c, int prec, char* A, int64_t lda, int64_t m, IncoreHooks* hk
   if (!e) return RGSQR_OK;
   const int64_t s = elem_bytes(prec);
   upto = std::min(upto, e->end);
-  const int64_t ch = std::max<int64_t>(hk->chunk, 64);
+  const int64_t ch = e->piece > 0 ? e->piece : std::max<int64_t>(hk->chunk, 64);
   while (e->applied < upto) {
-    const int64_t a = e->applied, b = std::min(e->end, (a / ch + 1) * ch);
+    const int64_t a = e->applied, b = std::min(e->end, a + ch);
     hk->need(b);
-    const int slot = e->n_done & 1;
+    const int slot = e->R12[1] ? (e->n_done & 1) : 0;
     if (e->free_ev[slot]) cudaStreamWaitEvent(st, e->free_ev[slot], 0);
     char* A2 = A + a * lda * s;
     int rc = op_inner(c, prec, e->Q1, e->ldq, A2, lda, m, e->w1, b - a, e->R12[slot], e->w1, e->R12op, e->w1, 0, st);

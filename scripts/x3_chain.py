@@ -16,12 +16,12 @@ from tests.gpu_util import to_dev, from_dev  # noqa: E402
 
 h = Handle(0)
 out = []
-for (m, n) in [(8192, 256), (65536, 256)]:
+for (m, n) in [(8192, 256), (65536, 256), (65536, 2048)]:
     A64, _ = gi.usv(m, n, kappa=1e3, seed=3)
     A = gi.to_storage(A64, "fp32")
     X = gi.to_float64(A, "fp32")
     ref = oracle.gram_cholesky_r(X)
-    for splitk, chain in [(0, 0), (1, 0), (2, 0), (4, 0), (8, 0), (16, 0), (32, 0), (0, 48), (0, 24), (0, 12), (0, 6)]:
+    for splitk, chain in [(0, 0), (0, 16), (0, 8), (0, 4), (0, 2), (1, 4), (4, 4), (16, 4), (1, 0)]:
         h.set_option("splitk", splitk)
         h.set_option("x3_chain", chain)
         Ad = to_dev(A, "fp32")
@@ -34,6 +34,26 @@ for (m, n) in [(8192, 256), (65536, 256)]:
         out.append(rec)
         print(json.dumps(rec), flush=True)
 h.set_option("splitk", 0)
-h.set_option("x3_chain", 0)
+h.set_option("x3_chain", 4)
+# throughput of the TF32X3 device path at configs[1]'s shape (fp32 storage), chains bounded vs not
+A = gi.gaussian(65536, 8192, seed=2, dtype="fp32")
+Ad = to_dev(A, "fp32")
+Qd = torch.empty_like(Ad)
+R = torch.empty((8192, 8192), dtype=torch.float32, device="cuda")
+for chain in (4, 0):
+    h.set_option("x3_chain", chain)
+    h.factor_device(Ad, 65536, 65536, 8192, Qd, R, precision="tf32x3")
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(3):
+        h.factor_device(Ad, 65536, 65536, 8192, Qd, R, precision="tf32x3")
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / 3
+    rec = {"m": 65536, "n": 8192, "x3_chain": chain, "ms": ms, "tflops": 2 * 65536 * 8192 ** 2 / ms / 1e9}
+    out.append(rec)
+    print(json.dumps(rec), flush=True)
+h.set_option("x3_chain", 4)
 os.makedirs("gpurun_out", exist_ok=True)
 json.dump(out, open("gpurun_out/x3_chain.json", "w"), indent=1)

@@ -201,7 +201,9 @@ def test_colchunk_node_vs_streamed_node(h, prec, budget_mib):
     budget = budget_mib * MiB * (2 if st == "fp32" else 1)
     out = {}
     for cc in (1, 0):
-        rc, Q, R, stt = factor(h, A, prec, budget, colchunk=cc)
+        # 2 MiB upload chunks: 64-column pieces at this height, so the first-projection phase
+        # and the chunked pieces of the column-chunked node all occur (32 MiB would be 1 chunk)
+        rc, Q, R, stt = factor(h, A, prec, budget, colchunk=cc, chunk_mib=2)
         assert rc == 0 and stt["n_ooc_nodes"] >= 1 and stt["arena_bytes"] <= budget
         if cc:
             assert stt["n_colchunk_nodes"] >= 1, stt
@@ -214,6 +216,7 @@ def test_colchunk_node_vs_streamed_node(h, prec, budget_mib):
         assert be < 5e-3 and re < 5e-3, (cc, be, re, stt)
         out[cc] = Rg
     h.set_option("colchunk", 1)
+    h.set_option("chunk_mib", 32)
     assert oracle.r_rel_error(out[1], out[0]) < 2e-3
 
 
@@ -225,19 +228,21 @@ def test_colchunk_node_dyadic_bitwise(h, prec):
     m, n = 16384, 1024
     A64, R0 = gi.dyadic_mixed(m, n, seed=9)
     A = gi.to_storage(A64, st)
-    for budget_mib in (34, 40):
+    for budget_mib, chunk in ((34, 32), (40, 2), (38, 1)):
         budget = budget_mib * MiB * (2 if st == "fp32" else 1)
-        rc, Q, R, stt = factor(h, A, prec, budget, colchunk=1)
+        rc, Q, R, stt = factor(h, A, prec, budget, colchunk=1, chunk_mib=chunk)
         assert rc == 0 and stt["n_colchunk_nodes"] >= 1, stt
         np.testing.assert_array_equal(R.astype(np.float64), R0)
         np.testing.assert_array_equal(gi.to_float64(Q, st), gi.hadamard(m, n))
+    h.set_option("chunk_mib", 32)
 
 
 def test_colchunk_serialized_equals_overlapped(h):
     """Race check of the column-chunked node: one stream (RGSQR_OPT_SERIALIZE) == overlapped, bitwise."""
     A = gi.gaussian(16384, 1024, seed=33, dtype="fp16")
-    _, Q1, R1, s1 = factor(h, A, "fp16", 40 * MiB, colchunk=1, serialize=1)
-    _, Q2, R2, s2 = factor(h, A, "fp16", 40 * MiB, colchunk=1, serialize=0)
+    _, Q1, R1, s1 = factor(h, A, "fp16", 40 * MiB, colchunk=1, serialize=1, chunk_mib=2)
+    _, Q2, R2, s2 = factor(h, A, "fp16", 40 * MiB, colchunk=1, serialize=0, chunk_mib=2)
+    h.set_option("chunk_mib", 32)
     assert s1["n_colchunk_nodes"] >= 1 and s2["n_colchunk_nodes"] >= 1
     np.testing.assert_array_equal(R1, R2)
     np.testing.assert_array_equal(Q1, Q2)
