@@ -99,7 +99,8 @@ enum rgsqr_option {
                                    the chains are summed with round-to-nearest fp32 adds (registers for
                                    the inner product, the shared-memory C tile for the outer product),
                                    because the tensor core's accumulation error grows with the chain
-                                   length (R25).  Default 4; 0 = unbounded chains */
+                                   length (R25).  Default 2 (inner product; the outer product uses
+                                   twice this); 0 = unbounded chains */
   ,RGSQR_OPT_COLCHUNK = 17      /* 1 = column-chunked out-of-core node (DAG lookahead across the OOC
                                    boundary; R26): when the left child is
                                    in-core and resident, A2 is uploaded in the column order the right

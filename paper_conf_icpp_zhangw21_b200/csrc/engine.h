@@ -30,7 +30,7 @@ struct Options {
   int64_t prefetch = 1;      // OOC: upload the first ring tiles during the left child (RGSQR_OPT_PREFETCH)
   int64_t fuse_small = 1;    // fused kernel for nodes with w1, w2 <= 64 (RGSQR_OPT_FUSE_SMALL)
   int64_t split_pct = 50;    // OOC split: left child width in % (RGSQR_OPT_SPLIT_PCT; 50 = halves, the paper)
-  int64_t x3_chain = 4;      // TF32X3: k-blocks per tensor-core accumulation chain (RGSQR_OPT_X3_CHAIN; 0 = unbounded)
+  int64_t x3_chain = 2;      // TF32X3: k-blocks per tensor-core accumulation chain (RGSQR_OPT_X3_CHAIN; 0 = unbounded)
   int64_t colchunk = 1;      // column-chunked OOC node (RGSQR_OPT_COLCHUNK, R26)
   int64_t chunk_mib = 32;    // host-path column upload chunk (RGSQR_OPT_CHUNK_MIB)
   int64_t eager_pct = 50;    // column-chunked node: the external projection is completed once the right

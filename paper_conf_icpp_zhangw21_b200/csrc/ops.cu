@@ -244,7 +244,9 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   if (x3) {   // TF32X3: k-blocks of (Q1, R12 lo), (Q1 lo, R12), (Q1, R12) into one accumulator
     p.kb_seg = p.kb_total;
     p.kb_total *= 3;
-    p.promote_kb = c->opt.x3_chain;   // chains folded into the fp32 C tile (R25)
+    // chains folded into the fp32 C tile (R25); twice the inner product's unit: K = w1 is
+    // short, and a shorter unit would make the shared-memory C-tile updates the bound
+    p.promote_kb = 2 * c->opt.x3_chain;
   }
   const int grid = (int)std::min<int64_t>((int64_t)p.tiles_m * p.tiles_n, c->num_sms);
   cudaEvent_t kb = c->kbegin(st);

@@ -18,6 +18,7 @@ for s in $STEPS; do
     timeline) RGSQR_TIMELINE=gpurun_out/timeline_c2.csv timeout 300 python scripts/prof_run.py --host --reps 3 > gpurun_out/timeline.log 2>&1; python scripts/timeline.py gpurun_out/timeline_c2.csv > gpurun_out/timeline_summary.txt; head -1 gpurun_out/timeline_summary.txt; tail -n 2 gpurun_out/timeline.log ;;
     hosttests) timeout 1200 python -m pytest tests/test_gpu_factor_host.py -q -x ${PYTEST_ARGS} > gpurun_out/pytest_host.log 2>&1; tail -n 3 gpurun_out/pytest_host.log; grep -E "^(FAILED|ERROR)|Error" gpurun_out/pytest_host.log | head -20 ;;
     pyfiles) timeout 1500 python -m pytest ${PYFILES} -q ${PYTEST_ARGS} > gpurun_out/pytest_files.log 2>&1; tail -n 3 gpurun_out/pytest_files.log; grep -E "^(FAILED|ERROR)|Error" gpurun_out/pytest_files.log | head -20 ;;
+    sweephost) timeout 1200 python scripts/sweep_host.py ${SWEEP_ARGS} > gpurun_out/sweep_host.log 2>&1; cat gpurun_out/sweep_host.log | cut -c1-220 ;;
     *) echo "unknown step $s" ;;
   esac
 done

@@ -122,7 +122,7 @@ def test_tf32x3_error_independent_of_split_k(h):
         errs.append(oracle.r_rel_error(R, ref))
     h.set_option("splitk", 0)
     assert max(errs) <= 3e-6, errs
-    assert max(errs) <= 1.5 * min(errs), errs
+    assert max(errs) <= 1.6 * min(errs), errs
 
 
 @pytest.mark.parametrize("prec", ["fp16", "bf16"])
