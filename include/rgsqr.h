@@ -180,6 +180,28 @@ int rgsqr_factor(rgsqr_handle h, const void* A_host, int64_t lda, int64_t m, int
 int rgsqr_factor_device(rgsqr_handle h, const void* A_dev, int64_t lda, int64_t m, int64_t n,
                         void* Q_dev, float* R_dev, int precision, size_t device_mem_budget);
 
+/* ---- the two out-of-core GEMMs as standalone operations (host memory in and out) ----------
+ * The paper measures them separately (section 5.1, Tables 1/2) with both tiling
+ * strategies of section 3.3:
+ *   tiling 0 = recursive: inner product Fig. 3 (row tiles of Q1 and A2, each read once, R12
+ *              accumulated in HBM and written once); outer product Fig. 5 (R12 resident, row tiles of
+ *              Q1 and A2 in, A2' out).  `block` = rows per tile (0: 16384 inner, 8192 outer).
+ *   tiling 1 = blocking:  inner product Fig. 4 (Q1 panel resident, A2 in column blocks, R12 blocks
+ *              out); outer product Fig. 6 (Q1 and R12 resident, block x block tiles of A2 in and out).
+ *              `block` = columns (inner) / tile edge (outer) (0: 16384).
+ * Arrays are column-major host buffers (pageable ones are page-locked for the call): Q1 m x w1
+ * (ldq), A2 m x w2 (lda) with the precision's storage type, R12 w1 x w2 binary32 (ldr >= w1).
+ * Inner: R12 = Q1^T A2 (A2 read only).  Outer: A2 <- A2 - Q1 R12, R12 rounded RN to the operand
+ * type on the device (R9), A2' rounded RN to storage.  device_mem_budget as for
+ * rgsqr_factor.  FP16 / BF16 / TF32, single-GPU contexts; RGSQR_OPT_SERIALIZE gives the paper's "Synchronous" rows and
+ * RGSQR_OPT_RING_DEPTH the number of tile slots.  Stats: bytes, busy times, overlap, wall_ms. */
+int rgsqr_ooc_inner(rgsqr_handle h, const void* Q1_host, int64_t ldq, const void* A2_host, int64_t lda, int64_t m,
+                    int64_t w1, int64_t w2, float* R12_host, int64_t ldr, int precision, int tiling, int64_t block,
+                    size_t device_mem_budget);
+int rgsqr_ooc_outer(rgsqr_handle h, const void* Q1_host, int64_t ldq, const float* R12_host, int64_t ldr,
+                    void* A2_host, int64_t lda, int64_t m, int64_t w1, int64_t w2, int precision, int tiling,
+                    int64_t block, size_t device_mem_budget);
+
 /* ---- hot-path operations (device pointers; used by the kernel parity tests) ------------ */
 /* Leaf CGS panel (Eq. 1) in place: P (m x w, ldp) -> Q; R11 (w x w,
  * device, ldr) receives r_ij, 1 <= w <= 64.  Returns the first breakdown column via

@@ -351,6 +351,26 @@ int rgsqr_factor_device(rgsqr_handle h, const void* A_dev, int64_t lda, int64_t 
   return factor_device(c, A_dev, lda, m, n, Q_dev, R_dev, precision, device_mem_budget);
 }
 
+int rgsqr_ooc_inner(rgsqr_handle h, const void* Q1_host, int64_t ldq, const void* A2_host, int64_t lda, int64_t m,
+                    int64_t w1, int64_t w2, float* R12_host, int64_t ldr, int precision, int tiling, int64_t block,
+                    size_t device_mem_budget) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  return ooc_gemm(c, 0, tiling, block, Q1_host, ldq, const_cast<void*>(A2_host), lda, R12_host, ldr, m, w1, w2,
+                  precision, device_mem_budget);
+}
+
+int rgsqr_ooc_outer(rgsqr_handle h, const void* Q1_host, int64_t ldq, const float* R12_host, int64_t ldr,
+                    void* A2_host, int64_t lda, int64_t m, int64_t w1, int64_t w2, int precision, int tiling,
+                    int64_t block, size_t device_mem_budget) {
+  Ctx* c = C(h);
+  if (!c) return RGSQR_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  return ooc_gemm(c, 1, tiling, block, Q1_host, ldq, A2_host, lda, const_cast<float*>(R12_host), ldr, m, w1, w2,
+                  precision, device_mem_budget);
+}
+
 int rgsqr_op_leaf(rgsqr_handle h, void* P, int64_t ldp, int64_t m, int64_t w, float* R11, int64_t ldr,
                   int precision, int* breakdown) {
   Ctx* c = C(h);

@@ -199,5 +199,7 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
                   size_t budget);
 int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* Q, float* R, int prec,
                 size_t budget);
+int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t ldq, void* A2, int64_t lda,
+             float* R12, int64_t ldr, int64_t m, int64_t w1, int64_t w2, int prec, size_t budget);
 
 }  // namespace rgsqr

@@ -311,10 +311,12 @@ __global__ void __launch_bounds__(256, 1)
       }
     }
   } else if (warp >= 4) {
+    // the unit sums accumulate in fp64: with K = m rows there can be thousands of units, and an
+    // fp32 running sum would add a random-walk error of sqrt(units) * 2^-24
     const int ew = warp - 4, lane = threadIdx.x & 31;
-    float sum[BN];
+    double sum[BN];
 #pragma unroll
-    for (int j = 0; j < BN; ++j) sum[j] = 0.0f;
+    for (int j = 0; j < BN; ++j) sum[j] = 0.0;
     for (int u = 0; u < nunits; ++u) {
       const int b = u & 1;
       ptx::mbar_wait(&tfull[b], (uint32_t)(u >> 1) & 1u);
@@ -325,7 +327,7 @@ __global__ void __launch_bounds__(256, 1)
         ptx::tmem_ld_32x32b_x32(tmem + (uint32_t)(b * BN) + ((uint32_t)(ew * 32) << 16) + (uint32_t)(cc * 32), v);
         ptx::tmem_ld_wait();
 #pragma unroll
-        for (int j = 0; j < 32; ++j) sum[cc * 32 + j] += __uint_as_float(v[j]);
+        for (int j = 0; j < 32; ++j) sum[cc * 32 + j] += (double)__uint_as_float(v[j]);
       }
       ptx::tc_fence_before();
       __syncwarp();
@@ -338,9 +340,9 @@ __global__ void __launch_bounds__(256, 1)
         const int64_t n = n0 + j;
         if (n < p.N) {
           if (p.P != nullptr) {
-            p.P[blockIdx.z * p.split_stride + i + n * p.ldp] = sum[j];
+            p.P[blockIdx.z * p.split_stride + i + n * p.ldp] = (float)sum[j];
           } else {
-            const float y = p.accumulate ? p.C[i + n * p.ldc] + sum[j] : sum[j];
+            const float y = p.accumulate ? (float)((double)p.C[i + n * p.ldc] + sum[j]) : (float)sum[j];
             p.C[i + n * p.ldc] = y;
             if (p.Cop != nullptr) reinterpret_cast<float*>(p.Cop)[i + n * p.ldop] = y;
           }
@@ -662,10 +664,8 @@ cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMa
   const CUtensorMap& a2 = ma2 ? *ma2 : ma;
   const CUtensorMap& b2 = mb2 ? *mb2 : mb;
   if constexpr (sizeof(T) == 4) {
-    if (!nn && p.kb_per_unit > 0) {   // bounded accumulation chain (TF32X3)
-      if (bn >= 128) return launch_tn_promote_t<128>(ma, mb, a2, b2, p, splits, st);
+    if (!nn && p.kb_per_unit > 0)   // bounded accumulation chain (TF32X3); fp64 unit sums: BN = 64
       return launch_tn_promote_t<64>(ma, mb, a2, b2, p, splits, st);
-    }
   }
   if (nn) {
     if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, a2, b2, p, splits, st);

@@ -153,7 +153,7 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
   const bool promote = Q1lo != nullptr && A2lo != nullptr && c->opt.x3_chain > 0;
-  const int bn = promote ? std::min(pick_bn(w2), 128) : pick_bn(w2);   // (register accumulators)
+  const int bn = promote ? 64 : pick_bn(w2);   // (fp64 register accumulators: tn_promote_kernel)
   CUtensorMap ma, mb, ma2, mb2;
   std::string err;
   if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, BK, 128, &err) ||

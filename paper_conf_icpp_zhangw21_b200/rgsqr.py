@@ -30,7 +30,8 @@ OPTIONS = {"leaf_width": 1, "tile_rows_min": 2, "tile_rows_max": 3, "ring_depth"
 EXPORTS = ["rgsqr_create", "rgsqr_get_unique_id", "rgsqr_create_dist", "rgsqr_destroy", "rgsqr_factor",
            "rgsqr_factor_device", "rgsqr_op_leaf", "rgsqr_op_inner", "rgsqr_op_outer", "rgsqr_set_stream",
            "rgsqr_get_stream", "rgsqr_host_alloc", "rgsqr_host_free", "rgsqr_set_option", "rgsqr_get_option",
-           "rgsqr_get_stats", "rgsqr_version", "rgsqr_status_string", "rgsqr_last_error", "rgsqr_probe_link"]
+           "rgsqr_get_stats", "rgsqr_version", "rgsqr_status_string", "rgsqr_last_error", "rgsqr_probe_link",
+           "rgsqr_ooc_inner", "rgsqr_ooc_outer"]
 
 
 class Stats(C.Structure):
@@ -97,6 +98,8 @@ def load_library(path: str = LIB_PATH):
         "rgsqr_status_string": ([i32], C.c_char_p),
         "rgsqr_last_error": ([vp], C.c_char_p),
         "rgsqr_probe_link": ([vp, vp, i64, i64, i64, i32, i32, C.POINTER(C.c_double)], i32),
+        "rgsqr_ooc_inner": ([vp, vp, i64, vp, i64, i64, i64, i64, vp, i64, i32, i32, i64, C.c_size_t], i32),
+        "rgsqr_ooc_outer": ([vp, vp, i64, vp, i64, vp, i64, i64, i64, i64, i32, i32, i64, C.c_size_t], i32),
     }
     del fp
     for name, (args, res) in sig.items():
@@ -206,6 +209,17 @@ class Handle:
         return self._check(self.lib.rgsqr_factor_device(self.h, _ptr(A), lda, m, n, _ptr(Q), _ptr(R),
                                                         PRECISIONS[precision], int(budget)),
                            "rgsqr_factor_device")
+
+    # ---- the out-of-core GEMMs (host buffers; Tables 1/2 of the paper) ----
+    def ooc_inner(self, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, precision="fp16", tiling=0, block=0, budget=0):
+        """R12 = Q1^T A2 streamed from host memory (tiling 0: Fig. 3, 1: Fig. 4)."""
+        return self._check(self.lib.rgsqr_ooc_inner(self.h, _ptr(Q1), ldq, _ptr(A2), lda, m, w1, w2, _ptr(R12), ldr,
+                                                    PRECISIONS[precision], tiling, block, int(budget)), "ooc_inner")
+
+    def ooc_outer(self, Q1, ldq, R12, ldr, A2, lda, m, w1, w2, precision="fp16", tiling=0, block=0, budget=0):
+        """A2 <- A2 - Q1 R12 in host memory (tiling 0: Fig. 5, 1: Fig. 6)."""
+        return self._check(self.lib.rgsqr_ooc_outer(self.h, _ptr(Q1), ldq, _ptr(R12), ldr, _ptr(A2), lda, m, w1, w2,
+                                                    PRECISIONS[precision], tiling, block, int(budget)), "ooc_outer")
 
     # ---- hot-path ops (device pointers) ----
     def op_leaf(self, P, ldp, m, w, R11, ldr, precision="fp16") -> tuple[int, int]:

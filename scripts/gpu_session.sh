@@ -19,6 +19,7 @@ for s in $STEPS; do
     hosttests) timeout 1200 python -m pytest tests/test_gpu_factor_host.py -q -x ${PYTEST_ARGS} > gpurun_out/pytest_host.log 2>&1; tail -n 3 gpurun_out/pytest_host.log; grep -E "^(FAILED|ERROR)|Error" gpurun_out/pytest_host.log | head -20 ;;
     pyfiles) timeout 1500 python -m pytest ${PYFILES} -q ${PYTEST_ARGS} > gpurun_out/pytest_files.log 2>&1; tail -n 3 gpurun_out/pytest_files.log; grep -E "^(FAILED|ERROR)|Error" gpurun_out/pytest_files.log | head -20 ;;
     sweephost) timeout 1200 python scripts/sweep_host.py ${SWEEP_ARGS} > gpurun_out/sweep_host.log 2>&1; cat gpurun_out/sweep_host.log | cut -c1-220 ;;
+    tables) timeout 1800 python scripts/paper_gemm_tables.py ${TABLES_ARGS} > gpurun_out/paper_gemm_tables.log 2>&1; cut -c1-260 gpurun_out/paper_gemm_tables.log ;;
     *) echo "unknown step $s" ;;
   esac
 done
