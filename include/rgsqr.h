@@ -114,6 +114,12 @@ enum rgsqr_option {
   ,RGSQR_OPT_CHUNK_MIB = 19     /* host path: MiB per column-chunk upload of an in-core or column-chunked
                                    node (the granularity at which the recursion waits for its columns and
                                    applies deferred products; >= 256 columns per product piece).  Default 32 */
+  ,RGSQR_OPT_VSHARDS = 20       /* p > 1: virtual row shards on ONE GPU (rgsqr_factor_device only; m must
+                                   split into p equal 16-byte aligned row blocks): the arithmetic of a p-GPU
+                                   row-sharded run -- every inner product as p local products (each with its
+                                   own split-K) summed in shard order, every leaf's round-0 vector as p local
+                                   vectors summed in shard order, no fused bottom node -- for testing the
+                                   multi-GPU algebra without p GPUs.  Default 1 */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

@@ -74,6 +74,12 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   c->begin_call();
   rc = sync_shape(c, m, &budget);
   if (rc < 0) return rc;
+  if (c->opt.vshards > 1) {
+    const int64_t p = c->opt.vshards;
+    if (c->nccl_comm) return fail(c, RGSQR_ERR_UNSUPPORTED, "virtual shards need a single-GPU context");
+    if (m % p != 0 || ((m / p) * elem_bytes(prec)) % 16 != 0)
+      return fail(c, RGSQR_ERR_UNSUPPORTED, "virtual shards: m must split into equal 16-byte aligned row blocks");
+  }
   auto t0 = std::chrono::steady_clock::now();
   const size_t ws = incore_workspace_bytes(c, prec, m, n);
   const size_t cap = resolve_budget(c, budget);
@@ -466,6 +472,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_COLCHUNK: return &o.colchunk;
     case RGSQR_OPT_EAGER_PCT: return &o.eager_pct;
     case RGSQR_OPT_CHUNK_MIB: return &o.chunk_mib;
+    case RGSQR_OPT_VSHARDS: return &o.vshards;
   }
   return nullptr;
 }
@@ -485,6 +492,7 @@ int rgsqr_set_option(rgsqr_handle h, int key, int64_t value) {
     case RGSQR_OPT_COLCHUNK: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_EAGER_PCT: if (value < 0 || value > 100) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_CHUNK_MIB: if (value < 1 || value > 1024) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_VSHARDS: if (value < 1 || value > 64) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_BLOCK_COLS: if (value < 8) return RGSQR_ERR_INVALID_ARG; break;
     default: if (value < 0) return RGSQR_ERR_INVALID_ARG;
   }

@@ -33,6 +33,7 @@ struct Options {
   int64_t x3_chain = 2;      // TF32X3: k-blocks per tensor-core accumulation chain (RGSQR_OPT_X3_CHAIN; 0 = unbounded)
   int64_t colchunk = 1;      // column-chunked OOC node (RGSQR_OPT_COLCHUNK, R26)
   int64_t chunk_mib = 32;    // host-path column upload chunk (RGSQR_OPT_CHUNK_MIB)
+  int64_t vshards = 1;       // virtual row shards on one GPU (RGSQR_OPT_VSHARDS, device path)
   int64_t eager_pct = 50;    // column-chunked node: the external projection is completed once the right
                              // child's leaves reach this % of its left half (RGSQR_OPT_EAGER_PCT)
 };

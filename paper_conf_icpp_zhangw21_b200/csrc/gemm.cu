@@ -217,12 +217,13 @@ __global__ void __launch_bounds__(128, 1)
 // owns TMEM lanes [32 (w-4), 32 (w-4) + 32)).  Output as gemm_kernel's TN epilogue.
 // ---------------------------------------------------------------------------------
 template <int BN>
-__global__ void __launch_bounds__(256, 1)
+__global__ void __launch_bounds__(128 + 16 * 32, 1)
     tn_promote_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                       const __grid_constant__ CUtensorMap mapA2, const __grid_constant__ CUtensorMap mapB2,
                       const GemmParams p) {
   using C = GemmCfg<float, false, BN>;
   static_assert(2 * BN <= 512, "two accumulators must fit TMEM");
+  static_assert(BN == 128, "16 accumulation warps x 32 columns");
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = ptx::smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
@@ -252,7 +253,7 @@ __global__ void __launch_bounds__(256, 1)
     }
     for (int b = 0; b < 2; ++b) {
       ptx::mbar_init(&tfull[b], 1);
-      ptx::mbar_init(&tempty[b], 4);
+      ptx::mbar_init(&tempty[b], 16);
     }
     ptx::fence_mbar_init();
   }
@@ -311,33 +312,35 @@ __global__ void __launch_bounds__(256, 1)
       }
     }
   } else if (warp >= 4) {
-    // the unit sums accumulate in fp64: with K = m rows there can be thousands of units, and an
-    // fp32 running sum would add a random-walk error of sqrt(units) * 2^-24
-    const int ew = warp - 4, lane = threadIdx.x & 31;
-    double sum[BN];
+    // 16 accumulation warps: warp w reads TMEM lanes [32 (w % 4), +32) (its lane quadrant) and
+    // columns [32 cg, 32 cg + 32), cg = (w - 4) / 4.  The unit sums accumulate in fp64: with K = m
+    // there can be thousands of units, and an fp32 running sum would add a random-walk error of
+    // sqrt(units) * 2^-24 (R25)
+    const int q = warp & 3, cg = (warp - 4) >> 2, lane = threadIdx.x & 31;
+    double sum[32];
 #pragma unroll
-    for (int j = 0; j < BN; ++j) sum[j] = 0.0;
+    for (int j = 0; j < 32; ++j) sum[j] = 0.0;
     for (int u = 0; u < nunits; ++u) {
       const int b = u & 1;
       ptx::mbar_wait(&tfull[b], (uint32_t)(u >> 1) & 1u);
       ptx::tc_fence_after();
 #pragma unroll
-      for (int cc = 0; cc < BN / 32; ++cc) {
-        uint32_t v[32];
-        ptx::tmem_ld_32x32b_x32(tmem + (uint32_t)(b * BN) + ((uint32_t)(ew * 32) << 16) + (uint32_t)(cc * 32), v);
+      for (int h = 0; h < 2; ++h) {   // two 16-column loads (register pressure at 640 threads)
+        uint32_t v[16];
+        ptx::tmem_ld_32x32b_x16(tmem + (uint32_t)(b * BN) + ((uint32_t)(q * 32) << 16) + (uint32_t)(cg * 32 + h * 16), v);
         ptx::tmem_ld_wait();
 #pragma unroll
-        for (int j = 0; j < 32; ++j) sum[cc * 32 + j] += (double)__uint_as_float(v[j]);
+        for (int j = 0; j < 16; ++j) sum[h * 16 + j] += (double)__uint_as_float(v[j]);
       }
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[b]);
     }
-    const int64_t i = m0 + ew * 32 + lane;
+    const int64_t i = m0 + q * 32 + lane;
     if (i < p.M) {
 #pragma unroll
-      for (int j = 0; j < BN; ++j) {
-        const int64_t n = n0 + j;
+      for (int j = 0; j < 32; ++j) {
+        const int64_t n = n0 + cg * 32 + j;
         if (n < p.N) {
           if (p.P != nullptr) {
             p.P[blockIdx.z * p.split_stride + i + n * p.ldp] = (float)sum[j];
@@ -653,7 +656,7 @@ static cudaError_t launch_tn_promote_t(const CUtensorMap& ma, const CUtensorMap&
     attr_set = true;
   }
   dim3 grid((unsigned)((p.M + C::BM - 1) / C::BM), (unsigned)((p.N + BN - 1) / BN), (unsigned)splits);
-  tn_promote_kernel<BN><<<grid, 256, SMEM, st>>>(ma, mb, ma2, mb2, p);
+  tn_promote_kernel<BN><<<grid, 128 + 16 * 32, SMEM, st>>>(ma, mb, ma2, mb2, p);
   return cudaGetLastError();
 }
 
@@ -664,8 +667,8 @@ cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMa
   const CUtensorMap& a2 = ma2 ? *ma2 : ma;
   const CUtensorMap& b2 = mb2 ? *mb2 : mb;
   if constexpr (sizeof(T) == 4) {
-    if (!nn && p.kb_per_unit > 0)   // bounded accumulation chain (TF32X3); fp64 unit sums: BN = 64
-      return launch_tn_promote_t<64>(ma, mb, a2, b2, p, splits, st);
+    if (!nn && p.kb_per_unit > 0)   // bounded accumulation chain (TF32X3), fp64 unit sums
+      return launch_tn_promote_t<128>(ma, mb, a2, b2, p, splits, st);
   }
   if (nn) {
     if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, a2, b2, p, splits, st);

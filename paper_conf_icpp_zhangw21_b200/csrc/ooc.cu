@@ -838,6 +838,7 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   int rc = validate(c, A, lda, m, n, Q, prec);
   if (rc < 0) return rc;
   if (!R && c->rank == 0) return fail(c, RGSQR_ERR_INVALID_ARG, "null R_out");
+  if (c->opt.vshards > 1) return fail(c, RGSQR_ERR_UNSUPPORTED, "virtual shards: device path only");
   reset_stats(c);
   rc = sync_shape(c, m, &budget);
   if (rc < 0) return rc;

@@ -138,7 +138,7 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
   if (rc < 0) return rc;
   Pipe P{c, c->compute(), c->st_h2d, c->st_d2h, s, {}};
   if (c->opt.serialize) P.sh = P.sd = P.sc;
-  const int K = (int)c->opt.ring_depth;
+  int K = (int)c->opt.ring_depth;   // (lowered to >= 2 slots when the budget is tight)
   P.freed.assign(K, nullptr);
   const char* hq = static_cast<const char*>(Q1);
   char* ha = static_cast<char*>(A2);
@@ -153,15 +153,23 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
   auto fits_rows = [&](size_t resident, size_t per_row, int64_t want) -> int64_t {
     const size_t free_b = c->arena.free_bytes();
     if (free_b < resident + ws_reserve) return 0;
-    int64_t t = (int64_t)((free_b - resident - ws_reserve) / ((size_t)K * per_row));
-    t = std::min<int64_t>({t, want, (m + 127) / 128 * 128});
-    return t / 128 * 128;
+    for (; K >= 2; --K) {
+      int64_t t = (int64_t)((free_b - resident - ws_reserve) / ((size_t)K * per_row));
+      t = std::min<int64_t>({t, want, (m + 127) / 128 * 128}) / 128 * 128;
+      if (t >= std::min<int64_t>(want, 1024) || K == 2) return t;
+    }
+    return 0;
+  };
+  auto fits_slots = [&](size_t per) -> bool {   // K column blocks / tiles of `per` bytes
+    const size_t free_b = c->arena.free_bytes();
+    while (K > 2 && (size_t)K * per + ws_reserve > free_b) --K;
+    return (size_t)K * per + ws_reserve <= free_b;
   };
   if (op == 0 && tiling == 0) {
     // ---- Fig. 3: R12 resident (fp32), row tiles of Q1 and A2 ----
     float* dR = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
     const int64_t t = dR ? fits_rows(0, (size_t)(w1 + w2) * s, block > 0 ? block : 16384) : 0;
-    if (!dR || t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner: R12 + 3 tiles do not fit");
+    if (!dR || t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner: R12 + 2 tiles do not fit");
     char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
     if (!ring) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner: ring");
     int64_t i = 0;
@@ -187,8 +195,8 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
     const int64_t b = std::min<int64_t>(w2, block > 0 ? block : 16384);
     char* dQ = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
     const size_t per = (size_t)m * b * s + (size_t)w1 * b * 4 + 512;
-    if (!dQ || c->arena.free_bytes() < (size_t)K * per + ws_reserve)
-      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner (blocking): panel + 3 column blocks do not fit");
+    if (!dQ || !fits_slots(per))
+      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner (blocking): panel + 2 column blocks do not fit");
     char* ring = static_cast<char*>(c->arena.alloc((size_t)K * per));
     if ((rc = P.up(dQ, m, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
     cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
@@ -227,7 +235,7 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
     if (tiling == 0) {
       // ---- Fig. 5: row tiles of Q1 and A2 in, A2' tiles out ----
       const int64_t t = fits_rows(0, (size_t)(w1 + w2) * s, block > 0 ? block : 8192);
-      if (t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer: R12 + 3 tiles do not fit");
+      if (t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer: R12 + 2 tiles do not fit");
       char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
       int64_t i = 0;
       for (int64_t r0 = 0; r0 < m; r0 += t, ++i) {
@@ -253,8 +261,8 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
       const int64_t b1 = std::min(b, (m + 127) / 128 * 128), b2 = std::min(b, w2);
       char* dQ = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
       const size_t per = (size_t)b1 * b2 * s;
-      if (!dQ || c->arena.free_bytes() < (size_t)K * per + ws_reserve)
-        return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer (blocking): Q1 + R12 + 3 tiles do not fit");
+      if (!dQ || !fits_slots(per))
+        return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer (blocking): Q1 + R12 + 2 tiles do not fit");
       char* ring = static_cast<char*>(c->arena.alloc((size_t)K * per));
       if ((rc = P.up(dQ, m, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
       cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);

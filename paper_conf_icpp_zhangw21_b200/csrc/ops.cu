@@ -100,6 +100,26 @@ template <typename T>
 static int op_inner_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* A2, int64_t lda, int64_t m,
                       int64_t w1, int64_t w2, float* R12, int64_t ldr, void* R12op, int64_t ldop, int accumulate,
                       cudaStream_t st, bool reduce_ranks) {
+  if (!c->nccl_comm && c->opt.vshards > 1 && reduce_ranks) {
+    // virtual row shards (RGSQR_OPT_VSHARDS): the multi-GPU arithmetic on one GPU --
+    // every shard's local Q1_s^T A2_s (its own split-K), then the sum over shards in shard order
+    const int64_t p = c->opt.vshards, ms = m / p;
+    if (accumulate) return fail(c, RGSQR_ERR_UNSUPPORTED, "inner: accumulate with shard reduction");
+    const size_t mark = c->arena.mark();
+    float* tmp = static_cast<float*>(c->arena.alloc((size_t)p * w1 * w2 * sizeof(float)));
+    if (!tmp) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner: no arena space for the shard partials");
+    for (int64_t sh = 0; sh < p; ++sh) {
+      const char* q = static_cast<const char*>(Q1) + sh * ms * (int64_t)sizeof(T);
+      const char* a = static_cast<const char*>(A2) + sh * ms * (int64_t)sizeof(T);
+      int rc = op_inner_local<T>(c, prec, q, ldq, a, lda, ms, w1, w2, tmp + sh * w1 * w2, w1, nullptr, 0, 0, st);
+      if (rc < 0) return rc;
+    }
+    RGSQR_CUDA(c, launch_splitk_reduce<T>(tmp, w1 * w2, w1, (int)p, R12, ldr, 0, static_cast<T*>(R12op), ldop, w1,
+                                          w2, st));
+    c->stats.n_other_launches++;
+    c->arena.release(mark);
+    return RGSQR_OK;
+  }
   if (!c->nccl_comm || !reduce_ranks)
     return op_inner_local<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
   if (accumulate) return fail(c, RGSQR_ERR_UNSUPPORTED, "inner: accumulate with rank reduction");
@@ -153,7 +173,7 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
   const int s = (int)sizeof(T);
   const int BK = gemm_block_k(s);
   const bool promote = Q1lo != nullptr && A2lo != nullptr && c->opt.x3_chain > 0;
-  const int bn = promote ? 64 : pick_bn(w2);   // (fp64 register accumulators: tn_promote_kernel)
+  const int bn = promote ? 128 : pick_bn(w2);   // (fp64 register accumulators: tn_promote_kernel)
   CUtensorMap ma, mb, ma2, mb2;
   std::string err;
   if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, BK, 128, &err) ||
@@ -403,7 +423,40 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
     return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: precision not supported");
   cudaError_t e;
   cudaEvent_t kb = c->kbegin(st);
-  if (!c->nccl_comm) {
+  if (!c->nccl_comm && c->opt.vshards > 1) {
+    // virtual row shards: each shard's round-0 vector (column norms, a_0.a_1) from a round-0-only
+    // launch over its rows, summed in shard order (the multi-GPU round-0 allreduce), then the main
+    // launch over all rows with the given vector
+    const int64_t ns = c->opt.vshards, ms = m / ns, L = LEAF_MAX_W + 2;
+    const size_t mark = c->arena.mark();
+    float* r0s = static_cast<float*>(c->arena.alloc((size_t)ns * L * sizeof(float)));
+    if (!r0s) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "leaf: no arena space for the shard round-0 vectors");
+    e = cudaSuccess;
+    for (int64_t sh = 0; sh < ns && e == cudaSuccess; ++sh) {
+      LeafParams p0 = p;
+      int Gs, rps;
+      leaf_geometry(c, ms, &Gs, &rps);
+      p0.P = static_cast<char*>(P) + sh * ms * elem_bytes(prec);
+      p0.m = ms;
+      p0.rows_per_cta = rps;
+      p0.r0_mode = 1;
+      p0.r0buf = r0s + sh * L;
+      e = [&]() -> cudaError_t {
+        switch (prec) {
+          case RGSQR_FP16: return launch_leaf<__half>(p0, Gs, st);
+          case RGSQR_BF16: return launch_leaf<__nv_bfloat16>(p0, Gs, st);
+          default: return launch_leaf<float>(p0, Gs, st);
+        }
+      }();
+    }
+    if (e == cudaSuccess)
+      e = launch_splitk_reduce<float>(r0s, L, L, (int)ns, c->d_r0buf, L, 0, nullptr, 0, w + 1, 1, st);
+    if (e == cudaSuccess) {
+      p.r0_mode = 2;
+      e = launch(p);
+    }
+    c->arena.release(mark);
+  } else if (!c->nccl_comm) {
     p.r0_mode = r0_pre ? 3 : 0;
     e = launch(p);
   } else {
@@ -488,7 +541,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
 // then runs the separate products), < 0 on error
 int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64_t lda, int64_t m, int64_t w1,
                   int64_t w2, float* R12, int64_t ldr, cudaStream_t st, bool r0_for_leaf) {
-  if (!c->opt.fuse_small || c->nccl_comm || w1 > 128 || w2 > 128 || w1 < 1 || w2 < 1) return 0;
+  if (!c->opt.fuse_small || c->nccl_comm || c->opt.vshards > 1 || w1 > 128 || w2 > 128 || w1 < 1 || w2 < 1) return 0;
   if (prec != RGSQR_FP16 && prec != RGSQR_BF16) return 0;
   const int W = (w1 <= 64 && w2 <= 64) ? 64 : 128;
   if (W == 128 && c->opt.fuse_small < 2) return 0;   // measured slower than the separate products
@@ -539,6 +592,7 @@ size_t incore_workspace_bytes(Ctx* c, int prec, int64_t m, int64_t n) {
   size_t b = 0;
   if (w1 > 0) b += (size_t)w1 * (n - w1) * elem_bytes(prec) + 1024;  // R12 operand copy
   if (w1 > 0 && c->nccl_comm) b += (size_t)w1 * (n - w1) * 4 + 1024;  // R12 rank-reduction buffer
+  if (w1 > 0 && c->opt.vshards > 1) b += (size_t)c->opt.vshards * w1 * (n - w1) * 4 + 1024;   // shard partials
   if (prec == RGSQR_TF32X3) b += (size_t)2 * m * n * 4 + 8192;          // hi/lo operands of the top node
   if (c->opt.reorth) {                                                   // CGS2: S (fp32) + leaf S block
     if (w1 > 0) b += (size_t)w1 * (n - w1) * 4 + 1024;

@@ -7,10 +7,12 @@ import pytest
 pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
 
+import oracle  # noqa: E402
 import rgsqr_inputs as gi  # noqa: E402
 from tests.gpu_util import to_dev, from_dev  # noqa: E402
 
 MiB = 1 << 20
+STOR = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}
 
 
 @pytest.fixture(scope="module")
@@ -90,3 +92,64 @@ def test_repeated_launches_keep_exchange_state(handles):
         R = torch.zeros((n, n), dtype=torch.float32, device="cuda")
         dist.op_leaf(Pd, m, m, n, R, n, precision="fp16")
         np.testing.assert_array_equal(R.cpu().numpy().T, np.eye(n))
+
+
+# ---- virtual row shards (RGSQR_OPT_VSHARDS): the multi-GPU arithmetic on one GPU ----------------
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+@pytest.mark.parametrize("p", [2, 4, 8])
+def test_vshards_dyadic_bitwise_equal_single(prec, p):
+    """p row shards on one GPU: every R12 as p local products summed in shard order, every leaf's
+    round-0 vector as p local vectors summed in shard order (the NCCL allreduces of a p-GPU run,
+    DESIGN.md 8; PAPER.md:171-173 row-local structure).  Exact-dyadic input: R == R0
+    and Q == H bitwise for every p, hence bitwise equal to the single-GPU result."""
+    from paper_conf_icpp_zhangw21_b200 import Handle
+    st = STOR[prec]
+    m, n = 65536, 512
+    A64, R0 = gi.dyadic_mixed(m, n, seed=13)
+    A = gi.to_storage(A64, st)
+    h = Handle(0)
+    h.set_option("vshards", p)
+    Ad = to_dev(A, st)
+    R = torch.empty((n, n), dtype=torch.float32, device="cuda")
+    rc = h.factor_device(Ad, m, m, n, Ad, R, precision=prec)
+    assert rc == 0
+    np.testing.assert_array_equal(R.cpu().numpy().T.astype(np.float64), R0)
+    np.testing.assert_array_equal(from_dev(Ad), gi.hadamard(m, n))
+    h.close()
+
+
+@pytest.mark.parametrize("prec", ["fp16", "tf32"])
+def test_vshards_gaussian_vs_single_and_oracle(prec):
+    from paper_conf_icpp_zhangw21_b200 import Handle
+    st = STOR[prec]
+    m, n = 16384, 1024
+    A = gi.gaussian(m, n, seed=17, dtype=st)
+    X = gi.to_float64(A, st)
+    ref = oracle.rgs(X, leaf=64)
+    h = Handle(0)
+    out = {}
+    for p in (1, 4):
+        h.set_option("vshards", p)
+        Ad = to_dev(A, st)
+        R = torch.empty((n, n), dtype=torch.float32, device="cuda")
+        assert h.factor_device(Ad, m, m, n, Ad, R, precision=prec) == 0
+        Rn = R.cpu().numpy().T.astype(np.float64)
+        Q = from_dev(Ad)
+        assert oracle.backward_error(X, Q, Rn) < 5e-3
+        assert oracle.r_rel_error(Rn, ref.R) < 5e-3
+        out[p] = Rn
+    assert oracle.r_rel_error(out[4], out[1]) < 2e-3
+    h.close()
+
+
+def test_vshards_rejects_unequal_shards():
+    from paper_conf_icpp_zhangw21_b200 import Handle, RgsqrError
+    h = Handle(0)
+    h.set_option("vshards", 3)
+    A = gi.gaussian(4096, 64, seed=1, dtype="fp16")
+    Ad = to_dev(A, "fp16")
+    R = torch.empty((64, 64), dtype=torch.float32, device="cuda")
+    with pytest.raises(RgsqrError) as e:
+        h.factor_device(Ad, 4096, 4096, 64, Ad, R, precision="fp16")
+    assert e.value.status == -5
+    h.close()
