@@ -228,7 +228,11 @@ int rgsqr_op_outer(rgsqr_handle h, const void* Q1, int64_t ldq, const void* R12o
 /* ---- support ------------------------------------------------------------------------ */
 int rgsqr_set_stream(rgsqr_handle h, void* cuda_stream);      /* NULL = library's own stream */
 int rgsqr_get_stream(rgsqr_handle h, void** cuda_stream);
-int rgsqr_host_alloc(rgsqr_handle h, size_t bytes, void** p);  /* pinned, first-touch */
+/* Pinned host memory on the GPU's NUMA node (sysfs numa_node of the GPU's PCI device): the pages
+ * are first-touched by threads bound to that node's CPUs, then page-locked (cudaHostRegister).
+ * Row shards of a multi-GPU run should live in their GPU's node.  Free with
+ * rgsqr_host_free on the same handle (or rgsqr_destroy frees what is left). */
+int rgsqr_host_alloc(rgsqr_handle h, size_t bytes, void** p);
 int rgsqr_host_free(rgsqr_handle h, void* p);
 int rgsqr_set_option(rgsqr_handle h, int key, int64_t value);
 int rgsqr_get_option(rgsqr_handle h, int key, int64_t* value);

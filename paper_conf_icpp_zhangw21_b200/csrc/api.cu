@@ -1,6 +1,13 @@
 // api.cu -- the extern "C" boundary declared in include/rgsqr.h.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
+#include <pthread.h>
+#include <sched.h>
+#include <sys/mman.h>
+
+#include <cctype>
+#include <cstdio>
+#include <thread>
 
 #include <chrono>
 #include <climits>
@@ -330,6 +337,10 @@ int rgsqr_destroy(rgsqr_handle h) {
   cudaFree(c->d_peers);
   cudaFree(c->d_r0buf);
   for (auto e : c->event_pool) cudaEventDestroy(e);
+  for (auto& a : c->host_allocs) {
+    cudaHostUnregister(a.first);
+    munmap(a.first, a.second);
+  }
   cudaStreamDestroy(c->st_own);
   cudaStreamDestroy(c->st_h2d);
   cudaStreamDestroy(c->st_d2h);
@@ -436,18 +447,85 @@ int rgsqr_get_stream(rgsqr_handle h, void** s) {
   return RGSQR_OK;
 }
 
+// NUMA node of the GPU (sysfs; -1 when unknown or single-node) and the CPUs of that node
+static int gpu_numa_node(int device) {
+  char bus[64] = {0};
+  if (cudaDeviceGetPCIBusId(bus, sizeof(bus), device) != cudaSuccess) return -1;
+  for (char* q = bus; *q; ++q) *q = (char)tolower(*q);
+  std::string path = std::string("/sys/bus/pci/devices/") + bus + "/numa_node";
+  FILE* f = fopen(path.c_str(), "r");
+  if (!f) return -1;
+  int node = -1;
+  if (fscanf(f, "%d", &node) != 1) node = -1;
+  fclose(f);
+  return node;
+}
+static std::vector<int> node_cpus(int node) {
+  std::vector<int> cpus;
+  if (node < 0) return cpus;
+  FILE* f = fopen(("/sys/devices/system/node/node" + std::to_string(node) + "/cpulist").c_str(), "r");
+  if (!f) return cpus;
+  char buf[4096] = {0};
+  if (fgets(buf, sizeof(buf), f)) {
+    for (char* tok = strtok(buf, ",\n"); tok; tok = strtok(nullptr, ",\n")) {
+      int a = -1, b = -1;
+      if (sscanf(tok, "%d-%d", &a, &b) == 2)
+        for (int x = a; x <= b; ++x) cpus.push_back(x);
+      else if (sscanf(tok, "%d", &a) == 1)
+        cpus.push_back(a);
+    }
+  }
+  fclose(f);
+  return cpus;
+}
+
+// Pinned host memory placed on the GPU's NUMA node: anonymous pages first-touched by threads bound
+// to that node's CPUs (the kernel's default policy allocates a page on the node of the CPU that first
+// writes it), then page-locked for DMA with cudaHostRegister.  The touch runs on up to 16 threads.
 int rgsqr_host_alloc(rgsqr_handle h, size_t bytes, void** p) {
   Ctx* c = C(h);
-  if (!c || !p) return RGSQR_ERR_INVALID_ARG;
+  if (!c || !p || bytes == 0) return RGSQR_ERR_INVALID_ARG;
   cudaSetDevice(c->device);
-  if (cudaHostAlloc(p, bytes, cudaHostAllocPortable) != cudaSuccess) return fail(c, RGSQR_ERR_HOST_MEM, "cudaHostAlloc");
+  void* mem = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+  if (mem == MAP_FAILED) return fail(c, RGSQR_ERR_HOST_MEM, "mmap failed");
+  const int node = gpu_numa_node(c->device);
+  const std::vector<int> cpus = node_cpus(node);
+  const int nt = (int)std::max<size_t>(1, std::min<size_t>(16, cpus.empty() ? 8 : cpus.size()));
+  const size_t page = 4096, per = ((bytes + nt - 1) / nt + page - 1) / page * page;
+  std::vector<std::thread> th;
+  for (int t = 0; t < nt; ++t) {
+    th.emplace_back([&, t] {
+      if (!cpus.empty()) {
+        cpu_set_t set;
+        CPU_ZERO(&set);
+        for (int cpu : cpus) CPU_SET(cpu, &set);
+        pthread_setaffinity_np(pthread_self(), sizeof(set), &set);
+      }
+      const size_t a = std::min(bytes, (size_t)t * per), b = std::min(bytes, a + per);
+      if (b > a) std::memset(static_cast<char*>(mem) + a, 0, b - a);
+    });
+  }
+  for (auto& x : th) x.join();
+  if (cudaHostRegister(mem, bytes, cudaHostRegisterPortable) != cudaSuccess) {
+    cudaGetLastError();
+    munmap(mem, bytes);
+    return fail(c, RGSQR_ERR_HOST_MEM, "cudaHostRegister of the host buffer failed");
+  }
+  c->host_allocs[mem] = bytes;
+  c->host_numa_node = node;
+  *p = mem;
   return RGSQR_OK;
 }
 
 int rgsqr_host_free(rgsqr_handle h, void* p) {
   Ctx* c = C(h);
   if (!c) return RGSQR_ERR_INVALID_ARG;
-  return cudaFreeHost(p) == cudaSuccess ? RGSQR_OK : RGSQR_ERR_CUDA;
+  auto it = c->host_allocs.find(p);
+  if (it == c->host_allocs.end()) return fail(c, RGSQR_ERR_INVALID_ARG, "rgsqr_host_free: not from rgsqr_host_alloc");
+  cudaHostUnregister(p);
+  munmap(p, it->second);
+  c->host_allocs.erase(it);
+  return RGSQR_OK;
 }
 
 static int64_t* opt_slot(Ctx* c, int key) {

@@ -6,6 +6,7 @@
 
 #include <cstdint>
 #include <functional>
+#include <map>
 #include <string>
 #include <vector>
 
@@ -104,6 +105,8 @@ struct Ctx {
   // a leaf exchange timed out (a rank did not arrive): late contributions may still land in the
   // never-reset exchange words, so the handle refuses further factorizations (rgsqr_destroy it)
   bool broken = false;
+  std::map<void*, size_t> host_allocs;       // rgsqr_host_alloc buffers (NUMA-placed, registered)
+  int host_numa_node = -1;                   // the GPU's NUMA node (-1: unknown / single node)
 
   cudaStream_t compute() const { return st_user ? st_user : st_own; }
   cudaEvent_t ev();

@@ -246,3 +246,25 @@ def test_colchunk_serialized_equals_overlapped(h):
     assert s1["n_colchunk_nodes"] >= 1 and s2["n_colchunk_nodes"] >= 1
     np.testing.assert_array_equal(R1, R2)
     np.testing.assert_array_equal(Q1, Q2)
+
+
+def test_host_alloc_numa_buffers(h):
+    """rgsqr_host_alloc: NUMA-placed, page-locked buffers (include/rgsqr.h) used as A / Q / R of the
+    out-of-core path; results equal those from pageable numpy buffers; freeing twice is an error."""
+    import ctypes
+    from paper_conf_icpp_zhangw21_b200 import RgsqrError
+    m, n = 8192, 512
+    A = gi.gaussian(m, n, seed=41, dtype="fp16")
+    nb = A.nbytes
+    pa, pq, pr = h.host_alloc(nb), h.host_alloc(nb), h.host_alloc(n * n * 4)
+    np.ctypeslib.as_array((ctypes.c_uint8 * nb).from_address(pa))[:] = A.reshape(-1, order="F").view(np.uint8)
+    assert h.factor(pa, m, m, n, pq, pr, precision="fp16", budget=6 * MiB) == 0
+    Qp = np.ctypeslib.as_array((ctypes.c_uint16 * (m * n)).from_address(pq)).view(np.float16).reshape((m, n), order="F")
+    Rp = np.ctypeslib.as_array((ctypes.c_float * (n * n)).from_address(pr)).reshape((n, n), order="F")
+    rc, Q, R, _ = factor(h, A, "fp16", 6 * MiB)
+    np.testing.assert_array_equal(Rp, R)
+    np.testing.assert_array_equal(Qp, Q)
+    for p_ in (pa, pq, pr):
+        h.host_free(p_)
+    with pytest.raises(RgsqrError):
+        h.host_free(pa)

@@ -41,7 +41,7 @@ def test_ooc_inner(h, prec, tiling, block):
     m, w1, w2 = 20000, 384, 520
     st, Q, A, Xq, Xa = _ops(prec, m, w1, w2, 3)
     R = np.full((w1, w2), np.nan, dtype=np.float32, order="F")
-    budget = 48 * MiB
+    budget = 48 * MiB * (2 if st == "fp32" else 1)
     h.ooc_inner(Q, m, A, m, m, w1, w2, R, w1, precision=prec, tiling=tiling, block=block, budget=budget)
     ref = Xq.T @ Xa
     bound = C[prec] * (np.abs(Xq).T @ np.abs(Xa))
@@ -55,10 +55,11 @@ def test_ooc_inner(h, prec, tiling, block):
 def test_ooc_outer(h, prec, tiling, block):
     m, w1, w2 = 20000, 256, 520
     st, Q, A, Xq, Xa = _ops(prec, m, w1, w2, 5)
-    R = np.asfortranarray(np.random.default_rng(1).standard_normal((w1, w2)).astype(np.float32) / np.sqrt(w1))
+    R = np.asfortranarray((np.random.default_rng(1).standard_normal((w1, w2)) / np.sqrt(w1)).astype(np.float32))
     Rop = gi.to_float64(gi.to_storage(R.astype(np.float64), st), st)     # R12 as the MMA operand (R9)
     A2 = np.array(A, order="F", copy=True)
-    h.ooc_outer(Q, m, R, w1, A2, m, m, w1, w2, precision=prec, tiling=tiling, block=block, budget=48 * MiB)
+    h.ooc_outer(Q, m, R, w1, A2, m, m, w1, w2, precision=prec, tiling=tiling, block=block,
+                budget=48 * MiB * (2 if st == "fp32" else 1))
     ref = Xa - Xq @ Rop
     got = gi.to_float64(A2, st)
     bound = U[prec] * np.abs(ref) + C[prec] * (np.abs(Xq) @ np.abs(Rop)) + 1e-30
