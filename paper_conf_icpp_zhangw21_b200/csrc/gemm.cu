@@ -36,6 +36,21 @@ struct GemmCfg {
   static constexpr uint32_t IDESC = ptx::idesc_f32acc(Elem<T>::kUmmaFormat, kNN ? 1u : 0u, 0u, BM, BN);
 };
 
+// Grouped rasterization of a (nx x ny) tile grid launched x-fastest: consecutive CTAs walk GROUP_M
+// M-tiles for each N-tile, so a wave of 148 CTAs covers ~16 x 9 tiles and both operands' K-panels are
+// re-read from L2 instead of DRAM (the plain x-fastest order re-reads every M-panel once per N-tile:
+// 2.5x the algorithmic DRAM bytes at 4096 x 65536 x 4096, profiles/r1_ncu_summary.md)
+__device__ __forceinline__ void grouped_tile(int bx, int by, int nx, int ny, int* tm, int* tn) {
+  constexpr int GROUP_M = 16;
+  const int L = by * nx + bx;
+  const int per_group = GROUP_M * ny;
+  const int g = L / per_group, first = g * GROUP_M;
+  const int gsz = min(nx - first, GROUP_M);
+  const int r = L - g * per_group;
+  *tm = first + r % gsz;
+  *tn = r / gsz;
+}
+
 template <typename T, bool kNN, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
@@ -51,8 +66,10 @@ __global__ void __launch_bounds__(128, 1)
   uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
 
   const int warp = threadIdx.x >> 5;
-  const int64_t m0 = (int64_t)blockIdx.x * C::BM;
-  const int64_t n0 = (int64_t)blockIdx.y * BN;
+  int tm, tn;
+  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, &tm, &tn);
+  const int64_t m0 = (int64_t)tm * C::BM;
+  const int64_t n0 = (int64_t)tn * BN;
   const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;
   const int64_t kb1 = min(p.kb_total, kb0 + p.kb_per_split);
   const int nkb = (int)(kb1 - kb0);
@@ -234,8 +251,10 @@ __global__ void __launch_bounds__(128 + 16 * 32, 1)
   uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
 
   const int warp = threadIdx.x >> 5;
-  const int64_t m0 = (int64_t)blockIdx.x * C::BM;
-  const int64_t n0 = (int64_t)blockIdx.y * BN;
+  int tm, tn;
+  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, &tm, &tn);
+  const int64_t m0 = (int64_t)tm * C::BM;
+  const int64_t n0 = (int64_t)tn * BN;
   const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;
   const int64_t kb1 = min(p.kb_total, kb0 + p.kb_per_split);
   const int nkb = kb1 > kb0 ? (int)(kb1 - kb0) : 0;

@@ -74,9 +74,9 @@ def test_ooc_gemm_serialized_equals_overlapped(h):
     for ser in (1, 0):
         h.set_option("serialize", ser)
         R = np.empty((w1, w2), dtype=np.float32, order="F")
-        h.ooc_inner(Q, m, A, m, m, w1, w2, R, w1, precision="fp16", tiling=0, block=2048, budget=16 * MiB)
+        h.ooc_inner(Q, m, A, m, m, w1, w2, R, w1, precision="fp16", tiling=0, block=2048, budget=32 * MiB)
         A2 = np.array(A, order="F", copy=True)
-        h.ooc_outer(Q, m, R, w1, A2, m, m, w1, w2, precision="fp16", tiling=0, block=2048, budget=16 * MiB)
+        h.ooc_outer(Q, m, R, w1, A2, m, m, w1, w2, precision="fp16", tiling=0, block=2048, budget=32 * MiB)
         out.append((R, A2))
     np.testing.assert_array_equal(out[0][0], out[1][0])
     np.testing.assert_array_equal(out[0][1], out[1][1])
