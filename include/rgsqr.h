@@ -120,6 +120,9 @@ enum rgsqr_option {
                                    own split-K) summed in shard order, every leaf's round-0 vector as p local
                                    vectors summed in shard order, no fused bottom node -- for testing the
                                    multi-GPU algebra without p GPUs.  Default 1 */
+  ,RGSQR_OPT_DEFER_PIECES = 21  /* host path: a node whose columns are still uploading applies its deferred
+                                   products (R23) in pieces of ~1/p of its A2 (p > 0) instead of
+                                   one upload chunk (0, default): fewer, wider GEMMs vs an earlier start */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

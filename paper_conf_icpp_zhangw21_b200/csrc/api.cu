@@ -551,6 +551,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_EAGER_PCT: return &o.eager_pct;
     case RGSQR_OPT_CHUNK_MIB: return &o.chunk_mib;
     case RGSQR_OPT_VSHARDS: return &o.vshards;
+    case RGSQR_OPT_DEFER_PIECES: return &o.defer_pieces;
   }
   return nullptr;
 }

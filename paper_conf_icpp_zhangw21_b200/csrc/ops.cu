@@ -665,8 +665,15 @@ static int incore_need(IncoreCtx& k, int64_t col_end) {
   }
   for (auto& d : k.deferred) {
     while (d.applied < std::min(col_end, d.end)) {
-      const int64_t a = d.applied;
-      const int64_t b = std::min(d.end, (a / k.hooks->chunk + 1) * k.hooks->chunk);
+      // pieces of the upload chunk, or (RGSQR_OPT_DEFER_PIECES = p > 0) about 1/p of the node's A2:
+      // narrow pieces let the recursion start on early columns, wide pieces keep the GEMMs efficient
+      const int64_t a = d.applied, ch = k.hooks->chunk;
+      int64_t piece = ch;
+      if (k.c->opt.defer_pieces > 0) {
+        const int64_t w2n = d.end - (d.c0 + d.w1);
+        piece = std::max(ch, (w2n / k.c->opt.defer_pieces + ch - 1) / ch * ch);
+      }
+      const int64_t b = piece == ch ? std::min(d.end, (a / ch + 1) * ch) : std::min(d.end, a + piece);
       k.hooks->need(b);
       const int64_t h = d.c0 + d.w1, off = a - h;
       const char* Q1 = k.A + d.c0 * k.lda * k.s;
