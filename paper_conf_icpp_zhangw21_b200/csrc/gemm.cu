@@ -40,8 +40,13 @@ struct GemmCfg {
 // M-tiles for each N-tile, so a wave of 148 CTAs covers ~16 x 9 tiles and both operands' K-panels are
 // re-read from L2 instead of DRAM (the plain x-fastest order re-reads every M-panel once per N-tile:
 // 2.5x the algorithmic DRAM bytes at 4096 x 65536 x 4096, profiles/r1_ncu_summary.md)
-__device__ __forceinline__ void grouped_tile(int bx, int by, int nx, int ny, int* tm, int* tn) {
-  constexpr int GROUP_M = 16;
+__device__ __forceinline__ void grouped_tile(int bx, int by, int nx, int ny, int group_m, int* tm, int* tn) {
+  if (group_m <= 1) {
+    *tm = bx;
+    *tn = by;
+    return;
+  }
+  const int GROUP_M = group_m;
   const int L = by * nx + bx;
   const int per_group = GROUP_M * ny;
   const int g = L / per_group, first = g * GROUP_M;
@@ -67,7 +72,7 @@ __global__ void __launch_bounds__(128, 1)
 
   const int warp = threadIdx.x >> 5;
   int tm, tn;
-  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, &tm, &tn);
+  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, p.group_m, &tm, &tn);
   const int64_t m0 = (int64_t)tm * C::BM;
   const int64_t n0 = (int64_t)tn * BN;
   const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;
@@ -252,7 +257,7 @@ __global__ void __launch_bounds__(128 + 16 * 32, 1)
 
   const int warp = threadIdx.x >> 5;
   int tm, tn;
-  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, &tm, &tn);
+  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, p.group_m, &tm, &tn);
   const int64_t m0 = (int64_t)tm * C::BM;
   const int64_t n0 = (int64_t)tn * BN;
   const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;

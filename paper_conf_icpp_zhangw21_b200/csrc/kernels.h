@@ -45,6 +45,7 @@ struct GemmParams {
   void* A2;
   int64_t lda2;
   int64_t kb_seg;           // > 0: K blocks per operand segment (TF32X3: hi.lo, lo.hi, hi.hi)
+  int group_m;              // > 1: grouped tile rasterization, this many M-tiles per group (gemm.cu)
   int64_t kb_per_unit;      // > 0 (fp32 TN only): k-blocks per tensor-core accumulation chain, the
                             // chains summed in fp32 registers (tn_promote_kernel, R25)
 };

@@ -193,6 +193,10 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
     p.kb_total *= 3;
   }
   const int64_t tiles = ((w1 + 127) / 128) * ((w2 + bn - 1) / bn);
+  // grouped rasterization only pays on grids of many waves (e.g. the Table 1 shapes); on the
+  // recursion's nodes (<= ~4 waves) the x-fastest order measured faster (RGSQR_GROUP_M overrides)
+  static const int env_group = getenv("RGSQR_GROUP_M") ? atoi(getenv("RGSQR_GROUP_M")) : -1;
+  p.group_m = env_group >= 0 ? env_group : (tiles > 8 * (int64_t)c->num_sms ? 16 : 0);
   // One wave: tiles x splits <= SMs (rounding up put 152 CTAs on 148 SMs at w1 = w2 = 512 and
   // doubled the kernel time: 57 vs 37 us, profiles/r1_splitk_scan.txt).
   int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : c->num_sms / tiles);
