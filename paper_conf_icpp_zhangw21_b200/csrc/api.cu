@@ -184,6 +184,7 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaMalloc(&c->d_r0buf, sizeof(float) * (LEAF_MAX_W + 2)) != cudaSuccess ||
       cudaMemset(c->d_xw, 0, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
       cudaMemset(c->d_xprev, 0, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||
+      cudaMemset(c->d_counter, 0, 4096) != cudaSuccess ||
       cudaMemcpy(c->d_peers, &c->d_xw, sizeof(void*), cudaMemcpyHostToDevice) != cudaSuccess) {
     delete c;
     return RGSQR_ERR_CUDA;

@@ -87,7 +87,8 @@ struct Ctx {
   float* d_partials = nullptr;
   float* d_sn_partials = nullptr;   // fused bottom node: [LEAF_MAX_G][4096] partials
   void* d_sn_r12op = nullptr;       // fused bottom node: 64 x 64 operand copy
-  unsigned int* d_counter = nullptr;
+  unsigned int* d_counter = nullptr;        // [0] leaf round-0 barrier, [16] fused node barriers
+  unsigned int counter_host[2] = {0, 0};     // their values after every enqueued barrier (never reset)
   unsigned int leaf_epoch = 0;
   int* d_breakdown = nullptr;
   void* nccl_comm = nullptr;

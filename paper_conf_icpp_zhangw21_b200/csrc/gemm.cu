@@ -41,6 +41,11 @@ struct GemmCfg {
 // re-read from L2 instead of DRAM (the plain x-fastest order re-reads every M-panel once per N-tile:
 // 2.5x the algorithmic DRAM bytes at 4096 x 65536 x 4096, profiles/r1_ncu_summary.md)
 __device__ __forceinline__ void grouped_tile(int bx, int by, int nx, int ny, int group_m, int* tm, int* tn) {
+#ifdef RGSQR_NO_GROUPED_TILE
+  *tm = bx;
+  *tn = by;
+  return;
+#endif
   if (group_m <= 1) {
     *tm = bx;
     *tn = by;

@@ -73,7 +73,9 @@ struct LeafParams {
   float* R;                 // w x w block of R (ldr)
   int64_t ldr;
   float* partials;          // [2][LEAF_MAX_W+2][grid] per-CTA partial sums
-  unsigned int* counter;    // grid barrier counter (zeroed by the launcher)
+  unsigned int* counter;    // grid barrier counter, never reset: round 0 waits for counter_target
+  unsigned int counter_target;       // (set by the launcher from *counter_host)
+  unsigned int* counter_host;        // host copy of the counter's value after all enqueued barriers
   long long* dbg;           // optional [w][8] clock64 stamps of CTA dbg_cta
   long long* dbg2;          // optional [grid][LEAF_MAX_W][2] globaltimer: critical publish, poll done
   int dbg_cta;
@@ -108,7 +110,9 @@ struct SmallNodeParams {
   int64_t ldr;
   float* partials;          // [grid][W*W], W = 64 or 128
   void* r12op;              // [W][W] operand copy ([j][i])
-  unsigned* counter;        // zeroed by the launcher
+  unsigned* counter;        // never reset: barrier k waits for counter_base + k G
+  unsigned counter_base;    // (set by the launcher from *counter_host)
+  unsigned* counter_host;   // host copy of the counter's value after all enqueued barriers
   float* r0_partials;       // non-null: also write the next leaf's round-0 partials of the new A2
                             // ([k][grid]: ||a_k||^2, k < w2, then a_0.a_1) -- leaf r0_mode 3
 };

@@ -338,7 +338,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       unsigned cv;
       do {
         asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cv) : "l"(p.counter) : "memory");
-      } while (cv < (unsigned)G);
+      } while ((int)(cv - p.counter_target) < 0);   // (wrap-safe: the counter is never reset)
     }
     __syncthreads();
     }
@@ -806,8 +806,12 @@ static cudaError_t launch_leaf_nr(const LeafParams& p, int grid, cudaStream_t st
     if (e != cudaSuccess) return e;
     attr_smem = smem;
   }
-  cudaError_t e = cudaMemsetAsync(p.counter, 0, sizeof(unsigned int), st);
-  if (e != cudaSuccess) return e;
+  // round 0's counter barrier (modes 0 and 1) waits for G more arrivals than all earlier launches
+  // enqueued on this counter: no per-launch reset (a memset node per leaf)
+  LeafParams q = p;
+  const bool barrier = q.r0_mode == 0 || q.r0_mode == 1;
+  if (barrier) q.counter_target = *p.counter_host + (unsigned)grid;
+  cudaError_t e;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(LEAF_THREADS);
@@ -818,7 +822,9 @@ static cudaError_t launch_leaf_nr(const LeafParams& p, int grid, cudaStream_t st
   attr[0].val.cooperative = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, leaf_cgs_kernel<T, NR, CW>, p);
+  e = cudaLaunchKernelEx(&cfg, leaf_cgs_kernel<T, NR, CW>, q);
+  if (e == cudaSuccess && barrier) *p.counter_host += (unsigned)grid;   // (only launched arrivals count)
+  return e;
 }
 
 template <typename T>

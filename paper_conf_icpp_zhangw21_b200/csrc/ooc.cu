@@ -569,6 +569,7 @@ struct Exec {
     size_t htop = 0;                 // bytes at the top of H used as scratch (left child, tail phase)
     int64_t ch = 0;                  // upload / product chunk width
     int64_t E1 = 0;                  // head columns projected before the right child (phase A)
+    int64_t pA = 0;                  // phase-A piece width
     int64_t pB = 0;                  // piece width of the remaining projection (phase B)
   };
   bool plan_cc(int64_t w1, int64_t w2, size_t free0, CCPlan* P) const {
@@ -592,9 +593,11 @@ struct Exec {
       const int64_t wt1 = std::min<int64_t>(wt, (int64_t)(X / colb) / 8 * 8);
       const int64_t wt2 = wt - wt1;
       const size_t tail_ws = (size_t)w1 * wt * (4 + s) + 1024 + (size_t)wt2 * colb + 256;
-      // phase A: the first E1 head columns projected in one piece before the right child starts
-      const int64_t E1 = std::min<int64_t>(wh, std::max<int64_t>(ch, (hw / 2) / ch * ch));
-      const size_t phaseA = (size_t)w1 * E1 * (4 + s) + 512;
+      // phase A: the right child's first half of head columns (E1) projected before it starts, in
+      // pieces of pA columns (two fp32 R12 buffers + one operand buffer), while the tail goes out
+      const int64_t E1 = std::min<int64_t>(wh, std::max<int64_t>(ch, hw / ch * ch));
+      const int64_t pA = std::min<int64_t>(E1, 4 * ch);
+      const size_t phaseA = (size_t)w1 * pA * (8 + s) + 1024;
       const size_t htop = (std::max({left_ws, rs1 + tail_ws, phaseA}) + 4095) / 4096 * 4096;
       if (htop > H || wt > w1) continue;
       P->wh = wh;
@@ -603,6 +606,7 @@ struct Exec {
       P->htop = htop;
       P->ch = ch;
       P->E1 = E1;
+      P->pA = pA;
       P->pB = pB;
       return true;
     }
@@ -741,26 +745,31 @@ struct Exec {
         cudaStreamWaitEvent(sc, feed.chunks[waited++].second, 0);
     };
     const int64_t E1 = std::min<int64_t>(P.E1, htop_col / ch * ch);   // (its columns must be uploaded)
+    cudaEvent_t phaseA_r[2] = {nullptr, nullptr};
     if (E1 > 0) {
+      const int64_t pA = std::min<int64_t>(P.pA, E1);
       if (left_r) cudaStreamWaitEvent(sc, left_r, 0);
       wsave = window(Htop, Hend);
-      ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * E1 * 4));
-      ext.R12op = c->arena.alloc((size_t)w1 * E1 * s);
+      ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * pA * 4));
+      ext.R12[1] = static_cast<float*>(c->arena.alloc((size_t)w1 * pA * 4));
+      ext.R12op = c->arena.alloc((size_t)w1 * pA * s);
       unwindow(wsave);
-      if (!ext.R12[0] || !ext.R12op)
+      if (!ext.R12[0] || !ext.R12[1] || !ext.R12op)
         return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the first projection");
-      ext.piece = E1;
+      ext.piece = pA;
       rc = apply_ext(c, prec, H, m, m, &hkA, E1, sc);
       if (rc < 0) return rc;
+      phaseA_r[0] = ext.free_ev[0];
+      phaseA_r[1] = ext.free_ev[1];
     }
     seg_end(2, sc, a_seg);
     cudaEvent_t phaseA_done = mark_ev(sc);
-    cudaEvent_t phaseA_r = ext.free_ev[0];
     // the rest of the head goes into H's top once the tail phase and phase A have released it
     cudaStreamWaitEvent(sh, phaseA_done, 0);
     cudaStreamWaitEvent(sh, tail_out, 0);
     if (r12t_out) cudaStreamWaitEvent(sh, r12t_out, 0);
-    if (phaseA_r) cudaStreamWaitEvent(sh, phaseA_r, 0);
+    for (cudaEvent_t e : phaseA_r)
+      if (e) cudaStreamWaitEvent(sh, e, 0);
     for (int64_t a = htop_col; a < wh;) {
       const int64_t end = std::min(wh, (a / ch + 1) * ch);
       if ((rc = head_chunk(a, end)) < 0) return rc;

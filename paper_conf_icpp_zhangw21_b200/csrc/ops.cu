@@ -392,6 +392,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   static const bool dbg = getenv("RGSQR_LEAF_DEBUG") != nullptr;
   static long long* dbg_buf = nullptr;
   p.counter = c->d_counter;
+  p.counter_host = &c->counter_host[0];
   p.epoch = ++c->leaf_epoch;
   p.xw = c->d_xw;
   p.xw_peers = c->d_peers;
@@ -569,6 +570,7 @@ int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64
   p.partials = c->d_sn_partials;
   p.r12op = c->d_sn_r12op;
   p.counter = c->d_counter + 16;
+  p.counter_host = &c->counter_host[1];
   p.r0_partials = r0_for_leaf ? c->d_partials : nullptr;
   cudaEvent_t kb = c->kbegin(st);
   cudaError_t e = prec == RGSQR_FP16 ? launch_small_node<__half>(p, G, st) : launch_small_node<__nv_bfloat16>(p, G, st);

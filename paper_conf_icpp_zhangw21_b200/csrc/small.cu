@@ -77,7 +77,8 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t* r, const void* p) {
                : "r"(a));
 }
 
-// grid barrier k (k = 1, 2, ...) on a zeroed counter: release this CTA's writes, acquire all
+// grid barrier on a never-reset counter: release this CTA's writes, wait until the counter reaches
+// `target` (wrap-safe), acquire all
 __device__ __forceinline__ void sn_grid_barrier(unsigned* counter, unsigned target) {
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -85,7 +86,7 @@ __device__ __forceinline__ void sn_grid_barrier(unsigned* counter, unsigned targ
     unsigned v;
     do {
       asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(counter) : "memory");
-    } while (v < target);
+    } while ((int)(v - target) < 0);
   }
   __syncthreads();
 }
@@ -162,7 +163,7 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
     }
     __syncthreads();                               // before the next half overwrites `as`
   }
-  sn_grid_barrier(p.counter, (unsigned)G);
+  sn_grid_barrier(p.counter, p.counter_base + (unsigned)G);
 
   // ---- phase 2: entries [g EPC, (g+1) EPC) summed over the G partials in a fixed order:
   //      warp k adds partials k, k+8, ... in order, then warp 0 the 8 groups ----
@@ -196,7 +197,7 @@ __global__ void __launch_bounds__(SN_THREADS, 1) small_node_kernel(SmallNodePara
       __syncthreads();
     }
   }
-  sn_grid_barrier(p.counter, (unsigned)(2 * G));
+  sn_grid_barrier(p.counter, p.counter_base + (unsigned)(2 * G));
 
   // ---- phase 3: A2_s -= Q1_s R12 per half; warp: m-tiles warp, warp + 8, ... (16 rows), all
   //      8 n-tiles of the half, K = W ----
@@ -309,8 +310,8 @@ static cudaError_t launch_small_node_w(const SmallNodeParams& p, int grid, cudaS
     if (e != cudaSuccess) return e;
     attr = smem;
   }
-  cudaError_t e = cudaMemsetAsync(p.counter, 0, sizeof(unsigned), st);
-  if (e != cudaSuccess) return e;
+  SmallNodeParams q = p;   // two barriers per launch on the never-reset counter
+  q.counter_base = *p.counter_host;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(SN_THREADS);
@@ -321,7 +322,9 @@ static cudaError_t launch_small_node_w(const SmallNodeParams& p, int grid, cudaS
   attr1[0].val.cooperative = 1;
   cfg.attrs = attr1;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, small_node_kernel<T, W>, p);
+  cudaError_t e = cudaLaunchKernelEx(&cfg, small_node_kernel<T, W>, q);
+  if (e == cudaSuccess) *p.counter_host += 2u * (unsigned)grid;   // (only launched arrivals count)
+  return e;
 }
 
 template <typename T>

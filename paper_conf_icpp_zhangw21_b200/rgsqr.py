@@ -15,7 +15,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "librgsqr.so")
+LIB_PATH = os.environ.get("RGSQR_LIB", os.path.join(_HERE, "librgsqr.so"))   # (override: A/B experiments)
 
 PRECISIONS = {"fp16": 0, "bf16": 1, "tf32": 2, "tf32x3": 3}
 STORAGE = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32", "tf32x3": "fp32"}
