@@ -123,6 +123,9 @@ enum rgsqr_option {
   ,RGSQR_OPT_DEFER_PIECES = 21  /* host path: a node whose columns are still uploading applies its deferred
                                    products (R23) in pieces of ~1/p of its A2 (p > 0) instead of
                                    one upload chunk (0, default): fewer, wider GEMMs vs an earlier start */
+  ,RGSQR_OPT_PHASEA_PCT = 22    /* column-chunked node: percentage of the right child's first half whose Q1
+                                   projection is applied before the right child starts (phase A, while the
+                                   tail goes out; default 100) */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

@@ -553,6 +553,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_CHUNK_MIB: return &o.chunk_mib;
     case RGSQR_OPT_VSHARDS: return &o.vshards;
     case RGSQR_OPT_DEFER_PIECES: return &o.defer_pieces;
+    case RGSQR_OPT_PHASEA_PCT: return &o.phasea_pct;
   }
   return nullptr;
 }
@@ -570,7 +571,8 @@ int rgsqr_set_option(rgsqr_handle h, int key, int64_t value) {
     case RGSQR_OPT_ALGO: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_REORTH: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_COLCHUNK: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
-    case RGSQR_OPT_EAGER_PCT: if (value < 0 || value > 100) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_EAGER_PCT:
+    case RGSQR_OPT_PHASEA_PCT: if (value < 0 || value > 100) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_CHUNK_MIB: if (value < 1 || value > 1024) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_VSHARDS: if (value < 1 || value > 64) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_BLOCK_COLS: if (value < 8) return RGSQR_ERR_INVALID_ARG; break;

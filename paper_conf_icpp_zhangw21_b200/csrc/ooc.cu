@@ -595,8 +595,8 @@ struct Exec {
       const size_t tail_ws = (size_t)w1 * wt * (4 + s) + 1024 + (size_t)wt2 * colb + 256;
       // phase A: the right child's first half of head columns (E1) projected before it starts, in
       // pieces of pA columns (two fp32 R12 buffers + one operand buffer), while the tail goes out
-      const int64_t E1 = std::min<int64_t>(wh, std::max<int64_t>(ch, hw / ch * ch));
-      const int64_t pA = std::min<int64_t>(E1, 4 * ch);
+      const int64_t E1 = std::min<int64_t>(wh, (hw * c->opt.phasea_pct / 100) / ch * ch);
+      const int64_t pA = std::max<int64_t>(ch, std::min<int64_t>(E1, 4 * ch));
       const size_t phaseA = (size_t)w1 * pA * (8 + s) + 1024;
       const size_t htop = (std::max({left_ws, rs1 + tail_ws, phaseA}) + 4095) / 4096 * 4096;
       if (htop > H || wt > w1) continue;

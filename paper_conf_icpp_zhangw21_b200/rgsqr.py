@@ -26,7 +26,7 @@ OPTIONS = {"leaf_width": 1, "tile_rows_min": 2, "tile_rows_max": 3, "ring_depth"
            "reorth": 12, "prefetch": 13, "fuse_small": 14, "split_pct": 15,
            "x3_chain": 16, "colchunk": 17, "eager_pct": 18,
            "chunk_mib": 19, "vshards": 20,
-           "defer_pieces": 21}
+           "defer_pieces": 21, "phasea_pct": 22}
 
 EXPORTS = ["rgsqr_create", "rgsqr_get_unique_id", "rgsqr_create_dist", "rgsqr_destroy", "rgsqr_factor",
            "rgsqr_factor_device", "rgsqr_op_leaf", "rgsqr_op_inner", "rgsqr_op_outer", "rgsqr_set_stream",
