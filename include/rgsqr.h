@@ -125,7 +125,7 @@ enum rgsqr_option {
                                    one upload chunk (0, default): fewer, wider GEMMs vs an earlier start */
   ,RGSQR_OPT_PHASEA_PCT = 22    /* column-chunked node: percentage of the right child's first half whose Q1
                                    projection is applied before the right child starts (phase A, while the
-                                   tail goes out; default 100) */
+                                   tail goes out; default 50) */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */

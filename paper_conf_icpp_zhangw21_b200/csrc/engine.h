@@ -35,7 +35,7 @@ struct Options {
   int64_t colchunk = 1;      // column-chunked OOC node (RGSQR_OPT_COLCHUNK, R26)
   int64_t chunk_mib = 32;    // host-path column upload chunk (RGSQR_OPT_CHUNK_MIB)
   int64_t vshards = 1;       // virtual row shards on one GPU (RGSQR_OPT_VSHARDS, device path)
-  int64_t phasea_pct = 100;  // column-chunked node: % of the right child's first half projected before it
+  int64_t phasea_pct = 50;  // column-chunked node: % of the right child's first half projected before it
   int64_t defer_pieces = 0;  // deferred products in ~1/p of the node's A2 (RGSQR_OPT_DEFER_PIECES; 0 = upload chunks)
   int64_t eager_pct = 50;    // column-chunked node: the external projection is completed once the right
                              // child's leaves reach this % of its left half (RGSQR_OPT_EAGER_PCT)

@@ -233,7 +233,9 @@ struct Exec {
       if (col_end - flushed < cw && col_end < w) return;
       wait(sd, sc);
       int rc = d2h(Q, 0, m, c0 + flushed, col_end - flushed, D + flushed * m * s, m);
-      if (rc == 0) rc = d2h_r(c0, c0 + flushed, w, col_end - flushed, Rs + flushed * w, w);
+      // (rows [0, col_end) only: the rest of these columns is below the diagonal, zero, and the
+      // host zeroes R_out's strict lower triangle itself)
+      if (rc == 0) rc = d2h_r(c0, c0 + flushed, col_end, col_end - flushed, Rs + flushed * w, w);
       if (rc < 0) err = rc;
       flushed = col_end;
     };
