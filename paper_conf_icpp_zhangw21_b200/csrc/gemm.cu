@@ -65,7 +65,7 @@ template <typename T, bool kNN, int BN>
 __global__ void __launch_bounds__(128, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                 const __grid_constant__ CUtensorMap mapA2, const __grid_constant__ CUtensorMap mapB2,
-                const GemmParams p) {
+                const GemmParams p, const int group_m) {
   using C = GemmCfg<T, kNN, BN>;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = ptx::smem_u32(smem_raw);
@@ -77,7 +77,7 @@ __global__ void __launch_bounds__(128, 1)
 
   const int warp = threadIdx.x >> 5;
   int tm, tn;
-  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, p.group_m, &tm, &tn);
+  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, group_m, &tm, &tn);
   const int64_t m0 = (int64_t)tm * C::BM;
   const int64_t n0 = (int64_t)tn * BN;
   const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;
@@ -247,7 +247,7 @@ template <int BN>
 __global__ void __launch_bounds__(128 + 16 * 32, 1)
     tn_promote_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                       const __grid_constant__ CUtensorMap mapA2, const __grid_constant__ CUtensorMap mapB2,
-                      const GemmParams p) {
+                      const GemmParams p, const GemmExtra x) {
   using C = GemmCfg<float, false, BN>;
   static_assert(2 * BN <= 512, "two accumulators must fit TMEM");
   static_assert(BN == 128, "16 accumulation warps x 32 columns");
@@ -262,13 +262,13 @@ __global__ void __launch_bounds__(128 + 16 * 32, 1)
 
   const int warp = threadIdx.x >> 5;
   int tm, tn;
-  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, p.group_m, &tm, &tn);
+  grouped_tile(blockIdx.x, blockIdx.y, gridDim.x, gridDim.y, x.group_m, &tm, &tn);
   const int64_t m0 = (int64_t)tm * C::BM;
   const int64_t n0 = (int64_t)tn * BN;
   const int64_t kb0 = (int64_t)blockIdx.z * p.kb_per_split;
   const int64_t kb1 = min(p.kb_total, kb0 + p.kb_per_split);
   const int nkb = kb1 > kb0 ? (int)(kb1 - kb0) : 0;
-  const int pk = p.kb_per_unit > 0 ? (int)p.kb_per_unit : max(nkb, 1);
+  const int pk = x.kb_per_unit > 0 ? (int)x.kb_per_unit : max(nkb, 1);
   const int nunits = nkb > 0 ? (nkb + pk - 1) / pk : 0;
 
   if (warp == 0 && ptx::elect_one()) {
@@ -659,7 +659,8 @@ template cudaError_t launch_nn<float>(int, const CUtensorMap&, const CUtensorMap
 // ---------------------------------------------------------------------------------
 template <typename T, bool kNN, int BN>
 static cudaError_t launch_gemm_t(const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& ma2,
-                                 const CUtensorMap& mb2, const GemmParams& p, int splits, cudaStream_t st) {
+                                 const CUtensorMap& mb2, const GemmParams& p, int splits, cudaStream_t st,
+                                 int group_m) {
   using C = GemmCfg<T, kNN, BN>;
   static bool attr_set = false;
   if (!attr_set) {
@@ -669,13 +670,14 @@ static cudaError_t launch_gemm_t(const CUtensorMap& ma, const CUtensorMap& mb, c
     attr_set = true;
   }
   dim3 grid((unsigned)((p.M + C::BM - 1) / C::BM), (unsigned)((p.N + BN - 1) / BN), (unsigned)splits);
-  gemm_kernel<T, kNN, BN><<<grid, 128, C::SMEM, st>>>(ma, mb, ma2, mb2, p);
+  gemm_kernel<T, kNN, BN><<<grid, 128, C::SMEM, st>>>(ma, mb, ma2, mb2, p, group_m);
   return cudaGetLastError();
 }
 
 template <int BN>
 static cudaError_t launch_tn_promote_t(const CUtensorMap& ma, const CUtensorMap& mb, const CUtensorMap& ma2,
-                                       const CUtensorMap& mb2, const GemmParams& p, int splits, cudaStream_t st) {
+                                       const CUtensorMap& mb2, const GemmParams& p, int splits, cudaStream_t st,
+                                       const GemmExtra& x) {
   using C = GemmCfg<float, false, BN>;
   constexpr int SMEM = C::SMEM + 64;
   static bool attr_set = false;
@@ -685,28 +687,29 @@ static cudaError_t launch_tn_promote_t(const CUtensorMap& ma, const CUtensorMap&
     attr_set = true;
   }
   dim3 grid((unsigned)((p.M + C::BM - 1) / C::BM), (unsigned)((p.N + BN - 1) / BN), (unsigned)splits);
-  tn_promote_kernel<BN><<<grid, 128 + 16 * 32, SMEM, st>>>(ma, mb, ma2, mb2, p);
+  tn_promote_kernel<BN><<<grid, 128 + 16 * 32, SMEM, st>>>(ma, mb, ma2, mb2, p, x);
   return cudaGetLastError();
 }
 
 template <typename T>
 cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMap& mb,
                         const GemmParams& p, int splits, cudaStream_t st, const CUtensorMap* ma2,
-                        const CUtensorMap* mb2) {
+                        const CUtensorMap* mb2, GemmExtra x) {
   const CUtensorMap& a2 = ma2 ? *ma2 : ma;
   const CUtensorMap& b2 = mb2 ? *mb2 : mb;
   if constexpr (sizeof(T) == 4) {
-    if (!nn && p.kb_per_unit > 0)   // bounded accumulation chain (TF32X3), fp64 unit sums
-      return launch_tn_promote_t<128>(ma, mb, a2, b2, p, splits, st);
+    if (!nn && x.kb_per_unit > 0)   // bounded accumulation chain (TF32X3), fp64 unit sums
+      return launch_tn_promote_t<128>(ma, mb, a2, b2, p, splits, st, x);
   }
+  const int g = x.group_m;
   if (nn) {
-    if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, a2, b2, p, splits, st);
-    if (bn == 128) return launch_gemm_t<T, true, 128>(ma, mb, a2, b2, p, splits, st);
-    return launch_gemm_t<T, true, 64>(ma, mb, a2, b2, p, splits, st);
+    if (bn == 256) return launch_gemm_t<T, true, 256>(ma, mb, a2, b2, p, splits, st, g);
+    if (bn == 128) return launch_gemm_t<T, true, 128>(ma, mb, a2, b2, p, splits, st, g);
+    return launch_gemm_t<T, true, 64>(ma, mb, a2, b2, p, splits, st, g);
   }
-  if (bn == 256) return launch_gemm_t<T, false, 256>(ma, mb, a2, b2, p, splits, st);
-  if (bn == 128) return launch_gemm_t<T, false, 128>(ma, mb, a2, b2, p, splits, st);
-  return launch_gemm_t<T, false, 64>(ma, mb, a2, b2, p, splits, st);
+  if (bn == 256) return launch_gemm_t<T, false, 256>(ma, mb, a2, b2, p, splits, st, g);
+  if (bn == 128) return launch_gemm_t<T, false, 128>(ma, mb, a2, b2, p, splits, st, g);
+  return launch_gemm_t<T, false, 64>(ma, mb, a2, b2, p, splits, st, g);
 }
 
 // Many splits: a CTA owns 32 consecutive output elements (coalesced 128-byte reads of every
@@ -877,11 +880,11 @@ cudaError_t launch_trmm_upper(const float* S, int64_t lds, float* R, int64_t ldr
 }
 
 template cudaError_t launch_gemm<__half>(bool, int, const CUtensorMap&, const CUtensorMap&, const GemmParams&, int,
-                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*);
+                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*, GemmExtra);
 template cudaError_t launch_gemm<__nv_bfloat16>(bool, int, const CUtensorMap&, const CUtensorMap&, const GemmParams&, int,
-                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*);
+                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*, GemmExtra);
 template cudaError_t launch_gemm<float>(bool, int, const CUtensorMap&, const CUtensorMap&, const GemmParams&, int,
-                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*);
+                                   cudaStream_t, const CUtensorMap*, const CUtensorMap*, GemmExtra);
 template cudaError_t launch_splitk_reduce<__half>(const float*, int64_t, int64_t, int, float*, int64_t,
                                                   int, __half*, int64_t, int64_t, int64_t, cudaStream_t);
 template cudaError_t launch_splitk_reduce<__nv_bfloat16>(const float*, int64_t, int64_t, int, float*,

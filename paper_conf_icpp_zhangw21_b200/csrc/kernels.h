@@ -45,9 +45,13 @@ struct GemmParams {
   void* A2;
   int64_t lda2;
   int64_t kb_seg;           // > 0: K blocks per operand segment (TF32X3: hi.lo, lo.hi, hi.hi)
-  int group_m;              // > 1: grouped tile rasterization, this many M-tiles per group (gemm.cu)
-  int64_t kb_per_unit;      // > 0 (fp32 TN only): k-blocks per tensor-core accumulation chain, the
-                            // chains summed in fp32 registers (tn_promote_kernel, R25)
+};
+// Launch-side extras of the TN/NN GEMM launches (kept out of GemmParams: its layout is the kernel's
+// parameter block, and growing it measurably changed gemm_kernel's code generation)
+struct GemmExtra {
+  int group_m = 0;          // > 1: grouped tile rasterization, this many M-tiles per group (gemm.cu)
+  int64_t kb_per_unit = 0;  // > 0 (fp32 TN only): k-blocks per tensor-core accumulation chain, the
+                            // chains summed in fp64 registers (tn_promote_kernel, R25)
 };
 
 struct NNParams {
@@ -127,7 +131,7 @@ int leaf_max_smem_rows(int w);
 template <typename T>
 cudaError_t launch_gemm(bool nn, int bn, const CUtensorMap& ma, const CUtensorMap& mb,
                         const GemmParams& p, int splits, cudaStream_t st, const CUtensorMap* ma2 = nullptr,
-                        const CUtensorMap* mb2 = nullptr);
+                        const CUtensorMap* mb2 = nullptr, GemmExtra x = GemmExtra{});
 template <typename T>
 cudaError_t launch_splitk_reduce(const float* P, int64_t split_stride, int64_t ldp, int splits,
                                  float* C, int64_t ldc, int accumulate, T* Cop, int64_t ldop,

@@ -196,14 +196,15 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
   // grouped rasterization only pays on grids of many waves (e.g. the Table 1 shapes); on the
   // recursion's nodes (<= ~4 waves) the x-fastest order measured faster (RGSQR_GROUP_M overrides)
   static const int env_group = getenv("RGSQR_GROUP_M") ? atoi(getenv("RGSQR_GROUP_M")) : -1;
-  p.group_m = env_group >= 0 ? env_group : (tiles > 8 * (int64_t)c->num_sms ? 16 : 0);
+  GemmExtra gx;
+  gx.group_m = env_group >= 0 ? env_group : (tiles > 8 * (int64_t)c->num_sms ? 16 : 0);
   // One wave: tiles x splits <= SMs (rounding up put 152 CTAs on 148 SMs at w1 = w2 = 512 and
   // doubled the kernel time: 57 vs 37 us, profiles/r1_splitk_scan.txt).
   int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : c->num_sms / tiles);
   splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.kb_total / 4));
   // TF32X3: the tensor-core accumulation chain is bounded in-kernel (RGSQR_OPT_X3_CHAIN k-blocks per
   // TMEM chain, the chains summed in fp32 registers: tn_promote_kernel, R25)
-  if (x3) p.kb_per_unit = c->opt.x3_chain;
+  if (x3) gx.kb_per_unit = c->opt.x3_chain;
   const size_t cap = std::min<size_t>((size_t)64 << 20, c->arena.free_bytes());
   while (splits > 1 && (size_t)splits * w1 * w2 * 4 + 256 > cap) --splits;
   p.kb_per_split = (p.kb_total + splits - 1) / splits;
@@ -220,7 +221,7 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
     p.P = P;
     p.ldp = w1;
     p.split_stride = w1 * w2;
-    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, (int)splits, st, x3 ? &ma2 : nullptr, x3 ? &mb2 : nullptr));
+    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, (int)splits, st, x3 ? &ma2 : nullptr, x3 ? &mb2 : nullptr, gx));
     RGSQR_CUDA(c, launch_splitk_reduce<T>(P, w1 * w2, w1, (int)splits, R12, ldr, accumulate,
                                           static_cast<T*>(R12op), ldop, w1, w2, st));
     c->stats.n_other_launches++;
@@ -230,7 +231,7 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
     p.accumulate = accumulate;
     p.Cop = R12op;
     p.ldop = ldop;
-    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, 1, st, x3 ? &ma2 : nullptr, x3 ? &mb2 : nullptr));
+    RGSQR_CUDA(c, launch_gemm<T>(false, bn, ma, mb, p, 1, st, x3 ? &ma2 : nullptr, x3 ? &mb2 : nullptr, gx));
   }
   c->kend(1, st, kb, (x3 ? 6.0 : 2.0) * m * w1 * w2, (double)m * (w1 + w2) * s * (x3 ? 2 : 1) + 4.0 * w1 * w2);
   c->arena.release(mark);
