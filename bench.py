@@ -50,6 +50,12 @@ WORKLOADS = {
                desc="fp16 A 65536x8192 Gaussian, device budget 1 GiB (out-of-core), 1 GPU (BASELINE.json configs[1])"),
     "c3": dict(m=262144, n=32768, prec="fp16", budget=8 << 30,
                desc="fp16 A 262144x32768 Gaussian, device budget 8 GiB (BASELINE.json configs[2])"),
+    # the paper's whole-QR shapes (Table 4; memory-capped simulation PAPER.md:324):
+    # fp32 host data on TF32 tensor cores, device capped at 16 GiB, QR blocksize 8192 for --algo blocked
+    "t4a": dict(m=65536, n=65536, prec="tf32", budget=16 << 30,
+                desc="fp32 A 65536x65536 Gaussian, TF32, device budget 16 GiB (PAPER.md Table 4 shape)"),
+    "t4b": dict(m=262144, n=65536, prec="tf32", budget=16 << 30,
+                desc="fp32 A 262144x65536 Gaussian, TF32, device budget 16 GiB (PAPER.md Table 4 shape)"),
 }
 DTYPE_NAME = {"fp16": "f16", "bf16": "bf16", "tf32": "tf32"}
 STORAGE = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}
@@ -208,6 +214,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--skip-device", action="store_true", help="skip the HBM-resident secondary measurement")
+    ap.add_argument("--algo", default="recursive", choices=["recursive", "blocked"],
+                    help="blocked = the paper's conventional blocked OOC CGS (PAPER.md:113), panel 8192")
     ap.add_argument("--no-ablation", action="store_true", help="skip the split-ratio e2e ablation")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
@@ -256,7 +264,13 @@ def main():
     flops = 2.0 * m * n * n          # per rank's rows; the job's flops are world x this
     stream = torch.cuda.current_stream()
     h.set_stream(stream.cuda_stream)
-    tensor_peak = peaks["bf16_tflops_sustained"] * (0.5 if prec == "tf32" else 1.0)
+    if args.algo == "blocked":
+        h.set_option("algo", 1)
+        h.set_option("block_cols", 8192)
+    tf32_peak = json.load(open(os.path.join(ROOT, "profiles", "r2_probe.json"))).get("matmul_tf32_TFLOPs") \
+        if os.path.exists(os.path.join(ROOT, "profiles", "r2_probe.json")) else None
+    tensor_peak = peaks["bf16_tflops_sustained"] * (1.0 if prec != "tf32" else
+                                                    (tf32_peak / peaks["bf16_tflops"] if tf32_peak else 0.5))
 
     # ---- input (host, seeded; rank r holds global rows [r m, (r+1) m)) ----
     A = gi.gaussian(m, n, seed=2, dtype=st_name, row0=rank * ((m + gi.ROW_BLOCK - 1) // gi.ROW_BLOCK) * gi.ROW_BLOCK)
@@ -317,6 +331,7 @@ def main():
            "overlap_ratio": so["overlap_ratio"],
            "busy_ms": {"h2d": so["h2d_busy_ms"], "d2h": so["d2h_busy_ms"], "compute": so["compute_busy_ms"]},
            "ooc_nodes": so["n_ooc_nodes"], "arena_bytes": so["arena_bytes"],
+           "ctx_device_bytes": so["ctx_device_bytes"], "colchunk_nodes": so["n_colchunk_nodes"],
            "arena_high_water": so["arena_high_water"]}
     # ablation (not the headline): OOC left child 62.5% of the columns instead of the paper's halves
     if world == 1 and not args.no_ablation:
@@ -416,7 +431,7 @@ def main():
                 "config": {"workload": wl["desc"], "m": m, "n": n, "precision": prec, "device_budget_bytes": budget,
                            "value_path": "rgsqr_factor: A/Q/R in pinned host memory, out-of-core under the budget",
                            "l2": "inputs (>= 1 GiB) larger than L2 (126 MB); no flush needed",
-                           "parallelism": parallelism, "m_global": m * world},
+                           "parallelism": parallelism, "m_global": m * world, "algo": args.algo},
                 "roofline": roof, "e2e": e2e, "device_resident": dev, "kernel_roofline": kroof,
                 "cpu_baseline": cpu, "gpu_launches": args.steps * launches_per_step, "clocks": clocks.summary()}
         print(json.dumps(line), flush=True)

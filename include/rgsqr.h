@@ -26,9 +26,10 @@
  *   - Stored-value rounding (Q, updated A2', R12 used as an MMA operand) is
  *     round-to-nearest-even (reading R5).
  *   - Ownership: the caller owns every buffer it passes; the library never frees
- *     or reallocates them.  The library owns all device memory it allocates: a
- *     single arena of at most `device_mem_budget` bytes (0 = all free memory
- *     minus a 512 MiB reserve), so the budget is enforced by construction.
+ *     or reallocates them.  The library owns all device memory it allocates: a few
+ *     context-lifetime buffers (stats.ctx_device_bytes, ~3 MB) plus a single arena of
+ *     the rest of `device_mem_budget` (0 = all free memory minus a 512 MiB reserve),
+ *     so the budget is enforced by construction (NCCL's own buffers excepted).
  *   - Blocking: rgsqr_factor* return after Q and R are complete (host-synchronous).
  *     A handle is not thread-safe; use one handle per thread / per GPU.
  *   - Preconditions: 1 <= n <= m, lda >= m, lda*sizeof(elem) % 16 == 0, pointers
@@ -165,6 +166,8 @@ typedef struct rgsqr_stats {
   int64_t n_colchunk_nodes;     /* out-of-core nodes run column-chunked (RGSQR_OPT_COLCHUNK) */
   int64_t colchunk_tail_cols;   /* columns of those nodes projected from the host before the right
                                    child (they did not fit beside Q1) */
+  int64_t ctx_device_bytes;     /* context-lifetime device buffers (leaf exchange words, partials, ...):
+                                   counted against device_mem_budget, arena_bytes + this <= budget */
 } rgsqr_stats;
 
 /* ---- lifetime -------------------------------------------------------------------- */

@@ -89,7 +89,8 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   }
   auto t0 = std::chrono::steady_clock::now();
   const size_t ws = incore_workspace_bytes(c, prec, m, n);
-  const size_t cap = resolve_budget(c, budget);
+  size_t cap = resolve_budget(c, budget);
+  cap = cap > c->ctx_bytes ? cap - c->ctx_bytes : 0;   // context buffers count against the budget
   if (ws > cap) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "workspace " + std::to_string(ws) + " > budget");
   rc = ensure_arena(c, ws);
   if (rc < 0) return rc;
@@ -108,6 +109,7 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   c->stats.wall_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
   c->stats.arena_bytes = (int64_t)c->arena.size;
   c->stats.arena_high_water = (int64_t)c->arena.high;
+  c->stats.ctx_device_bytes = (int64_t)c->ctx_bytes;
   c->stats.flops = (int64_t)(2.0 * m * (double)n * n);
   if (brk == -2) {
     c->broken = true;
@@ -175,7 +177,8 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaStreamCreateWithFlags(&c->st_d2r, cudaStreamNonBlocking) != cudaSuccess ||
       cudaStreamCreateWithFlags(&c->st_h2d2, cudaStreamNonBlocking) != cudaSuccess ||
       cudaMalloc(&c->d_partials, sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024) != cudaSuccess ||
-      cudaMalloc(&c->d_sn_partials, sizeof(float) * LEAF_MAX_G * 128 * 128) != cudaSuccess ||
+      cudaMalloc(&c->d_sn_partials, sizeof(float) * LEAF_MAX_G * 64 * 64) != cudaSuccess ||
+      cudaMalloc(&c->d_shape, 64) != cudaSuccess ||
       cudaMalloc(&c->d_sn_r12op, 128 * 128 * 4) != cudaSuccess ||
       cudaMalloc(&c->d_counter, 4096) != cudaSuccess || cudaMalloc(&c->d_breakdown, 256) != cudaSuccess ||
       cudaMalloc(&c->d_xw, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
@@ -189,6 +192,13 @@ int create_impl(rgsqr_handle* h, int device) {
     delete c;
     return RGSQR_ERR_CUDA;
   }
+  // every context-lifetime device buffer counts against each call's device_mem_budget (the arena gets
+  // the budget minus these bytes, stats.ctx_device_bytes)
+  c->ctx_bytes = sizeof(float) * 2 * (LEAF_MAX_W + 2) * 1024 + sizeof(float) * LEAF_MAX_G * 64 * 64 + 128 * 128 * 4 +
+                 4096 + 256 + sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE +
+                 sizeof(unsigned long long) * LEAF_XW_WORDS + sizeof(void*) * 64 + sizeof(float) * (LEAF_MAX_W + 2) +
+                 64;
+  c->ctx_bytes = (c->ctx_bytes + 4095) / 4096 * 4096 + 10 * 512;   // (allocation granularity slack)
   reset_stats(c);
   *h = reinterpret_cast<rgsqr_handle>(c);
   return RGSQR_OK;
@@ -205,13 +215,11 @@ int sync_shape(Ctx* c, int64_t m, size_t* budget) {
   if (!c->nccl_comm) return RGSQR_OK;
   const size_t b = resolve_budget(c, *budget);
   int64_t h[3] = {m, -m, -(int64_t)b};
-  int64_t* d = nullptr;
-  if (cudaMalloc(&d, sizeof(h)) != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, "cudaMalloc");
+  int64_t* d = static_cast<int64_t*>(c->d_shape);   // (context buffer: no allocation per call)
   cudaMemcpy(d, h, sizeof(h), cudaMemcpyHostToDevice);
   const int rc = g_nccl.allReduce(d, d, 3, NCCL_INT64, /*ncclMax*/ 2, c->nccl_comm, c->compute());
   cudaMemcpyAsync(h, d, sizeof(h), cudaMemcpyDeviceToHost, c->compute());
   cudaStreamSynchronize(c->compute());
-  cudaFree(d);
   if (rc != 0) return fail(c, RGSQR_ERR_NCCL, "shape allreduce");
   if (h[0] != -h[1]) return fail(c, RGSQR_ERR_INVALID_ARG, "row-sharded run needs the same local m on every rank");
   *budget = (size_t)(-h[2]);
@@ -331,6 +339,7 @@ int rgsqr_destroy(rgsqr_handle h) {
   cudaFree(c->d_partials);
   cudaFree(c->d_sn_partials);
   cudaFree(c->d_sn_r12op);
+  cudaFree(c->d_shape);
   cudaFree(c->d_counter);
   cudaFree(c->d_breakdown);
   cudaFree(c->d_xw);

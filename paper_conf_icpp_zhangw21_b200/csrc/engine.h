@@ -86,7 +86,9 @@ struct Ctx {
   size_t arena_alloc_size = 0;
   // small persistent device buffers (leaf barrier/partials, breakdown flag)
   float* d_partials = nullptr;
-  float* d_sn_partials = nullptr;   // fused bottom node: [LEAF_MAX_G][4096] partials
+  float* d_sn_partials = nullptr;   // fused bottom node: [LEAF_MAX_G][64 x 64] partials (128-wide: arena)
+  void* d_shape = nullptr;          // distributed shape / budget agreement (3 int64)
+  size_t ctx_bytes = 0;             // all context-lifetime device bytes (count against every budget)
   void* d_sn_r12op = nullptr;       // fused bottom node: 64 x 64 operand copy
   unsigned int* d_counter = nullptr;        // [0] leaf round-0 barrier, [16] fused node barriers
   unsigned int counter_host[2] = {0, 0};     // their values after every enqueued barrier (never reset)

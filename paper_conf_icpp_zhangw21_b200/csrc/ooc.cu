@@ -884,9 +884,8 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   auto tp1 = std::chrono::steady_clock::now();
 
   // ---- device arena = the budget ----
-  const size_t persistent = (size_t)2 * (LEAF_MAX_W + 2) * 1024 * 4 + 512;
   size_t cap = resolve_budget(c, budget);
-  cap = cap > persistent ? cap - persistent : 0;
+  cap = cap > c->ctx_bytes ? cap - c->ctx_bytes : 0;   // context buffers count against the budget
   auto t0 = std::chrono::steady_clock::now();
   rc = ensure_arena(c, cap);
   if (rc < 0) {
@@ -953,6 +952,7 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   st.overlap_ratio = sum - mx > 1e-9 ? std::min(1.0, std::max(0.0, (sum - st.wall_ms) / (sum - mx))) : 0.0;
   st.arena_bytes = (int64_t)c->arena.size;
   st.arena_high_water = (int64_t)c->arena.high;
+  st.ctx_device_bytes = (int64_t)c->ctx_bytes;
   st.flops = (int64_t)(2.0 * m * (double)n * n);
   if (brk == -2) {
     c->broken = true;

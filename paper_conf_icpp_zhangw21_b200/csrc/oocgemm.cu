@@ -133,7 +133,8 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
       !pin(R12, ((size_t)ldr * (w2 - 1) + w1) * 4))
     return fail(c, RGSQR_ERR_HOST_MEM, "ooc gemm: cudaHostRegister failed");
   c->stats.pin_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tp0).count();
-  const size_t cap = resolve_budget(c, budget);
+  size_t cap = resolve_budget(c, budget);
+  cap = cap > c->ctx_bytes ? cap - c->ctx_bytes : 0;   // context buffers count against the budget
   int rc = ensure_arena(c, cap);
   if (rc < 0) return rc;
   Pipe P{c, c->compute(), c->st_h2d, c->st_d2h, s, {}};
@@ -318,6 +319,7 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
   st.overlap_ratio = sum - mx > 1e-9 ? std::min(1.0, std::max(0.0, (sum - st.wall_ms) / (sum - mx))) : 0.0;
   st.arena_bytes = (int64_t)c->arena.size;
   st.arena_high_water = (int64_t)c->arena.high;
+  st.ctx_device_bytes = (int64_t)c->ctx_bytes;
   st.flops = (int64_t)(2.0 * (double)m * w1 * w2);
   c->collect_kernel_stats();
   return RGSQR_OK;

@@ -570,6 +570,11 @@ int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64
   p.ldr = ldr;
   p.partials = c->d_sn_partials;
   p.r12op = c->d_sn_r12op;
+  const size_t mark = c->arena.mark();
+  if (W == 128) {   // the opt-in 128-wide instance: its partials come from the arena
+    p.partials = static_cast<float*>(c->arena.alloc((size_t)G * 128 * 128 * sizeof(float)));
+    if (!p.partials) return 0;   // (no room: the caller runs the separate products)
+  }
   p.counter = c->d_counter + 16;
   p.counter_host = &c->counter_host[1];
   p.r0_partials = r0_for_leaf ? c->d_partials : nullptr;
@@ -578,6 +583,7 @@ int op_small_node(Ctx* c, int prec, const void* Q1, int64_t ldq, void* A2, int64
   if (e != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, std::string("fused node launch: ") + cudaGetErrorString(e));
   c->kend(3, st, kb, 4.0 * m * w1 * w2, 2.0 * m * (w1 + w2) + 2.0 * m * w2 + 4.0 * w1 * w2);
   c->stats.n_other_launches++;
+  c->arena.release(mark);   // (stream-ordered reuse: later kernels on st run after this one)
   return r0_for_leaf ? 2 : 1;
 }
 

@@ -46,7 +46,8 @@ class Stats(C.Structure):
                 ("first_breakdown_col", C.c_int64), ("flops", C.c_int64),
                 ("kern_ms", C.c_double * 4), ("kern_launches", C.c_int64 * 4),
                 ("kern_flops", C.c_double * 4), ("kern_bytes", C.c_double * 4),
-                ("n_colchunk_nodes", C.c_int64), ("colchunk_tail_cols", C.c_int64)]
+                ("n_colchunk_nodes", C.c_int64), ("colchunk_tail_cols", C.c_int64),
+                ("ctx_device_bytes", C.c_int64)]
 
     def as_dict(self):
         out = {}

@@ -47,7 +47,7 @@ def test_c3_exact_dyadic_bitwise(h):
     del A
     gc.collect()
     assert rc == 0
-    assert st["n_ooc_nodes"] >= 3 and st["arena_bytes"] <= BUDGET
+    assert st["n_ooc_nodes"] >= 3 and st["arena_bytes"] + st["ctx_device_bytes"] <= BUDGET
     # R == R0: the band of R0 (bandwidth 4) and zeros elsewhere
     for j in range(N):
         lo = max(0, j - 4)

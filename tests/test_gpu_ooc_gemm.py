@@ -47,7 +47,7 @@ def test_ooc_inner(h, prec, tiling, block):
     bound = C[prec] * (np.abs(Xq).T @ np.abs(Xa))
     assert np.all(np.abs(R - ref) <= bound), np.max(np.abs(R - ref) / bound)
     s = h.stats()
-    assert s["arena_bytes"] <= budget and s["h2d_bytes"] >= Q.nbytes + A.nbytes
+    assert s["arena_bytes"] + s["ctx_device_bytes"] <= budget and s["h2d_bytes"] >= Q.nbytes + A.nbytes
 
 
 @pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
