@@ -41,7 +41,7 @@ def test_ooc_inner(h, prec, tiling, block):
     m, w1, w2 = 20000, 384, 520
     st, Q, A, Xq, Xa = _ops(prec, m, w1, w2, 3)
     R = np.full((w1, w2), np.nan, dtype=np.float32, order="F")
-    budget = 48 * MiB * (2 if st == "fp32" else 1)
+    budget = 56 * MiB * (2 if st == "fp32" else 1)
     h.ooc_inner(Q, m, A, m, m, w1, w2, R, w1, precision=prec, tiling=tiling, block=block, budget=budget)
     ref = Xq.T @ Xa
     bound = C[prec] * (np.abs(Xq).T @ np.abs(Xa))
