@@ -175,8 +175,10 @@ struct Exec {
     size_t next0 = 0;         // chunks before this index were already awaited by the compute stream
   };
 
+  // defer_final (with Rs_ext): the last Q / R columns' download is returned as a closure instead of
+  // issued, so that the caller can queue a more urgent copy ahead of it on the copy engine
   int incore_node(int64_t c0, int64_t w, bool src_q, char* D, bool resident, cudaEvent_t* q_done,
-                  float* Rs_ext = nullptr, Feed* feed = nullptr) {
+                  float* Rs_ext = nullptr, Feed* feed = nullptr, std::function<int()>* defer_final = nullptr) {
     const size_t mark = c->arena.mark();
     float* Rs = Rs_ext ? Rs_ext : static_cast<float*>(c->arena.alloc((size_t)w * w * 4));
     if (!Rs) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core node: no space for R block");
@@ -246,6 +248,23 @@ struct Exec {
     seg_end(2, sc, a);
     hk.need(w);  // (no-op unless the recursion skipped columns)
     wait(sd, sc);
+    if (defer_final && Rs_ext) {
+      cudaEvent_t ready = mark_ev(sc);
+      const int64_t f0 = flushed;
+      *defer_final = [this, ready, f0, c0, w, D, Rs_ext]() -> int {
+        cudaStreamWaitEvent(sd, ready, 0);
+        if (f0 < w) {
+          int r = d2h(Q, 0, m, c0 + f0, w - f0, D + f0 * m * s, m);
+          if (r < 0) return r;
+          r = d2h_r(c0, c0 + f0, w, w - f0, Rs_ext + f0 * w, w);
+          if (r < 0) return r;
+        }
+        return RGSQR_OK;
+      };
+      if (q_done) *q_done = nullptr;
+      c->arena.release(mark);
+      return RGSQR_OK;
+    }
     if (flushed < w) {
       rc = d2h(Q, 0, m, c0 + flushed, w - flushed, D + flushed * m * s, m);
       if (rc < 0) return rc;
@@ -598,9 +617,9 @@ struct Exec {
       // phase A: the right child's first half of head columns (E1) projected before it starts, in
       // pieces of pA columns (two fp32 R12 buffers + one operand buffer), while the tail goes out
       const int64_t E1 = std::min<int64_t>(wh, (hw * c->opt.phasea_pct / 100) / ch * ch);
-      const int64_t pA = std::max<int64_t>(ch, std::min<int64_t>(E1, 4 * ch));
+      const int64_t pA = std::max<int64_t>(ch, std::min<int64_t>(E1, 2 * ch));
       const size_t phaseA = (size_t)w1 * pA * (8 + s) + 1024;
-      const size_t htop = (std::max({left_ws, rs1 + tail_ws, phaseA}) + 4095) / 4096 * 4096;
+      const size_t htop = (std::max({left_ws, rs1 + tail_ws, rs1 + phaseA}) + 4095) / 4096 * 4096;
       if (htop > H || wt > w1) continue;
       P->wh = wh;
       P->wt1 = wt1;
@@ -655,11 +674,11 @@ struct Exec {
       return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the left R block");
     }
     cudaEvent_t q1_done = nullptr;
-    int rc = incore_node(c0, w1, src_q, D, false, &q1_done, Rs1);
+    std::function<int()> left_final;   // the left child's last Q / R download, queued after the tail's
+    int rc = incore_node(c0, w1, src_q, D, false, &q1_done, Rs1, nullptr, &left_final);
     unwindow(wsave);
     if (rc < 0) return rc;
     cudaEvent_t left_done = mark_ev(sc);
-    cudaEvent_t left_r = r_done;
     // ---- uploads queued behind the left child's: tail piece 1, then the head clear of H's top ----
     cudaEvent_t ev_t1 = nullptr, ev_t2 = nullptr;
     if (wt1 > 0) {
@@ -727,6 +746,11 @@ struct Exec {
       if (rc < 0) return rc;
     }
     cudaEvent_t tail_out = mark_ev(sd);
+    // now the left child's last columns (nothing waits on them but the end of the call and the reuse of
+    // H's top, which holds its R block)
+    if (left_final && (rc = left_final()) < 0) return rc;
+    cudaEvent_t left_r = r_done;
+    cudaEvent_t left_q = mark_ev(sd);
     // ---- phase A: the first E1 head columns' projection in one piece (buffers at the bottom of H's
     //      top, once the left R block is downloaded), while the tail goes out ----
     ExtProduct ext;
@@ -750,8 +774,9 @@ struct Exec {
     cudaEvent_t phaseA_r[2] = {nullptr, nullptr};
     if (E1 > 0) {
       const int64_t pA = std::min<int64_t>(P.pA, E1);
-      if (left_r) cudaStreamWaitEvent(sc, left_r, 0);
-      wsave = window(Htop, Hend);
+      // (above the left R block, still downloading; over the tail's R12, which must be out)
+      if (r12t_out) cudaStreamWaitEvent(sc, r12t_out, 0);
+      wsave = window(Htop + ((size_t)w1 * w1 * 4 + 255) / 256 * 256, Hend);
       ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * pA * 4));
       ext.R12[1] = static_cast<float*>(c->arena.alloc((size_t)w1 * pA * 4));
       ext.R12op = c->arena.alloc((size_t)w1 * pA * s);
@@ -769,6 +794,8 @@ struct Exec {
     // the rest of the head goes into H's top once the tail phase and phase A have released it
     cudaStreamWaitEvent(sh, phaseA_done, 0);
     cudaStreamWaitEvent(sh, tail_out, 0);
+    if (left_r) cudaStreamWaitEvent(sh, left_r, 0);
+    cudaStreamWaitEvent(sh, left_q, 0);
     if (r12t_out) cudaStreamWaitEvent(sh, r12t_out, 0);
     for (cudaEvent_t e : phaseA_r)
       if (e) cudaStreamWaitEvent(sh, e, 0);
