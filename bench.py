@@ -181,7 +181,9 @@ def run_reference(args, wl, rank):
     if rank != 0:
         return
     m, n, prec = wl["m"], wl["n"], wl["prec"]
-    cols = 512
+    # the same 2048-column sample as our arm's cpu_baseline (~9 s per step on 16 cores; the whole
+    # configs[1] run is recorded separately in profiles/r2_cpu_oracle_c2.json)
+    cols = min(n, 2048)
     A = gi.gaussian(m, cols, seed=2, dtype=STORAGE[prec])
     cores = len(os.sched_getaffinity(0))
     for _ in range(args.warmup):
@@ -200,7 +202,10 @@ def run_reference(args, wl, rank):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": wl["desc"], "m": m, "n": n, "precision": prec,
                        "device_budget_bytes": wl["budget"], "sample_cols": cols},
-            "cpu_baseline": {"value": value, "unit": "TFLOPS", "cores": cores, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "TFLOPS", "cores": cores, "kind": "oracle", "sample": sample,
+                             **({"full_c2_measured": json.load(open(os.path.join(ROOT, "profiles", "r2_cpu_oracle_c2.json")))}
+                                if args.workload == "c2" and os.path.exists(os.path.join(ROOT, "profiles", "r2_cpu_oracle_c2.json"))
+                                else {})},
             "e2e": {"value": value, "unit": "TFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 

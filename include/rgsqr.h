@@ -70,7 +70,9 @@ enum rgsqr_option {
   RGSQR_OPT_TILE_ROWS_MIN = 2,  /* OOC row-tile ramp start (paper: 2048; default 4096) */
   RGSQR_OPT_TILE_ROWS_MAX = 3,  /* OOC row-tile cap (paper: 8192/16384; default 16384) */
   RGSQR_OPT_RING_DEPTH = 4,     /* K device slots per OOC stream ring (>= 2, default 3) */
-  RGSQR_OPT_ALGO = 5,           /* 0 = recursive (Eq. 2, default), 1 = blocked */
+  RGSQR_OPT_ALGO = 5,           /* 0 = recursive (Eq. 2, default), 1 = blocked with the
+                                   paper's OOC GEMM tilings, 2 = fused blocked: panel resident, trailing
+                                   matrix streamed in column blocks read and written once per panel */
   RGSQR_OPT_BLOCK_COLS = 6,     /* panel width b of the blocked algorithm (default 8192) */
   RGSQR_OPT_SERIALIZE = 7,      /* 1 = one stream, no overlap (the paper's "Synchronous" rows) */
   RGSQR_OPT_REUSE = 8,          /* 1 = QR-level data reuse, default 1 */

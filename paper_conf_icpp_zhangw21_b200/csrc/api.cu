@@ -577,7 +577,7 @@ int rgsqr_set_option(rgsqr_handle h, int key, int64_t value) {
     case RGSQR_OPT_TILE_ROWS_MIN:
     case RGSQR_OPT_TILE_ROWS_MAX: if (value < 128 || value % 128) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_RING_DEPTH: if (value < 2 || value > 16) return RGSQR_ERR_INVALID_ARG; break;
-    case RGSQR_OPT_ALGO: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_ALGO: if (value < 0 || value > 2) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_REORTH: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_COLCHUNK: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_EAGER_PCT:

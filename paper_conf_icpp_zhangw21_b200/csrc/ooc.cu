@@ -867,6 +867,72 @@ struct Exec {
     }
     return RGSQR_OK;
   }
+
+  // fused blocked algorithm (RGSQR_OPT_ALGO = 2; SURVEY.md 8(f) f1 "honesty" variant and f4's
+  // "fused-blocked top level"): the blocked loop of PAPER.md:113, but the panel Q stays resident and
+  // the trailing matrix streams through in COLUMN blocks, each read once and written once per panel:
+  // R12_j = Q^T A2_j and A2_j -= Q R12_j on the block while it is on the device (Fig. 4's inner tiling
+  // fused with the outer update).  Per panel i the trailing (n - ib) columns move once each way, so the
+  // whole factorization moves ~ (k+1)/2 m n words each way for k panels.
+  int fused_blocked(int64_t b) {
+    for (int64_t c0 = 0; c0 < n; c0 += b) {
+      const int64_t w1 = std::min(b, n - c0), rest = n - c0 - w1;
+      const bool src_q = c0 > 0;   // after the first panel the working matrix is the host Q copy
+      const size_t mark = c->arena.mark();
+      char* D = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
+      if (!D || c->arena.free_bytes() < incore_need(w1) - (size_t)m * w1 * s)
+        return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "fused blocked: panel of " + std::to_string(w1) + " columns does not fit");
+      cudaEvent_t q_done = nullptr;
+      int rc = incore_node(c0, w1, src_q, D, false, &q_done);
+      if (rc < 0) return rc;
+      if (rest > 0) {
+        c->stats.n_ooc_nodes++;
+        // K column-block slots: A2 block (m x cb), its R12 (fp32) and operand copy
+        const size_t per_col = (size_t)m * s + (size_t)w1 * (4 + s);
+        const size_t ws = (size_t)16 << 20;   // split-K partials of the per-block products
+        const size_t fr = c->arena.free_bytes();
+        int64_t cb = fr > ws ? (int64_t)((fr - ws) / ((size_t)K * per_col)) : 0;
+        cb = std::min<int64_t>(cb, rest);
+        if (cb >= 64) cb = cb / 64 * 64;
+        if (cb < 8) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "fused blocked: no room for column blocks");
+        const size_t slot_b = ((size_t)m * cb * s + 255) / 256 * 256, rb = ((size_t)w1 * cb * 4 + 255) / 256 * 256;
+        char* ring = static_cast<char*>(c->arena.alloc((size_t)K * (slot_b + rb + (size_t)w1 * cb * s + 256)));
+        if (!ring) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "fused blocked: ring");
+        std::vector<cudaEvent_t> freed(K, nullptr);
+        const int64_t h = c0 + w1;
+        int64_t j = 0;
+        for (int64_t a = 0; a < rest; a += cb, ++j) {
+          const int64_t cw = std::min(cb, rest - a);
+          const int k = (int)(j % K);
+          char* sa = ring + (size_t)k * (slot_b + rb + (size_t)w1 * cb * s + 256);
+          float* sr = reinterpret_cast<float*>(sa + slot_b);
+          char* so = sa + slot_b + rb;
+          if (freed[k]) {
+            cudaStreamWaitEvent(sh, freed[k], 0);
+            cudaStreamWaitEvent(sc, freed[k], 0);
+          }
+          if ((rc = h2d(sa, m, hsrc(src_q), 0, m, h + a, cw)) < 0) return rc;
+          cudaStreamWaitEvent(sc, mark_ev(sh), 0);
+          cudaEvent_t seg = seg_begin(sc);
+          rc = op_inner(c, prec, D, m, sa, m, m, w1, cw, sr, w1, so, w1, 0, sc);
+          if (rc < 0) return rc;
+          if ((rc = d2h_r(c0, h + a, w1, cw, sr, w1)) < 0) return rc;
+          cudaEvent_t r_out = r_done;
+          rc = op_outer(c, prec, D, m, so, w1, sa, m, m, w1, cw, sc);
+          if (rc < 0) return rc;
+          seg_end(2, sc, seg);
+          wait(sd, sc);
+          if ((rc = d2h(Q, 0, m, h + a, cw, sa, m)) < 0) return rc;
+          cudaEvent_t out = mark_ev(sd);
+          if (r_out) cudaStreamWaitEvent(sd, r_out, 0);   // (the slot's R12 is out too)
+          freed[k] = r_out ? mark_ev(sd) : out;
+        }
+      }
+      join_all();
+      c->arena.release(mark);
+    }
+    return RGSQR_OK;
+  }
 };
 
 }  // namespace
@@ -934,7 +1000,9 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
     zero = std::thread([R, n] {
       for (int64_t j = 0; j + 1 < n; ++j) std::memset(R + j * n + j + 1, 0, (size_t)(n - j - 1) * 4);
     });
-  rc = c->opt.algo == 1 ? x.blocked(std::min<int64_t>(c->opt.block_cols, n)) : x.node(0, n, false);
+  rc = c->opt.algo == 1   ? x.blocked(std::min<int64_t>(c->opt.block_cols, n))
+       : c->opt.algo == 2 ? x.fused_blocked(std::min<int64_t>(c->opt.block_cols, n))
+                          : x.node(0, n, false);
   int brk = INT_MAX;
   if (rc >= 0) {
     x.join_all();

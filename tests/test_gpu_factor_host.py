@@ -268,3 +268,30 @@ def test_host_alloc_numa_buffers(h):
         h.host_free(p_)
     with pytest.raises(RgsqrError):
         h.host_free(pa)
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+def test_fused_blocked_algorithm(h, prec):
+    """RGSQR_OPT_ALGO = 2 (fused blocked, SURVEY.md 8(f) f1 honesty variant): the blocked loop of
+    PAPER.md:113 with the panel resident and the trailing matrix read and written once per panel in
+    column blocks.  Against the oracle, exact-dyadic bitwise, and its byte count: each direction moves
+    m s sum_i (n - i b) = m n s (k + 1) / 2 for k = n / b panels."""
+    st = STOR[prec]
+    m, n, b = 16384, 1024, 256
+    s = 4 if st == "fp32" else 2
+    budget = (24 if s == 2 else 48) * MiB
+    A = gi.gaussian(m, n, seed=51, dtype=st)
+    X = gi.to_float64(A, st)
+    rc, Q, R, stt = factor(h, A, prec, budget, algo=2, block_cols=b)
+    assert rc == 0
+    Rg = R.astype(np.float64)
+    ref = oracle.rgs(X, leaf=64)
+    assert oracle.backward_error(X, gi.to_float64(Q, st), Rg) < 5e-3
+    assert oracle.r_rel_error(Rg, ref.R) < 5e-3
+    k = n // b
+    assert stt["h2d_matrix_bytes"] == m * n * s * (k + 1) // 2
+    assert stt["d2h_matrix_bytes"] == m * n * s * (k + 1) // 2
+    A64, R0 = gi.dyadic_mixed(m, n, seed=52)
+    rc, Q, R, _ = factor(h, gi.to_storage(A64, st), prec, budget, algo=2, block_cols=b)
+    np.testing.assert_array_equal(R.astype(np.float64), R0)
+    np.testing.assert_array_equal(gi.to_float64(Q, st), gi.hadamard(m, n))
