@@ -889,8 +889,8 @@ struct Exec {
         c->stats.n_ooc_nodes++;
         // K column-block slots: A2 block (m x cb), its R12 (fp32) and operand copy
         const size_t per_col = (size_t)m * s + (size_t)w1 * (4 + s);
-        const size_t ws = (size_t)16 << 20;   // split-K partials of the per-block products
         const size_t fr = c->arena.free_bytes();
+        const size_t ws = std::min<size_t>((size_t)16 << 20, fr / 4);   // split-K partials of the block products
         int64_t cb = fr > ws ? (int64_t)((fr - ws) / ((size_t)K * per_col)) : 0;
         cb = std::min<int64_t>(cb, rest);
         if (cb >= 64) cb = cb / 64 * 64;

@@ -36,7 +36,7 @@ RUNS = {
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--which", default="c3")
-    ap.add_argument("--algos", default="recursive,blocked")
+    ap.add_argument("--algos", default="recursive,blocked,fused")
     ap.add_argument("--out", default="gpurun_out/paper_runs.json")
     a = ap.parse_args()
     h = Handle(0)
@@ -55,7 +55,7 @@ def main():
         gi.gaussian(m, n, seed=3, dtype=st, out=A)
         gen_s = time.time() - t0
         for algo in a.algos.split(","):
-            h.set_option("algo", 1 if algo == "blocked" else 0)
+            h.set_option("algo", {"recursive": 0, "blocked": 1, "fused": 2}[algo])
             h.set_option("block_cols", cfg["block"])
             h.factor(pa, m, m, n, pq, pr, precision=cfg["prec"], budget=cfg["budget"])   # warm-up
             s = h.stats()
