@@ -619,7 +619,8 @@ struct Exec {
       const int64_t E1 = std::min<int64_t>(wh, (hw * c->opt.phasea_pct / 100) / ch * ch);
       const int64_t pA = std::max<int64_t>(ch, std::min<int64_t>(E1, 2 * ch));
       const size_t phaseA = (size_t)w1 * pA * (8 + s) + 1024;
-      const size_t htop = (std::max({left_ws, rs1 + tail_ws, rs1 + phaseA}) + 4095) / 4096 * 4096;
+      const size_t t2 = (size_t)wt2 * colb + 256;
+      const size_t htop = (std::max({left_ws, rs1 + tail_ws, rs1 + t2 + phaseA}) + 4095) / 4096 * 4096;
       if (htop > H || wt > w1) continue;
       P->wh = wh;
       P->wt1 = wt1;
@@ -698,11 +699,15 @@ struct Exec {
     };
     // ---- 2. the tail: workspace and second piece in the top of H, above the left R block (so that
     //      nothing waits for that block's download) ----
-    wsave = window(Htop + ((size_t)w1 * w1 * 4 + 255) / 256 * 256, Hend);
+    // (T2 first: phase A's buffers later go above T2 -- T2 is downloaded while phase A runs -- and over
+    // the tail's R12 buffers, whose use is over by then)
+    const size_t rs1b = ((size_t)w1 * w1 * 4 + 255) / 256 * 256;
+    wsave = window(Htop + rs1b, Hend);
+    char* T2 = wt2 > 0 ? static_cast<char*>(c->arena.alloc(colb * wt2)) : nullptr;
     float* R12t = static_cast<float*>(c->arena.alloc((size_t)w1 * wt * 4));
     char* R12top = static_cast<char*>(c->arena.alloc((size_t)w1 * wt * s));
-    char* T2 = wt2 > 0 ? static_cast<char*>(c->arena.alloc(colb * wt2)) : nullptr;
     unwindow(wsave);
+    const size_t t2b = wt2 > 0 ? (colb * wt2 + 255) / 256 * 256 : 0;
     if (!R12t || !R12top || (wt2 > 0 && !T2))
       return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "column-chunked node: no space for the tail products");
     int64_t a_head = 0;
@@ -774,9 +779,9 @@ struct Exec {
     cudaEvent_t phaseA_r[2] = {nullptr, nullptr};
     if (E1 > 0) {
       const int64_t pA = std::min<int64_t>(P.pA, E1);
-      // (above the left R block, still downloading; over the tail's R12, which must be out)
+      // (above the left R block and T2, both still downloading; over the tail's R12, which must be out)
       if (r12t_out) cudaStreamWaitEvent(sc, r12t_out, 0);
-      wsave = window(Htop + ((size_t)w1 * w1 * 4 + 255) / 256 * 256, Hend);
+      wsave = window(Htop + rs1b + t2b, Hend);
       ext.R12[0] = static_cast<float*>(c->arena.alloc((size_t)w1 * pA * 4));
       ext.R12[1] = static_cast<float*>(c->arena.alloc((size_t)w1 * pA * 4));
       ext.R12op = c->arena.alloc((size_t)w1 * pA * s);
