@@ -594,7 +594,7 @@ struct Exec {
     int64_t pB = 0;                  // piece width of the remaining projection (phase B)
   };
   bool plan_cc(int64_t w1, int64_t w2, size_t free0, CCPlan* P) const {
-    if (w2 > w1 || (m * s * 64) % 256 != 0) return false;
+    if ((m * s * 64) % 256 != 0) return false;   // (the tail must fit D: wt <= w1, checked below)
     const int64_t leaf = std::max(1, leaf_width_for(c, m));
     int64_t cw = (c->opt.chunk_mib << 20) / std::max<int64_t>(1, m * s);
     cw = std::max<int64_t>(leaf, cw / 64 * 64);
