@@ -234,8 +234,7 @@ struct Exec {
       }
       if (col_end - flushed < cw && col_end < w) return;
       wait(sd, sc);
-      // (defer_final: the Q columns stay on the device and go out with the final closure)
-      int rc = defer_final ? RGSQR_OK : d2h(Q, 0, m, c0 + flushed, col_end - flushed, D + flushed * m * s, m);
+      int rc = d2h(Q, 0, m, c0 + flushed, col_end - flushed, D + flushed * m * s, m);
       // (rows [0, col_end) only: the rest of these columns is below the diagonal, zero, and the
       // host zeroes R_out's strict lower triangle itself)
       if (rc == 0) rc = d2h_r(c0, c0 + flushed, col_end, col_end - flushed, Rs + flushed * w, w);
@@ -250,19 +249,14 @@ struct Exec {
     hk.need(w);  // (no-op unless the recursion skipped columns)
     wait(sd, sc);
     if (defer_final && Rs_ext) {
-      // the node's Q (all of it: the leaf_done flushes sent only R) and its last R columns, as a
-      // closure the caller queues when the copy engine should take them
       cudaEvent_t ready = mark_ev(sc);
       const int64_t f0 = flushed;
       *defer_final = [this, ready, f0, c0, w, D, Rs_ext]() -> int {
         cudaStreamWaitEvent(sd, ready, 0);
         if (f0 < w) {
-          int r = d2h_r(c0, c0 + f0, w, w - f0, Rs_ext + f0 * w, w);
+          int r = d2h(Q, 0, m, c0 + f0, w - f0, D + f0 * m * s, m);
           if (r < 0) return r;
-        }
-        const int64_t qc = std::max<int64_t>(1, ((int64_t)32 << 20) / std::max<int64_t>(1, m * s));
-        for (int64_t a = 0; a < w; a += qc) {   // (in 32 MiB pieces: other copies can interleave)
-          int r = d2h(Q, 0, m, c0 + a, std::min(qc, w - a), D + a * m * s, m);
+          r = d2h_r(c0, c0 + f0, w, w - f0, Rs_ext + f0 * w, w);
           if (r < 0) return r;
         }
         return RGSQR_OK;
@@ -761,7 +755,7 @@ struct Exec {
     // H's top, which holds its R block)
     if (left_final && (rc = left_final()) < 0) return rc;
     cudaEvent_t left_r = r_done;
-    cudaEvent_t left_q = mark_ev(sd);   // Q1 is on the host (D may be overwritten after this)
+    cudaEvent_t left_q = mark_ev(sd);
     // ---- phase A: the first E1 head columns' projection in one piece (buffers at the bottom of H's
     //      top, once the left R block is downloaded), while the tail goes out ----
     ExtProduct ext;
@@ -806,6 +800,7 @@ struct Exec {
     cudaStreamWaitEvent(sh, phaseA_done, 0);
     cudaStreamWaitEvent(sh, tail_out, 0);
     if (left_r) cudaStreamWaitEvent(sh, left_r, 0);
+    cudaStreamWaitEvent(sh, left_q, 0);
     if (r12t_out) cudaStreamWaitEvent(sh, r12t_out, 0);
     for (cudaEvent_t e : phaseA_r)
       if (e) cudaStreamWaitEvent(sh, e, 0);
@@ -833,7 +828,6 @@ struct Exec {
       cudaEvent_t q1_dead = mark_ev(sc);
       cudaStreamWaitEvent(sh, q1_dead, 0);
       cudaStreamWaitEvent(sh, tail_out, 0);
-      cudaStreamWaitEvent(sh, left_q, 0);   // Q1 itself went out after the tail (deferred download)
       if (h2d(D, m, Q, 0, m, h + wh, wt) < 0) return;
       feed.chunks.back().second = mark_ev(sh);
     };
