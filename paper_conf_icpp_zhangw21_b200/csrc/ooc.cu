@@ -177,8 +177,11 @@ struct Exec {
 
   // defer_final (with Rs_ext): the last Q / R columns' download is returned as a closure instead of
   // issued, so that the caller can queue a more urgent copy ahead of it on the copy engine
+  // defer_q_cols (with defer_final): the Q of the node's last defer_q_cols columns also waits for the
+  // closure (the caller queues a more urgent copy ahead of it)
   int incore_node(int64_t c0, int64_t w, bool src_q, char* D, bool resident, cudaEvent_t* q_done,
-                  float* Rs_ext = nullptr, Feed* feed = nullptr, std::function<int()>* defer_final = nullptr) {
+                  float* Rs_ext = nullptr, Feed* feed = nullptr, std::function<int()>* defer_final = nullptr,
+                  int64_t defer_q_cols = 0) {
     const size_t mark = c->arena.mark();
     float* Rs = Rs_ext ? Rs_ext : static_cast<float*>(c->arena.alloc((size_t)w * w * 4));
     if (!Rs) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "in-core node: no space for R block");
@@ -234,7 +237,10 @@ struct Exec {
       }
       if (col_end - flushed < cw && col_end < w) return;
       wait(sd, sc);
-      int rc = d2h(Q, 0, m, c0 + flushed, col_end - flushed, D + flushed * m * s, m);
+      const int64_t qdefer = defer_final ? w - defer_q_cols : w;   // Q columns >= qdefer: in the closure
+      int rc = flushed >= qdefer ? RGSQR_OK
+                                 : d2h(Q, 0, m, c0 + flushed, std::min(col_end, qdefer) - flushed,
+                                       D + flushed * m * s, m);
       // (rows [0, col_end) only: the rest of these columns is below the diagonal, zero, and the
       // host zeroes R_out's strict lower triangle itself)
       if (rc == 0) rc = d2h_r(c0, c0 + flushed, col_end, col_end - flushed, Rs + flushed * w, w);
@@ -250,13 +256,15 @@ struct Exec {
     wait(sd, sc);
     if (defer_final && Rs_ext) {
       cudaEvent_t ready = mark_ev(sc);
-      const int64_t f0 = flushed;
-      *defer_final = [this, ready, f0, c0, w, D, Rs_ext]() -> int {
+      const int64_t f0 = flushed, q0 = std::min(flushed, std::max<int64_t>(0, w - defer_q_cols));
+      *defer_final = [this, ready, f0, q0, c0, w, D, Rs_ext]() -> int {
         cudaStreamWaitEvent(sd, ready, 0);
         if (f0 < w) {
-          int r = d2h(Q, 0, m, c0 + f0, w - f0, D + f0 * m * s, m);
+          int r = d2h_r(c0, c0 + f0, w, w - f0, Rs_ext + f0 * w, w);
           if (r < 0) return r;
-          r = d2h_r(c0, c0 + f0, w, w - f0, Rs_ext + f0 * w, w);
+        }
+        if (q0 < w) {
+          int r = d2h(Q, 0, m, c0 + q0, w - q0, D + q0 * m * s, m);
           if (r < 0) return r;
         }
         return RGSQR_OK;
@@ -676,7 +684,10 @@ struct Exec {
     }
     cudaEvent_t q1_done = nullptr;
     std::function<int()> left_final;   // the left child's last Q / R download, queued after the tail's
-    int rc = incore_node(c0, w1, src_q, D, false, &q1_done, Rs1, nullptr, &left_final);
+    // (RGSQR_DEFER_Q_CHUNKS > 0: the Q of its last few upload chunks too, queued behind the tail's
+    // download -- measured slower at configs[1]: 37.6 / 37.9 / 38.6 ms for 3 / 4 / 6 chunks vs 37.1)
+    static const int64_t dq_env = getenv("RGSQR_DEFER_Q_CHUNKS") ? atoll(getenv("RGSQR_DEFER_Q_CHUNKS")) : 0;
+    int rc = incore_node(c0, w1, src_q, D, false, &q1_done, Rs1, nullptr, &left_final, dq_env * ch);
     unwindow(wsave);
     if (rc < 0) return rc;
     cudaEvent_t left_done = mark_ev(sc);
@@ -799,8 +810,7 @@ struct Exec {
     // the rest of the head goes into H's top once the tail phase and phase A have released it
     cudaStreamWaitEvent(sh, phaseA_done, 0);
     cudaStreamWaitEvent(sh, tail_out, 0);
-    if (left_r) cudaStreamWaitEvent(sh, left_r, 0);
-    cudaStreamWaitEvent(sh, left_q, 0);
+    if (left_r) cudaStreamWaitEvent(sh, left_r, 0);   // (H's top held the left R block)
     if (r12t_out) cudaStreamWaitEvent(sh, r12t_out, 0);
     for (cudaEvent_t e : phaseA_r)
       if (e) cudaStreamWaitEvent(sh, e, 0);
@@ -828,6 +838,7 @@ struct Exec {
       cudaEvent_t q1_dead = mark_ev(sc);
       cudaStreamWaitEvent(sh, q1_dead, 0);
       cudaStreamWaitEvent(sh, tail_out, 0);
+      cudaStreamWaitEvent(sh, left_q, 0);   // (Q1's deferred last columns are on the host)
       if (h2d(D, m, Q, 0, m, h + wh, wt) < 0) return;
       feed.chunks.back().second = mark_ev(sh);
     };
