@@ -188,7 +188,10 @@ int create_impl(rgsqr_handle* h, int device) {
       cudaMemset(c->d_xw, 0, sizeof(unsigned long long) * LEAF_XW_WORDS * LEAF_XW_STRIDE) != cudaSuccess ||
       cudaMemset(c->d_xprev, 0, sizeof(unsigned long long) * LEAF_XW_WORDS) != cudaSuccess ||
       cudaMemset(c->d_counter, 0, 4096) != cudaSuccess ||
-      cudaMemcpy(c->d_peers, &c->d_xw, sizeof(void*), cudaMemcpyHostToDevice) != cudaSuccess) {
+      cudaMemcpy(c->d_peers, &c->d_xw, sizeof(void*), cudaMemcpyHostToDevice) != cudaSuccess ||
+      // (cudaMemset / pageable cudaMemcpy may return before the device write lands, and the work
+      // streams are non-blocking: drain the device before any of them can read these buffers)
+      cudaDeviceSynchronize() != cudaSuccess) {
     delete c;
     return RGSQR_ERR_CUDA;
   }
@@ -216,7 +219,9 @@ int sync_shape(Ctx* c, int64_t m, size_t* budget) {
   const size_t b = resolve_budget(c, *budget);
   int64_t h[3] = {m, -m, -(int64_t)b};
   int64_t* d = static_cast<int64_t*>(c->d_shape);   // (context buffer: no allocation per call)
-  cudaMemcpy(d, h, sizeof(h), cudaMemcpyHostToDevice);
+  // stream-ordered: a pageable cudaMemcpy may return before its DMA lands, and the compute stream
+  // is non-blocking -- the allreduce could then reduce (and we read back) the previous call's values
+  cudaMemcpyAsync(d, h, sizeof(h), cudaMemcpyHostToDevice, c->compute());
   const int rc = g_nccl.allReduce(d, d, 3, NCCL_INT64, /*ncclMax*/ 2, c->nccl_comm, c->compute());
   cudaMemcpyAsync(h, d, sizeof(h), cudaMemcpyDeviceToHost, c->compute());
   cudaStreamSynchronize(c->compute());
@@ -301,7 +306,7 @@ static int create_dist_impl(Ctx* c, int rank, int nranks, const unsigned char id
     char* dbuf = nullptr;
     const size_t hs = sizeof(cudaIpcMemHandle_t);
     if (cudaMalloc(&dbuf, hs * (nranks + 1)) != cudaSuccess) return fail(c, RGSQR_ERR_CUDA, "cudaMalloc");
-    cudaMemcpy(dbuf + hs * nranks, &mine, hs, cudaMemcpyHostToDevice);
+    cudaMemcpyAsync(dbuf + hs * nranks, &mine, hs, cudaMemcpyHostToDevice, c->st_own);
     if (g_nccl.allGather(dbuf + hs * nranks, dbuf, hs, /*ncclChar*/ 0, c->nccl_comm, c->st_own) != 0) {
       cudaFree(dbuf);
       return fail(c, RGSQR_ERR_NCCL, "ncclAllGather of IPC handles");
@@ -319,10 +324,10 @@ static int create_dist_impl(Ctx* c, int rank, int nranks, const unsigned char id
       c->ipc_opened.push_back(ptr);
     }
   }
-  cudaMemcpy(c->d_peers, peers.data(), sizeof(void*) * nranks, cudaMemcpyHostToDevice);
+  cudaMemcpyAsync(c->d_peers, peers.data(), sizeof(void*) * nranks, cudaMemcpyHostToDevice, c->st_own);
   // every rank has zeroed its words (create_impl) before anyone may add into them
   float one = 0.f;
-  cudaMemcpy(c->d_r0buf, &one, sizeof(float), cudaMemcpyHostToDevice);
+  cudaMemcpyAsync(c->d_r0buf, &one, sizeof(float), cudaMemcpyHostToDevice, c->st_own);
   if (nccl_allreduce(c, c->d_r0buf, 1, NCCL_FLOAT32, c->st_own) < 0 || cudaStreamSynchronize(c->st_own) != cudaSuccess)
     return fail(c, RGSQR_ERR_NCCL, "initial barrier");
   return RGSQR_OK;

@@ -153,3 +153,46 @@ def test_vshards_rejects_unequal_shards():
         h.factor_device(Ad, 4096, 4096, 64, Ad, R, precision="fp16")
     assert e.value.status == -5
     h.close()
+
+
+def test_host_colchunk_dist_equals_plain(handles):
+    """The column-chunked out-of-core node (R26) in a distributed context: its tail, phase-A
+    and piece-wise projections reduce R12 across ranks (ncclAllReduce).  The distributed context
+    reserves the reduction buffers, so its plan (tail width) can differ from the plain one: Gaussian
+    results agree to rounding, exact-dyadic results are bitwise R0 / H for both."""
+    plain, dist = handles
+    m, n = 16384, 1024
+    A = gi.gaussian(m, n, seed=14, dtype="fp16")
+    A64, R0 = gi.dyadic_mixed(m, n, seed=15)
+    Ad = gi.to_storage(A64, "fp16")
+    out = []
+    for h in (plain, dist):
+        h.set_option("chunk_mib", 2)
+        Q = np.empty_like(A, order="F")
+        R = np.zeros((n, n), dtype=np.float32, order="F")
+        assert h.factor(A, m, m, n, Q, R, precision="fp16", budget=40 * MiB) == 0
+        st = h.stats()
+        assert st["n_colchunk_nodes"] == 1, (h is plain, {k: st[k] for k in ("h2d_bytes", "n_ooc_nodes", "arena_bytes", "ctx_device_bytes") if k in st}, st)
+        out.append(R.astype(np.float64))
+        Qd = np.empty_like(Ad, order="F")
+        Rd = np.zeros((n, n), dtype=np.float32, order="F")
+        assert h.factor(Ad, m, m, n, Qd, Rd, precision="fp16", budget=40 * MiB) == 0
+        assert h.stats()["n_colchunk_nodes"] == 1
+        np.testing.assert_array_equal(Rd.astype(np.float64), R0)
+        np.testing.assert_array_equal(gi.to_float64(Qd, "fp16"), gi.hadamard(m, n))
+        h.set_option("chunk_mib", 32)
+    assert np.linalg.norm(out[0] - out[1]) / np.linalg.norm(out[0]) < 2e-3
+
+
+def test_budget_agreement_follows_each_call(handles):
+    """The distributed budget agreement (ncclAllReduce of the shape / budget words) must see THIS
+    call's budget: a smaller budget in the previous call must not leak into the next plan."""
+    _, dist = handles
+    m, n = 8192, 256
+    A = gi.gaussian(m, n, seed=21, dtype="fp16")
+    for b in (12, 40, 10, 64, 12):
+        Q = np.empty_like(A, order="F")
+        R = np.zeros((n, n), dtype=np.float32, order="F")
+        assert dist.factor(A, m, m, n, Q, R, precision="fp16", budget=b * MiB) == 0
+        st = dist.stats()
+        assert st["arena_bytes"] == b * MiB - st["ctx_device_bytes"], (b, st["arena_bytes"])
