@@ -333,11 +333,22 @@ def main():
            "h2d_bytes_per_step": so["h2d_bytes"], "d2h_bytes_per_step": so["d2h_bytes"],
            "path": "rgsqr_factor (C ABI), A/Q/R in pinned host memory, budget %d MiB (same run as value)"
                    % (budget // MiB),
-           "overlap_ratio": so["overlap_ratio"],
-           "busy_ms": {"h2d": so["h2d_busy_ms"], "d2h": so["d2h_busy_ms"], "compute": so["compute_busy_ms"]},
+           "graph_replay": bool(so["graph_replay"]),
            "ooc_nodes": so["n_ooc_nodes"], "arena_bytes": so["arena_bytes"],
            "ctx_device_bytes": so["ctx_device_bytes"], "colchunk_nodes": so["n_colchunk_nodes"],
            "arena_high_water": so["arena_high_water"]}
+    # per-stream busy times / overlap ratio: not measured inside a replayed CUDA graph, so one
+    # untimed eager call of the same schedule (RGSQR_OPT_GRAPH = 0) reports them
+    h.set_option("graph", 0)
+    h.factor(pa, lda, m, n, pq, pr, precision=prec, budget=budget)
+    torch.cuda.synchronize()
+    se = h.stats()
+    h.set_option("graph", 1)
+    e2e["eager_diagnostic"] = {"wall_ms": se["wall_ms"], "overlap_ratio": se["overlap_ratio"],
+                               "busy_ms": {"h2d": se["h2d_busy_ms"], "d2h": se["d2h_busy_ms"],
+                                           "compute": se["compute_busy_ms"]},
+                               "note": "one untimed call with eager launches (RGSQR_OPT_GRAPH=0); the timed "
+                                       "steps replay the captured CUDA graph (DESIGN.md R30)"}
     # ablation (not the headline): OOC left child 62.5% of the columns instead of the paper's halves
     if world == 1 and not args.no_ablation:
         h.set_option("split_pct", 62)

@@ -129,6 +129,12 @@ enum rgsqr_option {
   ,RGSQR_OPT_PHASEA_PCT = 22    /* column-chunked node: percentage of the right child's first half whose Q1
                                    projection is applied before the right child starts (phase A, while the
                                    tail goes out; default 50) */
+  ,RGSQR_OPT_GRAPH = 23         /* 1 (default): replay repeated rgsqr_factor / rgsqr_factor_device calls as one
+                                   CUDA graph (captured on the first call with a given signature: buffers,
+                                   shape, precision, budget, options, stream).  Host path: only when A, Q and
+                                   R are already page-locked (rgsqr_host_alloc / cudaHostAlloc /
+                                   cudaHostRegister) -- the captured copies address them directly.  Single-GPU
+                                   contexts; off while RGSQR_OPT_PROFILE is set.  0: eager launches */
 };
 
 /* Counters of the last rgsqr_factor* call (bytes are host<->device link bytes). */
@@ -170,6 +176,9 @@ typedef struct rgsqr_stats {
                                    child (they did not fit beside Q1) */
   int64_t ctx_device_bytes;     /* context-lifetime device buffers (leaf exchange words, partials, ...):
                                    counted against device_mem_budget, arena_bytes + this <= budget */
+  int64_t graph_replay;         /* 1: this call ran as a CUDA graph (RGSQR_OPT_GRAPH); the per-stream busy
+                                   times and overlap_ratio are then not measured (0) */
+  int64_t graph_captures;       /* graphs captured by this handle so far */
 } rgsqr_stats;
 
 /* ---- lifetime -------------------------------------------------------------------- */

@@ -14,7 +14,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "librgsqr.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-SOURCES = ["api.cu", "ops.cu", "gemm.cu", "leaf.cu", "ooc.cu", "oocgemm.cu", "small.cu"]
+SOURCES = ["api.cu", "ops.cu", "gemm.cu", "leaf.cu", "ooc.cu", "oocgemm.cu", "small.cu", "graph.cu"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3",
          "-Xptxas", "-v", "--expt-relaxed-constexpr", "-cudart", "static"]

@@ -29,6 +29,7 @@ int ensure_arena(Ctx* c, size_t want) {
     return RGSQR_OK;
   }
   if (c->arena.base) {
+    graph_drop_all(c);   // (captured schedules address the old arena)
     cudaFree(c->arena.base);
     c->arena = Arena{};
   }
@@ -96,11 +97,34 @@ int factor_device(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void
   if (rc < 0) return rc;
   cudaStream_t st = c->compute();
   const int s = elem_bytes(prec);
-  if (Q != A)
-    RGSQR_CUDA(c, cudaMemcpy2DAsync(Q, lda * s, A, lda * s, m * s, n, cudaMemcpyDeviceToDevice, st));
-  RGSQR_CUDA(c, cudaMemsetAsync(R, 0, (size_t)n * n * sizeof(float), st));
-  RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), st));
-  rc = incore_factor(c, prec, Q, lda, m, n, R, n, 0, st);
+  auto schedule = [&]() -> int {
+    if (Q != A)
+      RGSQR_CUDA(c, cudaMemcpy2DAsync(Q, lda * s, A, lda * s, m * s, n, cudaMemcpyDeviceToDevice, st));
+    RGSQR_CUDA(c, cudaMemsetAsync(R, 0, (size_t)n * n * sizeof(float), st));
+    RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), st));
+    return incore_factor(c, prec, Q, lda, m, n, R, n, 0, st);
+  };
+  if (graph_allowed(c)) {
+    // replay the captured schedule (graph.cu); the first call with this signature captures it
+    auto key = graph_key(c, 1, {reinterpret_cast<int64_t>(A), reinterpret_cast<int64_t>(Q),
+                                reinterpret_cast<int64_t>(R), lda, m, n, prec});
+    GraphEntry* g = graph_find(c, key);
+    if (!g && !graph_known_bad(c, key)) {
+      unsigned cnt0[2];
+      const size_t amark = c->arena.mark();
+      if (graph_capture_begin(c, st, cnt0)) {
+        const int src = schedule();
+        graph_capture_end(c, st, std::move(key), cnt0, src, &g);
+        if (!g) {   // capture failed: nothing ran, re-run eagerly
+          c->arena.release(amark);
+          reset_stats(c);
+        }
+      }
+    }
+    rc = g ? graph_launch(c, g, st) : schedule();
+  } else {
+    rc = schedule();
+  }
   if (rc < 0) return rc;
   int brk = INT_MAX;
   RGSQR_CUDA(c, cudaMemcpyAsync(&brk, c->d_breakdown, sizeof(int), cudaMemcpyDeviceToHost, st));
@@ -340,6 +364,7 @@ int rgsqr_destroy(rgsqr_handle h) {
   cudaDeviceSynchronize();
   for (void* ptr : c->ipc_opened) cudaIpcCloseMemHandle(ptr);
   if (c->nccl_comm && g_nccl.commDestroy) g_nccl.commDestroy(c->nccl_comm);
+  graph_drop_all(c);
   if (c->arena.base) cudaFree(c->arena.base);
   cudaFree(c->d_partials);
   cudaFree(c->d_sn_partials);
@@ -568,6 +593,7 @@ static int64_t* opt_slot(Ctx* c, int key) {
     case RGSQR_OPT_VSHARDS: return &o.vshards;
     case RGSQR_OPT_DEFER_PIECES: return &o.defer_pieces;
     case RGSQR_OPT_PHASEA_PCT: return &o.phasea_pct;
+    case RGSQR_OPT_GRAPH: return &o.graph;
   }
   return nullptr;
 }
@@ -584,7 +610,8 @@ int rgsqr_set_option(rgsqr_handle h, int key, int64_t value) {
     case RGSQR_OPT_RING_DEPTH: if (value < 2 || value > 16) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_ALGO: if (value < 0 || value > 2) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_REORTH: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
-    case RGSQR_OPT_COLCHUNK: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
+    case RGSQR_OPT_COLCHUNK:
+    case RGSQR_OPT_GRAPH: if (value != 0 && value != 1) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_EAGER_PCT:
     case RGSQR_OPT_PHASEA_PCT: if (value < 0 || value > 100) return RGSQR_ERR_INVALID_ARG; break;
     case RGSQR_OPT_CHUNK_MIB: if (value < 1 || value > 1024) return RGSQR_ERR_INVALID_ARG; break;

@@ -6,6 +6,7 @@
 
 #include <cstdint>
 #include <functional>
+#include <initializer_list>
 #include <map>
 #include <string>
 #include <vector>
@@ -37,8 +38,18 @@ struct Options {
   int64_t vshards = 1;       // virtual row shards on one GPU (RGSQR_OPT_VSHARDS, device path)
   int64_t phasea_pct = 50;  // column-chunked node: % of the right child's first half projected before it
   int64_t defer_pieces = 0;  // deferred products in ~1/p of the node's A2 (RGSQR_OPT_DEFER_PIECES; 0 = upload chunks)
+  int64_t graph = 1;         // replay repeated calls as CUDA graphs (RGSQR_OPT_GRAPH, graph.cu)
   int64_t eager_pct = 50;    // column-chunked node: the external projection is completed once the right
                              // child's leaves reach this % of its left half (RGSQR_OPT_EAGER_PCT)
+};
+
+struct GraphEntry {         // an instantiated factorization schedule (graph.cu)
+  std::vector<int64_t> key;
+  cudaGraphExec_t exec = nullptr;
+  unsigned cnt0[2] = {0, 0}, cnt1[2] = {0, 0};   // barrier counters at capture start / end
+  rgsqr_stats stats{};
+  size_t arena_high = 0;     // arena high-water mark of the captured schedule
+  uint64_t last_use = 0;
 };
 
 struct KernSeg {
@@ -110,6 +121,13 @@ struct Ctx {
   // a leaf exchange timed out (a rank did not arrive): late contributions may still land in the
   // never-reset exchange words, so the handle refuses further factorizations (rgsqr_destroy it)
   bool broken = false;
+  std::vector<GraphEntry> graphs;            // captured schedules (RGSQR_OPT_GRAPH)
+  uint64_t graph_clock = 0;
+  int64_t n_graph_captures = 0;
+  bool graph_failed = false;                 // capture not supported here: eager launches from then on
+  bool capturing = false;                    // inside a stream capture (no timing events)
+  std::vector<cudaEvent_t> capture_events;   // fresh events handed out during a capture
+  std::vector<std::vector<int64_t>> graph_bad;   // signatures whose capture failed: eager
   std::map<void*, size_t> host_allocs;       // rgsqr_host_alloc buffers (NUMA-placed, registered)
   int host_numa_node = -1;                   // the GPU's NUMA node (-1: unknown / single node)
 
@@ -135,6 +153,17 @@ struct Ctx {
   }
   void collect_kernel_stats();  // after a synchronize
 };
+
+// CUDA-graph replay (graph.cu)
+std::vector<int64_t> graph_key(Ctx* c, int kind, std::initializer_list<int64_t> call);
+bool graph_allowed(Ctx* c);
+GraphEntry* graph_find(Ctx* c, const std::vector<int64_t>& key);
+bool graph_known_bad(Ctx* c, const std::vector<int64_t>& key);
+void graph_drop_all(Ctx* c);
+int graph_capture_begin(Ctx* c, cudaStream_t st, unsigned cnt0[2]);
+int graph_capture_end(Ctx* c, cudaStream_t st, std::vector<int64_t> key, const unsigned cnt0[2], int rc,
+                      GraphEntry** out);
+int graph_launch(Ctx* c, GraphEntry* g, cudaStream_t st);
 
 // status helpers
 int fail(Ctx* c, int status, const std::string& msg);

@@ -60,11 +60,13 @@ struct Exec {
 
   // ---- timing / accounting helpers ----
   cudaEvent_t seg_begin(cudaStream_t st) {
+    if (c->capturing) return nullptr;   // (a replayed graph is not timed per segment)
     cudaEvent_t e = c->ev();
     cudaEventRecord(e, st);
     return e;
   }
   void seg_end(int kind, cudaStream_t st, cudaEvent_t a) {
+    if (!a) return;
     cudaEvent_t b = c->ev();
     cudaEventRecord(b, st);
     c->segs.push_back({kind, a, b});
@@ -74,6 +76,20 @@ struct Exec {
     cudaEvent_t e = c->ev();
     cudaEventRecord(e, signaller);
     cudaStreamWaitEvent(waiter, e, 0);
+  }
+  // graph capture: the copy streams join the capture from the compute stream, and all of them
+  // join back into it before the capture ends
+  void fork_from_compute() {
+    wait(sh, sc);
+    wait(sd, sc);
+    wait(sr, sc);
+    if (sh2) wait(sh2, sc);
+  }
+  void join_into_compute() {
+    wait(sc, sh);
+    wait(sc, sd);
+    wait(sc, sr);
+    if (sh2) wait(sc, sh2);
   }
   void join_all() {
     wait(sc, sh);
@@ -1010,15 +1026,41 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   x.join_all();
   cudaEvent_t t_ref = c->ev();
   cudaEventRecord(t_ref, x.sc);
-  RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), x.sc));
   std::thread zero;
   if (R)
     zero = std::thread([R, n] {
       for (int64_t j = 0; j + 1 < n; ++j) std::memset(R + j * n + j + 1, 0, (size_t)(n - j - 1) * 4);
     });
-  rc = c->opt.algo == 1   ? x.blocked(std::min<int64_t>(c->opt.block_cols, n))
-       : c->opt.algo == 2 ? x.fused_blocked(std::min<int64_t>(c->opt.block_cols, n))
-                          : x.node(0, n, false);
+  auto schedule = [&]() -> int {
+    RGSQR_CUDA(c, cudaMemsetAsync(c->d_breakdown, 0x7f, sizeof(int), x.sc));
+    return c->opt.algo == 1   ? x.blocked(std::min<int64_t>(c->opt.block_cols, n))
+           : c->opt.algo == 2 ? x.fused_blocked(std::min<int64_t>(c->opt.block_cols, n))
+                              : x.node(0, n, false);
+  };
+  // CUDA-graph replay (graph.cu) when the caller's buffers were already page-locked (the captured
+  // copies address them directly; buffers this call registered are unregistered at its end)
+  if (graph_allowed(c) && registered.empty()) {
+    auto key = graph_key(c, 2, {reinterpret_cast<int64_t>(A), reinterpret_cast<int64_t>(Q),
+                                reinterpret_cast<int64_t>(R), lda, m, n, prec});
+    GraphEntry* g = graph_find(c, key);
+    if (!g && !graph_known_bad(c, key)) {
+      unsigned cnt0[2];
+      const size_t amark = c->arena.mark();
+      if (graph_capture_begin(c, x.sc, cnt0)) {
+        x.fork_from_compute();
+        int src = schedule();
+        if (src >= 0) x.join_into_compute();
+        graph_capture_end(c, x.sc, std::move(key), cnt0, src, &g);
+        if (!g) {   // capture failed: nothing ran, re-run eagerly
+          c->arena.release(amark);
+          reset_stats(c);
+        }
+      }
+    }
+    rc = g ? graph_launch(c, g, x.sc) : schedule();
+  } else {
+    rc = schedule();
+  }
   int brk = INT_MAX;
   if (rc >= 0) {
     x.join_all();

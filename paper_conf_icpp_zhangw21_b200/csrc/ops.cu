@@ -32,6 +32,15 @@ void Ctx::collect_kernel_stats() {
 }
 
 cudaEvent_t Ctx::ev() {
+  if (capturing) {
+    // never-recorded events for a capture: a pooled event may still carry a record from an
+    // earlier eager call, and waiting on it inside the capture would cross the capture boundary
+    // (the executor waits on slot-free events before their first record: a no-op by design)
+    cudaEvent_t e;
+    cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    capture_events.push_back(e);
+    return e;
+  }
   if (event_next == event_pool.size()) {
     cudaEvent_t e;
     cudaEventCreate(&e);

@@ -26,7 +26,7 @@ OPTIONS = {"leaf_width": 1, "tile_rows_min": 2, "tile_rows_max": 3, "ring_depth"
            "reorth": 12, "prefetch": 13, "fuse_small": 14, "split_pct": 15,
            "x3_chain": 16, "colchunk": 17, "eager_pct": 18,
            "chunk_mib": 19, "vshards": 20,
-           "defer_pieces": 21, "phasea_pct": 22}
+           "defer_pieces": 21, "phasea_pct": 22, "graph": 23}
 
 EXPORTS = ["rgsqr_create", "rgsqr_get_unique_id", "rgsqr_create_dist", "rgsqr_destroy", "rgsqr_factor",
            "rgsqr_factor_device", "rgsqr_op_leaf", "rgsqr_op_inner", "rgsqr_op_outer", "rgsqr_set_stream",
@@ -47,7 +47,8 @@ class Stats(C.Structure):
                 ("kern_ms", C.c_double * 4), ("kern_launches", C.c_int64 * 4),
                 ("kern_flops", C.c_double * 4), ("kern_bytes", C.c_double * 4),
                 ("n_colchunk_nodes", C.c_int64), ("colchunk_tail_cols", C.c_int64),
-                ("ctx_device_bytes", C.c_int64)]
+                ("ctx_device_bytes", C.c_int64), ("graph_replay", C.c_int64),
+                ("graph_captures", C.c_int64)]
 
     def as_dict(self):
         out = {}

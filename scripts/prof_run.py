@@ -20,11 +20,14 @@ ap.add_argument("--n", type=int, default=8192)
 ap.add_argument("--prec", default="fp16")
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--host", action="store_true", help="use the host (out-of-core) path, 1 GiB budget")
+ap.add_argument("--profile", action="store_true", help="per-kernel-class CUDA-event accounting (RGSQR_OPT_PROFILE)")
 a = ap.parse_args()
 build.build()
 st = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}[a.prec]
 A = gi.gaussian(a.m, a.n, seed=2, dtype=st)
 h = Handle(0)
+if a.profile:
+    h.set_option("profile", 1)
 if a.host:
     Q = np.empty_like(A, order="F")
     R = np.empty((a.n, a.n), dtype=np.float32, order="F")
@@ -37,4 +40,8 @@ else:
     for _ in range(a.reps):
         h.factor_device(Ad, a.m, a.m, a.n, Qd, Rd, precision=a.prec, budget=1 << 30)
 torch.cuda.synchronize()
-print("stats", h.stats())
+st = h.stats()
+print("stats", st)
+if a.profile:
+    print("kern_ms leaf/inner/outer/other", [round(x, 3) for x in st["kern_ms"]], "sum", round(sum(st["kern_ms"]), 3),
+          "wall", round(st["wall_ms"], 3))
