@@ -43,12 +43,19 @@ struct Options {
                              // child's leaves reach this % of its left half (RGSQR_OPT_EAGER_PCT)
 };
 
+struct TimedSeg {
+  int kind;                  // 0 h2d, 1 d2h, 2 compute
+  cudaEvent_t a, b;
+};
+
 struct GraphEntry {         // an instantiated factorization schedule (graph.cu)
   std::vector<int64_t> key;
   cudaGraphExec_t exec = nullptr;
   unsigned cnt0[2] = {0, 0}, cnt1[2] = {0, 0};   // barrier counters at capture start / end
   rgsqr_stats stats{};
   size_t arena_high = 0;     // arena high-water mark of the captured schedule
+  std::vector<TimedSeg> segs;             // RGSQR_TIMELINE: the schedule's timed segments (external
+  std::vector<cudaEvent_t> tl_events;     //   event record nodes) and the events they own
   uint64_t last_use = 0;
 };
 
@@ -77,10 +84,6 @@ struct Arena {
   size_t free_bytes() const { return size > top ? size - ((top + 255) & ~size_t(255)) : 0; }
 };
 
-struct TimedSeg {
-  int kind;                  // 0 h2d, 1 d2h, 2 compute
-  cudaEvent_t a, b;
-};
 
 struct Ctx {
   int device = 0;
@@ -127,6 +130,8 @@ struct Ctx {
   bool graph_failed = false;                 // capture not supported here: eager launches from then on
   bool capturing = false;                    // inside a stream capture (no timing events)
   std::vector<cudaEvent_t> capture_events;   // fresh events handed out during a capture
+  bool graph_timeline = false;               // capture timing segments (RGSQR_TIMELINE)
+  std::vector<cudaEvent_t> graph_tl_events;  // their events (moved into the graph entry)
   std::vector<std::vector<int64_t>> graph_bad;   // signatures whose capture failed: eager
   std::map<void*, size_t> host_allocs;       // rgsqr_host_alloc buffers (NUMA-placed, registered)
   int host_numa_node = -1;                   // the GPU's NUMA node (-1: unknown / single node)

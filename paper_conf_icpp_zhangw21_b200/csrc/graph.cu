@@ -43,8 +43,15 @@ std::vector<int64_t> graph_key(Ctx* c, int kind, std::initializer_list<int64_t> 
 }
 
 bool graph_allowed(Ctx* c) {
-  static const bool env_off = getenv("RGSQR_LEAF_DEBUG") || getenv("RGSQR_LEAF_DEBUG2") || getenv("RGSQR_TIMELINE");
+  static const bool env_off = getenv("RGSQR_LEAF_DEBUG") || getenv("RGSQR_LEAF_DEBUG2");
   return c->opt.graph != 0 && !c->opt.profile && !c->graph_failed && c->nccl_comm == nullptr && !env_off;
+}
+
+static void destroy_entry(GraphEntry& g) {
+  if (g.exec) cudaGraphExecDestroy(g.exec);
+  for (cudaEvent_t e : g.tl_events) cudaEventDestroy(e);
+  g.exec = nullptr;
+  g.tl_events.clear();
 }
 
 bool graph_known_bad(Ctx* c, const std::vector<int64_t>& key) {
@@ -63,8 +70,7 @@ GraphEntry* graph_find(Ctx* c, const std::vector<int64_t>& key) {
 }
 
 void graph_drop_all(Ctx* c) {
-  for (auto& g : c->graphs)
-    if (g.exec) cudaGraphExecDestroy(g.exec);
+  for (auto& g : c->graphs) destroy_entry(g);
   c->graphs.clear();
 }
 
@@ -78,6 +84,8 @@ int graph_capture_begin(Ctx* c, cudaStream_t st, unsigned cnt0[2]) {
     return 0;   // not capturing: the caller runs eagerly
   }
   c->capturing = true;
+  static const bool timeline = getenv("RGSQR_TIMELINE") != nullptr;
+  c->graph_timeline = timeline;
   set_counters_kernel<<<1, 1, 0, st>>>(c->d_counter, cnt0[0], c->d_counter + 16, cnt0[1]);
   return 1;
 }
@@ -93,7 +101,11 @@ int graph_capture_end(Ctx* c, cudaStream_t st, std::vector<int64_t> key, const u
   if (g) cudaGraphDestroy(g);
   for (cudaEvent_t ev : c->capture_events) cudaEventDestroy(ev);   // (internal edges of the graph now)
   c->capture_events.clear();
+  std::vector<cudaEvent_t> tl_events;
+  tl_events.swap(c->graph_tl_events);
   if (rc < 0 || e != cudaSuccess || !exec) {
+    for (cudaEvent_t ev : tl_events) cudaEventDestroy(ev);
+    c->segs.clear();
     // nothing captured ran: the barrier counters are where they were; the caller re-runs the
     // schedule eagerly (a genuine error, e.g. a budget too small, then surfaces from that run)
     c->counter_host[0] = cnt0[0];
@@ -107,7 +119,7 @@ int graph_capture_end(Ctx* c, cudaStream_t st, std::vector<int64_t> key, const u
     size_t lru = 0;
     for (size_t i = 1; i < c->graphs.size(); ++i)
       if (c->graphs[i].last_use < c->graphs[lru].last_use) lru = i;
-    cudaGraphExecDestroy(c->graphs[lru].exec);
+    destroy_entry(c->graphs[lru]);
     c->graphs.erase(c->graphs.begin() + lru);
   }
   GraphEntry ge;
@@ -119,6 +131,8 @@ int graph_capture_end(Ctx* c, cudaStream_t st, std::vector<int64_t> key, const u
   ge.cnt1[1] = c->counter_host[1];
   ge.stats = c->stats;
   ge.arena_high = c->arena.high;
+  ge.segs = c->segs;
+  ge.tl_events = std::move(tl_events);
   ge.last_use = ++c->graph_clock;
   c->graphs.push_back(std::move(ge));
   *out = &c->graphs.back();
@@ -133,6 +147,7 @@ int graph_launch(Ctx* c, GraphEntry* g, cudaStream_t st) {
   c->counter_host[0] = g->cnt1[0];
   c->counter_host[1] = g->cnt1[1];
   c->arena.high = std::max(c->arena.high, g->arena_high);
+  c->segs = g->segs;   // (RGSQR_TIMELINE: the graph's own event record nodes)
   RGSQR_CUDA(c, cudaGraphLaunch(g->exec, st));
   return RGSQR_OK;
 }

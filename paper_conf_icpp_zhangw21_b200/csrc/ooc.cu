@@ -59,16 +59,27 @@ struct Exec {
   cudaStream_t sh2 = nullptr;    // second upload queue (column-chunked node's late tail piece)
 
   // ---- timing / accounting helpers ----
-  cudaEvent_t seg_begin(cudaStream_t st) {
-    if (c->capturing) return nullptr;   // (a replayed graph is not timed per segment)
-    cudaEvent_t e = c->ev();
-    cudaEventRecord(e, st);
+  // per-segment timing events; inside a graph capture only for RGSQR_TIMELINE, as external event
+  // record nodes (events owned by the graph entry, valid after every replay)
+  cudaEvent_t seg_event(cudaStream_t st) {
+    cudaEvent_t e;
+    if (c->capturing) {
+      cudaEventCreate(&e);
+      c->graph_tl_events.push_back(e);
+      cudaEventRecordWithFlags(e, st, cudaEventRecordExternal);
+    } else {
+      e = c->ev();
+      cudaEventRecord(e, st);
+    }
     return e;
+  }
+  cudaEvent_t seg_begin(cudaStream_t st) {
+    if (c->capturing && !c->graph_timeline) return nullptr;   // (replays are not timed per segment)
+    return seg_event(st);
   }
   void seg_end(int kind, cudaStream_t st, cudaEvent_t a) {
     if (!a) return;
-    cudaEvent_t b = c->ev();
-    cudaEventRecord(b, st);
+    cudaEvent_t b = seg_event(st);
     c->segs.push_back({kind, a, b});
   }
   void wait(cudaStream_t waiter, cudaStream_t signaller) {

@@ -20,6 +20,7 @@ ap.add_argument("--n", type=int, default=8192)
 ap.add_argument("--prec", default="fp16")
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--host", action="store_true", help="use the host (out-of-core) path, 1 GiB budget")
+ap.add_argument("--pinned", action="store_true", help="host path with rgsqr_host_alloc buffers (CUDA-graph replay)")
 ap.add_argument("--profile", action="store_true", help="per-kernel-class CUDA-event accounting (RGSQR_OPT_PROFILE)")
 a = ap.parse_args()
 build.build()
@@ -28,7 +29,14 @@ A = gi.gaussian(a.m, a.n, seed=2, dtype=st)
 h = Handle(0)
 if a.profile:
     h.set_option("profile", 1)
-if a.host:
+if a.host and a.pinned:
+    import ctypes
+    nb = A.nbytes
+    pa, pq, pr = h.host_alloc(nb), h.host_alloc(nb), h.host_alloc(a.n * a.n * 4)
+    np.ctypeslib.as_array((ctypes.c_uint8 * nb).from_address(pa))[:] = A.reshape(-1, order="F").view(np.uint8)
+    for _ in range(a.reps):
+        h.factor(pa, a.m, a.m, a.n, pq, pr, precision=a.prec, budget=1 << 30)
+elif a.host:
     Q = np.empty_like(A, order="F")
     R = np.empty((a.n, a.n), dtype=np.float32, order="F")
     for _ in range(a.reps):
