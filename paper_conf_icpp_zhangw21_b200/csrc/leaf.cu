@@ -330,9 +330,11 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       part[warp][k] = dot4(cx, cy);
     }
     __syncthreads();
+    PRO_STAMP(8);
     const float s = cta_sum(&part[0][0], LEAF_MAX_W + 2, L);
     if ((threadIdx.x & 3) == 0 && (threadIdx.x >> 2) < L) p.partials[(size_t)(threadIdx.x >> 2) * G + g] = s;
     __syncthreads();
+    PRO_STAMP(9);
     if (threadIdx.x == 0) {  // release: orders this CTA's partial stores (bar.sync cumulativity)
       asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.counter) : "memory");
       unsigned cv;
@@ -341,6 +343,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       } while ((int)(cv - p.counter_target) < 0);   // (wrap-safe: the counter is never reset)
     }
     __syncthreads();
+    PRO_STAMP(10);
     }
     constexpr int KPW = (LEAF_MAX_W + 2 + LEAF_WARPS - 1) / LEAF_WARPS;
     constexpr int QMAX = (LEAF_MAX_G + 31) / 32;

@@ -515,11 +515,13 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
             avg(10, 11, t0, t1), avg(8, 12, t0, t1));
   }
   if (p.dbg) {
-    long long pb[8];
-    cudaMemcpyAsync(pb, p.dbg + 16 * LEAF_MAX_W, sizeof(long long) * 8, cudaMemcpyDeviceToHost, st);
+    long long pb[12];
+    cudaMemcpyAsync(pb, p.dbg + 16 * LEAF_MAX_W, sizeof(long long) * 12, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
-    fprintf(stderr, "[leaf prologue/epilogue cycles] xprev+load %lld round0 %lld tables %lld rounds %lld join %lld store %lld\n",
-            pb[1] - pb[0], pb[2] - pb[1], pb[3] - pb[2], pb[4] - pb[3], pb[5] - pb[4], pb[6] - pb[5]);
+    fprintf(stderr, "[leaf prologue/epilogue cycles] xprev+load %lld round0 %lld (dots %lld partials %lld barrier %lld "
+            "gather %lld) tables %lld rounds %lld join %lld store %lld\n",
+            pb[1] - pb[0], pb[2] - pb[1], pb[8] - pb[1], pb[9] - pb[8], pb[10] - pb[9], pb[2] - pb[10],
+            pb[3] - pb[2], pb[4] - pb[3], pb[5] - pb[4], pb[6] - pb[5]);
   }
   if (p.dbg2) {
     std::vector<long long> hb((size_t)2 * LEAF_MAX_W * G);
