@@ -35,15 +35,26 @@ struct Pipe {
   cudaStream_t sc, sh, sd;
   int64_t s;
   std::vector<cudaEvent_t> freed;   // per slot: the slot may be overwritten after this event
-  cudaEvent_t seg_begin(cudaStream_t st) {
-    cudaEvent_t e = c->ev();
-    cudaEventRecord(e, st);
+  // (inside a graph capture: timed only for RGSQR_TIMELINE, as external event record nodes)
+  cudaEvent_t seg_event(cudaStream_t st) {
+    cudaEvent_t e;
+    if (c->capturing) {
+      cudaEventCreate(&e);
+      c->graph_tl_events.push_back(e);
+      cudaEventRecordWithFlags(e, st, cudaEventRecordExternal);
+    } else {
+      e = c->ev();
+      cudaEventRecord(e, st);
+    }
     return e;
   }
+  cudaEvent_t seg_begin(cudaStream_t st) {
+    if (c->capturing && !c->graph_timeline) return nullptr;
+    return seg_event(st);
+  }
   void seg_end(int kind, cudaStream_t st, cudaEvent_t a) {
-    cudaEvent_t b = c->ev();
-    cudaEventRecord(b, st);
-    c->segs.push_back({kind, a, b});
+    if (!a) return;
+    c->segs.push_back({kind, a, seg_event(st)});
   }
   cudaEvent_t mark(cudaStream_t st) {
     cudaEvent_t e = c->ev();
@@ -166,78 +177,14 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
     while (K > 2 && (size_t)K * per + ws_reserve > free_b) --K;
     return (size_t)K * per + ws_reserve <= free_b;
   };
-  if (op == 0 && tiling == 0) {
-    // ---- Fig. 3: R12 resident (fp32), row tiles of Q1 and A2 ----
-    float* dR = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
-    const int64_t t = dR ? fits_rows(0, (size_t)(w1 + w2) * s, block > 0 ? block : 16384) : 0;
-    if (!dR || t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner: R12 + 2 tiles do not fit");
-    char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
-    if (!ring) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner: ring");
-    int64_t i = 0;
-    for (int64_t r0 = 0; r0 < m; r0 += t, ++i) {
-      const int64_t tr = std::min(t, m - r0);
-      const int k = (int)(i % K);
-      char* sq = ring + (size_t)k * t * (w1 + w2) * s;
-      char* sa = sq + (size_t)t * w1 * s;
-      if (P.freed[k]) cudaStreamWaitEvent(P.sh, P.freed[k], 0);
-      if ((rc = P.up(sq, t, hq, ldq, r0, 0, tr, w1, s)) < 0) return rc;
-      if ((rc = P.up(sa, t, ha, lda, r0, 0, tr, w2, s)) < 0) return rc;
-      cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
-      cudaEvent_t a = P.seg_begin(P.sc);
-      rc = op_inner(c, prec, sq, t, sa, t, tr, w1, w2, dR, w1, nullptr, w1, i > 0 ? 1 : 0, P.sc, false);
-      if (rc < 0) return rc;
-      P.seg_end(2, P.sc, a);
-      P.freed[k] = P.mark(P.sc);
-    }
-    cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
-    if ((rc = P.down(hr, ldr, 0, 0, dR, w1, w1, w2, 4)) < 0) return rc;
-  } else if (op == 0) {
-    // ---- Fig. 4: Q1 (the panel) resident, column blocks of A2, R12 blocks out ----
-    const int64_t b = std::min<int64_t>(w2, block > 0 ? block : 16384);
-    char* dQ = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
-    const size_t per = (size_t)m * b * s + (size_t)w1 * b * 4 + 512;
-    if (!dQ || !fits_slots(per))
-      return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner (blocking): panel + 2 column blocks do not fit");
-    char* ring = static_cast<char*>(c->arena.alloc((size_t)K * per));
-    if ((rc = P.up(dQ, m, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
-    cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
-    int64_t i = 0;
-    for (int64_t c0 = 0; c0 < w2; c0 += b, ++i) {
-      const int64_t bw = std::min(b, w2 - c0);
-      const int k = (int)(i % K);
-      char* sa = ring + (size_t)k * per;
-      float* sr = reinterpret_cast<float*>(sa + (size_t)m * b * s);
-      if (P.freed[k]) cudaStreamWaitEvent(P.sh, P.freed[k], 0);
-      if ((rc = P.up(sa, m, ha, lda, 0, c0, m, bw, s)) < 0) return rc;
-      cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
-      if (P.freed[k]) cudaStreamWaitEvent(P.sc, P.freed[k], 0);   // the block's previous R12 is out
-      cudaEvent_t a = P.seg_begin(P.sc);
-      rc = op_inner(c, prec, dQ, m, sa, m, m, w1, bw, sr, w1, nullptr, w1, 0, P.sc, false);
-      if (rc < 0) return rc;
-      P.seg_end(2, P.sc, a);
-      cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
-      if ((rc = P.down(hr, ldr, 0, c0, sr, w1, w1, bw, 4)) < 0) return rc;
-      P.freed[k] = P.mark(P.sd);
-    }
-  } else {
-    // ---- outer product: R12 uploaded once (fp32) and rounded to the operand type on the device ----
-    char* dRop = static_cast<char*>(c->arena.alloc((size_t)w1 * w2 * s));
-    const size_t mk = c->arena.mark();
-    float* dRf = static_cast<float*>(c->arena.alloc((size_t)w1 * std::min<int64_t>(w2, 4096) * 4));
-    if (!dRop || !dRf) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer: R12 does not fit");
-    for (int64_t c0 = 0; c0 < w2; c0 += 4096) {   // (staged in 4096-column pieces)
-      const int64_t cw = std::min<int64_t>(4096, w2 - c0);
-      if ((rc = P.up(dRf, w1, hr, ldr, 0, c0, w1, cw, 4)) < 0) return rc;
-      cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
-      if ((rc = cast_r12(c, prec, dRf, w1, dRop + (size_t)c0 * w1 * s, w1, w1, cw, P.sc)) < 0) return rc;
-      cudaStreamWaitEvent(P.sh, P.mark(P.sc), 0);
-    }
-    c->arena.release(mk);
-    if (tiling == 0) {
-      // ---- Fig. 5: row tiles of Q1 and A2 in, A2' tiles out ----
-      const int64_t t = fits_rows(0, (size_t)(w1 + w2) * s, block > 0 ? block : 8192);
-      if (t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer: R12 + 2 tiles do not fit");
+  auto schedule = [&]() -> int {
+    if (op == 0 && tiling == 0) {
+      // ---- Fig. 3: R12 resident (fp32), row tiles of Q1 and A2 ----
+      float* dR = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
+      const int64_t t = dR ? fits_rows(0, (size_t)(w1 + w2) * s, block > 0 ? block : 16384) : 0;
+      if (!dR || t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner: R12 + 2 tiles do not fit");
       char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
+      if (!ring) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner: ring");
       int64_t i = 0;
       for (int64_t r0 = 0; r0 < m; r0 += t, ++i) {
         const int64_t tr = std::min(t, m - r0);
@@ -249,43 +196,144 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
         if ((rc = P.up(sa, t, ha, lda, r0, 0, tr, w2, s)) < 0) return rc;
         cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
         cudaEvent_t a = P.seg_begin(P.sc);
-        rc = op_outer(c, prec, sq, t, dRop, w1, sa, t, tr, w1, w2, P.sc);
+        rc = op_inner(c, prec, sq, t, sa, t, tr, w1, w2, dR, w1, nullptr, w1, i > 0 ? 1 : 0, P.sc, false);
         if (rc < 0) return rc;
         P.seg_end(2, P.sc, a);
-        cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
-        if ((rc = P.down(ha, lda, r0, 0, sa, t, tr, w2, s)) < 0) return rc;
-        P.freed[k] = P.mark(P.sd);
+        P.freed[k] = P.mark(P.sc);
       }
-    } else {
-      // ---- Fig. 6: Q1 resident too, b x b tiles of A2 in and out ----
-      const int64_t b = block > 0 ? block : 16384;
-      const int64_t b1 = std::min(b, (m + 127) / 128 * 128), b2 = std::min(b, w2);
+      cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
+      if ((rc = P.down(hr, ldr, 0, 0, dR, w1, w1, w2, 4)) < 0) return rc;
+    } else if (op == 0) {
+      // ---- Fig. 4: Q1 (the panel) resident, column blocks of A2, R12 blocks out ----
+      const int64_t b = std::min<int64_t>(w2, block > 0 ? block : 16384);
       char* dQ = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
-      const size_t per = (size_t)b1 * b2 * s;
+      const size_t per = (size_t)m * b * s + (size_t)w1 * b * 4 + 512;
       if (!dQ || !fits_slots(per))
-        return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer (blocking): Q1 + R12 + 2 tiles do not fit");
+        return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner (blocking): panel + 2 column blocks do not fit");
       char* ring = static_cast<char*>(c->arena.alloc((size_t)K * per));
       if ((rc = P.up(dQ, m, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
       cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
       int64_t i = 0;
-      for (int64_t r0 = 0; r0 < m; r0 += b1)
-        for (int64_t c0 = 0; c0 < w2; c0 += b2, ++i) {
-          const int64_t tr = std::min(b1, m - r0), tc = std::min(b2, w2 - c0);
+      for (int64_t c0 = 0; c0 < w2; c0 += b, ++i) {
+        const int64_t bw = std::min(b, w2 - c0);
+        const int k = (int)(i % K);
+        char* sa = ring + (size_t)k * per;
+        float* sr = reinterpret_cast<float*>(sa + (size_t)m * b * s);
+        if (P.freed[k]) cudaStreamWaitEvent(P.sh, P.freed[k], 0);
+        if ((rc = P.up(sa, m, ha, lda, 0, c0, m, bw, s)) < 0) return rc;
+        cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
+        if (P.freed[k]) cudaStreamWaitEvent(P.sc, P.freed[k], 0);   // the block's previous R12 is out
+        cudaEvent_t a = P.seg_begin(P.sc);
+        rc = op_inner(c, prec, dQ, m, sa, m, m, w1, bw, sr, w1, nullptr, w1, 0, P.sc, false);
+        if (rc < 0) return rc;
+        P.seg_end(2, P.sc, a);
+        cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
+        if ((rc = P.down(hr, ldr, 0, c0, sr, w1, w1, bw, 4)) < 0) return rc;
+        P.freed[k] = P.mark(P.sd);
+      }
+    } else {
+      // ---- outer product: R12 uploaded once (fp32) and rounded to the operand type on the device ----
+      char* dRop = static_cast<char*>(c->arena.alloc((size_t)w1 * w2 * s));
+      const size_t mk = c->arena.mark();
+      float* dRf = static_cast<float*>(c->arena.alloc((size_t)w1 * std::min<int64_t>(w2, 4096) * 4));
+      if (!dRop || !dRf) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer: R12 does not fit");
+      for (int64_t c0 = 0; c0 < w2; c0 += 4096) {   // (staged in 4096-column pieces)
+        const int64_t cw = std::min<int64_t>(4096, w2 - c0);
+        if ((rc = P.up(dRf, w1, hr, ldr, 0, c0, w1, cw, 4)) < 0) return rc;
+        cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
+        if ((rc = cast_r12(c, prec, dRf, w1, dRop + (size_t)c0 * w1 * s, w1, w1, cw, P.sc)) < 0) return rc;
+        cudaStreamWaitEvent(P.sh, P.mark(P.sc), 0);
+      }
+      c->arena.release(mk);
+      if (tiling == 0) {
+        // ---- Fig. 5: row tiles of Q1 and A2 in, A2' tiles out ----
+        const int64_t t = fits_rows(0, (size_t)(w1 + w2) * s, block > 0 ? block : 8192);
+        if (t < 128) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer: R12 + 2 tiles do not fit");
+        char* ring = static_cast<char*>(c->arena.alloc((size_t)K * t * (w1 + w2) * s));
+        int64_t i = 0;
+        for (int64_t r0 = 0; r0 < m; r0 += t, ++i) {
+          const int64_t tr = std::min(t, m - r0);
           const int k = (int)(i % K);
-          char* sa = ring + (size_t)k * per;
+          char* sq = ring + (size_t)k * t * (w1 + w2) * s;
+          char* sa = sq + (size_t)t * w1 * s;
           if (P.freed[k]) cudaStreamWaitEvent(P.sh, P.freed[k], 0);
-          if ((rc = P.up(sa, b1, ha, lda, r0, c0, tr, tc, s)) < 0) return rc;
+          if ((rc = P.up(sq, t, hq, ldq, r0, 0, tr, w1, s)) < 0) return rc;
+          if ((rc = P.up(sa, t, ha, lda, r0, 0, tr, w2, s)) < 0) return rc;
           cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
           cudaEvent_t a = P.seg_begin(P.sc);
-          rc = op_outer(c, prec, dQ + (size_t)r0 * s, m, dRop + (size_t)c0 * w1 * s, w1, sa, b1, tr, w1, tc, P.sc);
+          rc = op_outer(c, prec, sq, t, dRop, w1, sa, t, tr, w1, w2, P.sc);
           if (rc < 0) return rc;
           P.seg_end(2, P.sc, a);
           cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
-          if ((rc = P.down(ha, lda, r0, c0, sa, b1, tr, tc, s)) < 0) return rc;
+          if ((rc = P.down(ha, lda, r0, 0, sa, t, tr, w2, s)) < 0) return rc;
           P.freed[k] = P.mark(P.sd);
         }
+      } else {
+        // ---- Fig. 6: Q1 resident too, b x b tiles of A2 in and out ----
+        const int64_t b = block > 0 ? block : 16384;
+        const int64_t b1 = std::min(b, (m + 127) / 128 * 128), b2 = std::min(b, w2);
+        char* dQ = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
+        const size_t per = (size_t)b1 * b2 * s;
+        if (!dQ || !fits_slots(per))
+          return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer (blocking): Q1 + R12 + 2 tiles do not fit");
+        char* ring = static_cast<char*>(c->arena.alloc((size_t)K * per));
+        if ((rc = P.up(dQ, m, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
+        cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
+        int64_t i = 0;
+        for (int64_t r0 = 0; r0 < m; r0 += b1)
+          for (int64_t c0 = 0; c0 < w2; c0 += b2, ++i) {
+            const int64_t tr = std::min(b1, m - r0), tc = std::min(b2, w2 - c0);
+            const int k = (int)(i % K);
+            char* sa = ring + (size_t)k * per;
+            if (P.freed[k]) cudaStreamWaitEvent(P.sh, P.freed[k], 0);
+            if ((rc = P.up(sa, b1, ha, lda, r0, c0, tr, tc, s)) < 0) return rc;
+            cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
+            cudaEvent_t a = P.seg_begin(P.sc);
+            rc = op_outer(c, prec, dQ + (size_t)r0 * s, m, dRop + (size_t)c0 * w1 * s, w1, sa, b1, tr, w1, tc, P.sc);
+            if (rc < 0) return rc;
+            P.seg_end(2, P.sc, a);
+            cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
+            if ((rc = P.down(ha, lda, r0, c0, sa, b1, tr, tc, s)) < 0) return rc;
+            P.freed[k] = P.mark(P.sd);
+          }
+      }
     }
+    return RGSQR_OK;
+  };
+  // CUDA-graph replay (graph.cu, R30) when the caller's buffers were already page-locked
+  if (graph_allowed(c) && registered.empty()) {
+    auto key = graph_key(c, 3, {op, tiling, block, reinterpret_cast<int64_t>(Q1), reinterpret_cast<int64_t>(A2),
+                                reinterpret_cast<int64_t>(R12), ldq, lda, ldr, m, w1, w2, prec});
+    GraphEntry* g = graph_find(c, key);
+    if (!g && !graph_known_bad(c, key)) {
+      unsigned cnt0[2];
+      const size_t amark = c->arena.mark();
+      const int K0 = K;
+      if (graph_capture_begin(c, P.sc, cnt0)) {
+        cudaEvent_t f = P.mark(P.sc);   // the copy streams join the capture
+        cudaStreamWaitEvent(P.sh, f, 0);
+        cudaStreamWaitEvent(P.sd, f, 0);
+        int src = schedule();
+        if (src >= 0) {
+          cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
+          cudaStreamWaitEvent(P.sc, P.mark(P.sd), 0);
+        }
+        graph_capture_end(c, P.sc, std::move(key), cnt0, src, &g);
+        if (!g) {   // capture failed: nothing ran, re-run eagerly
+          const double pin_ms = c->stats.pin_ms;
+          c->arena.release(amark);
+          reset_stats(c);
+          c->stats.pin_ms = pin_ms;
+          K = K0;
+          P.freed.assign(K, nullptr);
+        }
+      }
+    }
+    rc = g ? graph_launch(c, g, P.sc) : schedule();
+  } else {
+    rc = schedule();
   }
+  if (rc < 0) return rc;
   cudaError_t e1 = cudaStreamSynchronize(P.sc);
   cudaError_t e2 = cudaStreamSynchronize(c->st_h2d);
   cudaError_t e3 = cudaStreamSynchronize(c->st_d2h);

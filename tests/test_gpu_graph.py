@@ -171,3 +171,38 @@ def test_no_graph_for_pageable_buffers_or_profiling(h):
     rc, _, _, s = P.factor("fp16", 8 * MiB)
     assert rc == 0 and s["graph_replay"] == 1
     P.free()
+
+
+@pytest.mark.parametrize("op,tiling,block", [("inner", 0, 2048), ("inner", 1, 128), ("outer", 0, 2048),
+                                             ("outer", 1, 256)])
+def test_ooc_gemm_graph_replay_equals_eager(h, op, tiling, block):
+    """rgsqr_ooc_inner / rgsqr_ooc_outer (Tables 1/2 operations) on page-locked buffers: replays
+    equal the eager run bitwise (the outer product updates A2 in place, so each call restarts from
+    the same A2)."""
+    m, w1, w2 = 16384, 256, 512
+    Q = gi.gaussian(m, w1, seed=71, dtype="fp16")
+    A = gi.gaussian(m, w2, seed=72, dtype="fp16")
+    R = (gi.gaussian(w1, w2, seed=73, dtype="fp32") * 0.05).astype(np.float32)
+    pq, pa, pr = h.host_alloc(Q.nbytes), h.host_alloc(A.nbytes), h.host_alloc(R.nbytes)
+    vq = np.ctypeslib.as_array((ctypes.c_uint8 * Q.nbytes).from_address(pq))
+    va = np.ctypeslib.as_array((ctypes.c_uint8 * A.nbytes).from_address(pa))
+    vr = np.ctypeslib.as_array((ctypes.c_uint8 * R.nbytes).from_address(pr))
+    vq[:] = Q.reshape(-1, order="F").view(np.uint8)
+    outs = []
+    for g in (0, 1, 1, 1):
+        h.set_option("graph", g)
+        va[:] = A.reshape(-1, order="F").view(np.uint8)
+        vr[:] = R.reshape(-1, order="F").view(np.uint8)
+        if op == "inner":
+            h.ooc_inner(pq, m, pa, m, m, w1, w2, pr, w1, precision="fp16", tiling=tiling, block=block,
+                        budget=48 * MiB)
+        else:
+            h.ooc_outer(pq, m, pr, w1, pa, m, m, w1, w2, precision="fp16", tiling=tiling, block=block,
+                        budget=48 * MiB)
+        assert h.stats()["graph_replay"] == g
+        outs.append((va.copy(), vr.copy()))
+    for a_, r_ in outs[1:]:
+        np.testing.assert_array_equal(a_, outs[0][0])
+        np.testing.assert_array_equal(r_, outs[0][1])
+    for p_ in (pq, pa, pr):
+        h.host_free(p_)
