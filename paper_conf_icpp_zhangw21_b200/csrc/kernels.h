@@ -24,6 +24,9 @@ constexpr size_t LEAF_SMEM_BUDGET = 200 * 1024;
 constexpr int LEAF_WRING = 3;
 // rows per CTA the leaf's critical group holds in registers (8 rows x 256 threads)
 constexpr int LEAF_MAX_RP = 2048;
+// rows per CTA of a "tall" leaf panel (row state in shared memory, leaf.cu NR == 0): 8192 x 148 SMs
+// = 1.2M rows on one GPU (configs[3] at p = 1); the panel width then shrinks to what fits on chip
+constexpr int LEAF_MAX_RP_TALL = 8192;
 // smem column stride of the leaf panel slice: >= rows and == 4 (mod 32), so that the
 // float4 reads of 8 threads at the same row in 8 different columns hit 32 distinct banks
 __host__ __device__ inline int leaf_ld(int rows) { return ((rows + 31) / 32) * 32 + 4; }

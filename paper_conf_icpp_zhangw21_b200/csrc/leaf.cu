@@ -157,7 +157,10 @@ __device__ __forceinline__ void store4<float>(float* dst, float4 v) {
 }
 
 // CW: warps of the critical group (the other 16 - CW are the bulk group);
-// NR: rows per critical-group thread (rows_per_cta <= 32 CW NR)
+// NR: rows per critical-group thread (rows_per_cta <= 32 CW NR), their row state held in registers;
+// NR == 0 ("tall" panels, rows_per_cta up to LEAF_MAX_RP_TALL): the critical group loops over any
+// number of rows per thread with the row state read from the panel's shared-memory columns (u_t and
+// q_t replace a_t in place), for panels whose slices exceed the register rows
 template <typename T, int NR, int CW>
 __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p) {
   extern __shared__ __align__(16) float sp[];      // [w][LD] column-major panel slice
@@ -421,10 +424,11 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   PRO_STAMP(3);
   constexpr int BAR_Q = 4, BAR_W = 6;
   if (is_crit) {
-    // row state of this thread's rows rr[j] = tid + 32 CW j, j < NR
-    int rr[NR];
-    bool vr[NR];
-    float ru[NR], rq1[NR], rq2[NR], rq3[NR], ra2[NR], ra3[NR];
+    // row state of this thread's rows rr[j] = tid + 32 CW j, j < NR (NR == 0: none, see above)
+    constexpr int NRA = NR > 0 ? NR : 1;
+    int rr[NRA];
+    bool vr[NRA];
+    float ru[NRA], rq1[NRA], rq2[NRA], rq3[NRA], ra2[NRA], ra3[NRA];
 #pragma unroll
     for (int j = 0; j < NR; ++j) {
       rr[j] = threadIdx.x + GROUP * j;
@@ -511,7 +515,40 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       //      u_{t+1}.u_{t+1}, u_{t+1}.a_{t+2}, q_t.a_{t+2}, q_t.a_{t+3}, q_t.a_{t+4} ----
       const bool h2 = t + 2 < w, h3 = t + 3 < w, h4 = t + 4 < w;
       float s0, s1, s2, s3, s4;
-      {
+      if constexpr (NR == 0) {
+        // tall panel: rows tid + 32 CW j of the shared-memory slice, same arithmetic as below;
+        // u_{t+1} replaces a_{t+1} in column t+1 (no reader of a_{t+1} is left: the critical dots
+        // use a_{t+2..t+4}, the bulk round t-1 still running reads a_{t+2..t+4} and q's)
+        const float* wsrc = (t + 1 <= 4) ? sp + (more ? t + 1 : t) * LD : wring + ((t + 1) % LEAF_WRING) * LD;
+        float* ut = sp + t * LD;
+        const float* q1p = sp + (t >= 1 ? t - 1 : t) * LD;
+        const float* q2p = sp + (t >= 2 ? t - 2 : t) * LD;
+        const float* q3p = sp + (t >= 3 ? t - 3 : t) * LD;
+        const float* a2p = sp + (h2 ? t + 2 : t) * LD;
+        const float* a3p = sp + (h3 ? t + 3 : t) * LD;
+        const float* a4p = sp + (h4 ? t + 4 : t) * LD;
+        float* un = sp + (more ? t + 1 : t) * LD;
+        s0 = s1 = s2 = s3 = s4 = 0.0f;
+#pragma unroll 2
+        for (int r = threadIdx.x; r < rows; r += GROUP) {
+          const float u = ut[r];
+          const float q1 = t >= 1 ? q1p[r] : 0.0f, q2 = t >= 2 ? q2p[r] : 0.0f, q3 = t >= 3 ? q3p[r] : 0.0f;
+          const float wv = more ? wsrc[r] : 0.0f;
+          const float a2 = h2 ? a2p[r] : 0.0f, a3 = h3 ? a3p[r] : 0.0f, a4 = h4 ? a4p[r] : 0.0f;
+          const float q = u * inv;
+          float x = fmaf(-q3, c3, wv);
+          x = fmaf(-q2, c2, x);
+          x = fmaf(-q1, c1, x);
+          const float av = fmaf(-q, ct, x);
+          ut[r] = q;
+          if (more) un[r] = av;
+          s0 = fmaf(av, av, s0);
+          s1 = fmaf(av, a2, s1);
+          s2 = fmaf(q, a2, s2);
+          s3 = fmaf(q, a3, s3);
+          s4 = fmaf(q, a4, s4);
+        }
+      } else {
         const float* wsrc = (t + 1 <= 4) ? sp + (more ? t + 1 : t) * LD : wring + ((t + 1) % LEAF_WRING) * LD;
         const float* a4p = sp + (h4 ? t + 4 : t) * LD;
         float* ut = sp + t * LD;
@@ -553,7 +590,10 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
       }
       if (!more) {
-        // the last column: its rows of Q straight from registers
+        // the last column: its rows of Q straight from registers (tall: from this thread's smem rows)
+        if constexpr (NR == 0) {
+          for (int r = threadIdx.x; r < rows; r += GROUP) P[r0 + r + (int64_t)t * p.ldp] = Elem<T>::store(sp[t * LD + r]);
+        }
 #pragma unroll
         for (int j = 0; j < NR; ++j)
           if (vr[j]) P[r0 + rr[j] + (int64_t)t * p.ldp] = Elem<T>::store(rq1[j]);
@@ -608,6 +648,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
       }
       // q_t of this thread's rows to global memory (rounded once), inside the exchange wait
+      if constexpr (NR == 0) {
+        for (int r = threadIdx.x; r < rows; r += GROUP) P[r0 + r + (int64_t)t * p.ldp] = Elem<T>::store(sp[t * LD + r]);
+      }
 #pragma unroll
       for (int j = 0; j < NR; ++j)
         if (vr[j]) P[r0 + rr[j] + (int64_t)t * p.ldp] = Elem<T>::store(rq1[j]);
@@ -740,15 +783,18 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         const float* cf = coef[t % 3];
         const float* an = sp + (t + 3) * LD;
         float* wd = wring + ((t + 3) % LEAF_WRING) * LD;
-        // row pairs (2 pi, 2 pi + 1), pi = btid + BULK j: float2 loads, 4 independent chains
-        constexpr int NP = (NR * GROUP + 2 * BULK - 1) / (2 * BULK);
+        // row pairs (2 pi, 2 pi + 1), pi = btid + BULK (j + NP c): float2 loads, 4 independent chains;
+        // tall panels take their row pairs in chunks c of NP per thread
+        constexpr int NP = NR > 0 ? (NR * GROUP + 2 * BULK - 1) / (2 * BULK) : 4;
         const int npairs = (rows + 1) / 2;
+        const int nchunk = NR > 0 ? 1 : (npairs + NP * BULK - 1) / (NP * BULK);
+        for (int ch = 0; ch < nchunk; ++ch) {
         float2 e0[NP], e1[NP];
         int pb[NP];
 #pragma unroll
         for (int j = 0; j < NP; ++j) {
           e0[j] = e1[j] = make_float2(0.f, 0.f);
-          pb[j] = 2 * min(btid + BULK * j, LD / 2 - 1);   // pairs >= npairs: computed, not stored
+          pb[j] = 2 * min(btid + BULK * (j + NP * ch), LD / 2 - 1);   // pairs >= npairs: computed, not stored
         }
         int k = 0;
         for (; k + 4 <= t - 1; k += 4) {
@@ -780,10 +826,11 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
 #pragma unroll
         for (int j = 0; j < NP; ++j)
-          if (btid + BULK * j < npairs) {
+          if (btid + BULK * (j + NP * ch) < npairs) {
             const float2 av = *reinterpret_cast<const float2*>(an + pb[j]);
             *reinterpret_cast<float2*>(wd + pb[j]) = make_float2(av.x - (e0[j].x + e1[j].x), av.y - (e0[j].y + e1[j].y));
           }
+        }
       }
       BULK_STAMP(11);
       bar_arrive_n(BAR_W + (t & 1), LEAF_THREADS);
@@ -836,7 +883,8 @@ cudaError_t launch_leaf(const LeafParams& p, int grid, cudaStream_t st) {
   if (p.rows_per_cta <= 512) return launch_leaf_nr<T, 2, 8>(p, grid, st);
   if (p.rows_per_cta <= 1024) return launch_leaf_nr<T, 4, 8>(p, grid, st);
   if (p.rows_per_cta <= 2048) return launch_leaf_nr<T, 8, 8>(p, grid, st);
-  return cudaErrorInvalidValue;   // rows_per_cta > LEAF_MAX_RP: rejected by op_leaf
+  if (p.rows_per_cta <= LEAF_MAX_RP_TALL) return launch_leaf_nr<T, 0, 8>(p, grid, st);   // tall panel
+  return cudaErrorInvalidValue;   // rows_per_cta > LEAF_MAX_RP_TALL: rejected by op_leaf
 }
 
 int leaf_max_smem_rows(int w) { return (int)((LEAF_SMEM_BUDGET) / ((size_t)(w + LEAF_WRING) * sizeof(float))); }

@@ -373,7 +373,7 @@ static void leaf_geometry(Ctx* c, int64_t m, int* grid, int* rp) {
 int leaf_width_for(Ctx* c, int64_t m) {
   int G, rp;
   leaf_geometry(c, m, &G, &rp);
-  if (rp > LEAF_MAX_RP) return 0;
+  if (rp > LEAF_MAX_RP_TALL) return 0;
   int64_t wmax = (int64_t)LEAF_SMEM_BUDGET / ((int64_t)leaf_ld(rp) * 4) - LEAF_WRING;
   int64_t w = std::min<int64_t>({c->opt.leaf_width, (int64_t)LEAF_MAX_W, wmax});
   if (w >= 8) w &= ~int64_t(7);
@@ -384,9 +384,9 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
             int64_t col_offset, cudaStream_t st, bool r0_pre) {
   int G, rp;
   leaf_geometry(c, m, &G, &rp);
-  if (rp > LEAF_MAX_RP)
+  if (rp > LEAF_MAX_RP_TALL)
     return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: " + std::to_string(m) + " rows exceed " +
-                                              std::to_string(LEAF_MAX_RP) + " per CTA");
+                                              std::to_string(LEAF_MAX_RP_TALL) + " per CTA");
   if (w < 1 || w > LEAF_MAX_W || (size_t)(w + LEAF_WRING) * leaf_ld(rp) * 4 > LEAF_SMEM_BUDGET)
     return fail(c, RGSQR_ERR_UNSUPPORTED, "leaf: panel " + std::to_string(m) + "x" + std::to_string(w) +
                                               " does not fit on chip");

@@ -21,10 +21,11 @@ ap.add_argument("--prec", default="fp16")
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--host", action="store_true", help="use the host (out-of-core) path, 1 GiB budget")
 ap.add_argument("--pinned", action="store_true", help="host path with rgsqr_host_alloc buffers (CUDA-graph replay)")
+ap.add_argument("--budget-gib", type=float, default=1.0)
 ap.add_argument("--profile", action="store_true", help="per-kernel-class CUDA-event accounting (RGSQR_OPT_PROFILE)")
 a = ap.parse_args()
 build.build()
-st = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}[a.prec]
+st = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32", "tf32x3": "fp32"}[a.prec]
 A = gi.gaussian(a.m, a.n, seed=2, dtype=st)
 h = Handle(0)
 if a.profile:
@@ -46,7 +47,7 @@ else:
     Qd = torch.empty_like(Ad)
     Rd = torch.empty((a.n, a.n), dtype=torch.float32, device="cuda")
     for _ in range(a.reps):
-        h.factor_device(Ad, a.m, a.m, a.n, Qd, Rd, precision=a.prec, budget=1 << 30)
+        h.factor_device(Ad, a.m, a.m, a.n, Qd, Rd, precision=a.prec, budget=int(a.budget_gib * (1 << 30)))
 torch.cuda.synchronize()
 st = h.stats()
 print("stats", st)

@@ -147,3 +147,21 @@ def test_fused_bottom_node_matches_separate_products(h, prec):
     h.set_option("fuse_small", 1)
     assert oracle.r_rel_error(out[1][1], out[0][1]) < 2e-3
     assert oracle.r_rel_error(out[2][1], out[0][1]) < 2e-3
+
+
+@pytest.mark.parametrize("prec", ["fp16", "bf16"])
+def test_tall_panel_leaves(h, prec):
+    """More rows than the leaf's register rows (> 2048 per CTA, configs[3]-shaped at p <= 2): the planner picks
+    the widest leaf that fits on chip (8 here) and the tall leaf kernel; parity as test_gaussian_vs_oracle."""
+    m, n = 600000, 96
+    st = STOR[prec]
+    A = gi.gaussian(m, n, seed=4, dtype=st)
+    X = gi.to_float64(A, st)
+    rc, Q, R = run(h, A, st, prec, m, n)
+    assert rc == 0
+    ref = oracle.rgs(X, leaf=8)
+    assert oracle.is_upper_triangular(R)
+    assert oracle.backward_error(X, Q, R) <= TOL[prec]
+    assert oracle.r_rel_error(R, ref.R) <= TOL[prec]
+    # element-wise on R against the oracle's R (the leading block)
+    np.testing.assert_allclose(R[:32, :32], ref.R[:32, :32], atol=TOL[prec] * np.abs(ref.R).max())

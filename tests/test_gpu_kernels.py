@@ -69,7 +69,10 @@ def test_outer_product(h, prec, storage, m, w1, w2):
 
 
 @pytest.mark.parametrize("prec,storage", PRECS)
-@pytest.mark.parametrize("m,w", [(20000, 64), (4096, 32), (1000, 7), (300, 64), (65536, 64), (131072, 48), (262144, 24)])
+# (400000, 15), (600000, 9), (1048576, 4): more than LEAF_MAX_RP = 2048 rows per CTA -> the tall leaf
+# (row state in shared memory, kernels.h LEAF_MAX_RP_TALL); widths are the widest that fit on chip
+@pytest.mark.parametrize("m,w", [(20000, 64), (4096, 32), (1000, 7), (300, 64), (65536, 64), (131072, 48), (262144, 24),
+                                 (400000, 15), (600000, 9), (1048576, 4)])
 def test_leaf_cgs(h, prec, storage, m, w):
     A = _rand(m, w, 31, storage)
     X = gi.to_float64(A, storage)
