@@ -797,6 +797,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           pb[j] = 2 * min(btid + BULK * (j + NP * ch), LD / 2 - 1);   // pairs >= npairs: computed, not stored
         }
         int k = 0;
+#pragma unroll 2
         for (; k + 4 <= t - 1; k += 4) {
           const float4 c0 = *reinterpret_cast<const float4*>(cf + k);
 #pragma unroll
