@@ -21,7 +21,7 @@ for (m, n) in [(8192, 256), (65536, 256), (65536, 2048)]:
     A = gi.to_storage(A64, "fp32")
     X = gi.to_float64(A, "fp32")
     ref = oracle.gram_cholesky_r(X)
-    for splitk, chain in [(0, 2), (1, 2), (4, 2), (16, 2), (0, 1)]:
+    for splitk, chain in [(0, 2), (1, 2), (16, 2), (0, 4), (1, 4), (4, 4), (16, 4), (0, 8), (1, 8)]:
         h.set_option("splitk", splitk)
         h.set_option("x3_chain", chain)
         Ad = to_dev(A, "fp32")
@@ -40,7 +40,7 @@ A = gi.gaussian(65536, 8192, seed=2, dtype="fp32")
 Ad = to_dev(A, "fp32")
 Qd = torch.empty_like(Ad)
 R = torch.empty((8192, 8192), dtype=torch.float32, device="cuda")
-for chain in (2, 4, 0):
+for chain in (2, 4, 8):
     h.set_option("x3_chain", chain)
     h.factor_device(Ad, 65536, 65536, 8192, Qd, R, precision="tf32x3")
     torch.cuda.synchronize()
