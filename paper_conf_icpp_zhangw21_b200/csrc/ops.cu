@@ -206,7 +206,10 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
   // recursion's nodes (<= ~4 waves) the x-fastest order measured faster (RGSQR_GROUP_M overrides)
   static const int env_group = getenv("RGSQR_GROUP_M") ? atoi(getenv("RGSQR_GROUP_M")) : -1;
   GemmExtra gx;
-  gx.group_m = env_group >= 0 ? env_group : (tiles > 8 * (int64_t)c->num_sms ? 16 : 0);
+  // (TF32X3's 128 x 128 fp32 tiles need ~128 B/clk/SM of operands: grouping 4 M-tiles keeps more of
+  // them in L2 there, 108 -> 105 ms at configs[1]'s shape)
+  gx.group_m = env_group >= 0 ? env_group
+                              : (tiles > 8 * (int64_t)c->num_sms ? 16 : (x3 && tiles > 2 * (int64_t)c->num_sms ? 4 : 0));
   // One wave: tiles x splits <= SMs (rounding up put 152 CTAs on 148 SMs at w1 = w2 = 512 and
   // doubled the kernel time: 57 vs 37 us, profiles/r1_splitk_scan.txt).
   int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : c->num_sms / tiles);
