@@ -265,6 +265,18 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   if (s == 2 && w1 <= 1024) bn = std::min(bn, 128);
   CUtensorMap ma, mb, mc;
   std::string err;
+  // TMA needs 16-byte row pitches: a narrow node's R12 (w1 * s < 16 bytes, the 4-column leaves of tall
+  // panels, R31) is copied to a padded scratch block first
+  const size_t mark = c->arena.mark();
+  if ((ldr * s) % 16 != 0) {
+    const int64_t ldp = (w1 * s + 15) / 16 * 16 / s;
+    void* pad = c->arena.alloc((size_t)ldp * w2 * s);
+    if (!pad) return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "outer: no space for the padded R12 operand");
+    RGSQR_CUDA(c, cudaMemcpy2DAsync(pad, (size_t)ldp * s, R12op, (size_t)ldr * s, (size_t)w1 * s, (size_t)w2,
+                                    cudaMemcpyDeviceToDevice, st));
+    R12op = pad;
+    ldr = ldp;
+  }
   if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
       !encode_tmap_2d(&mb, prec, R12op, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err) ||
       !encode_tmap_2d(&mc, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, 128, 64, &err, 2))
@@ -272,7 +284,7 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   const bool x3 = Q1lo != nullptr && R12lo != nullptr;
   CUtensorMap ma2, mb2;
   if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)m * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
-             !encode_tmap_2d(&mb2, prec, R12lo, (uint64_t)w1, (uint64_t)w2, (uint64_t)w1 * s, BK, bn, &err)))
+             !encode_tmap_2d(&mb2, prec, R12lo, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err)))
     return fail(c, RGSQR_ERR_INVALID_ARG, "outer (tf32x3): " + err);
   NNParams p{};
   p.tiles_m = (int)((m + 127) / 128);
@@ -291,6 +303,7 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   c->kend(2, st, kb, (x3 ? 6.0 : 2.0) * m * w1 * w2,
           (double)m * w1 * s * (x3 ? 2 : 1) + (double)w1 * w2 * s * (x3 ? 2 : 1) + 2.0 * m * w2 * s);
   c->stats.n_nn_launches++;
+  c->arena.release(mark);   // (stream-ordered reuse: later kernels on st run after this one)
   return RGSQR_OK;
 }
 
@@ -347,14 +360,15 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
       const size_t mark = c->arena.mark();
       float* q_hi = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
       float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
-      float* r_hi = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
-      float* r_lo = static_cast<float*>(c->arena.alloc((size_t)w1 * w2 * 4));
+      const int64_t lr = (w1 + 3) / 4 * 4;   // 16-byte TMA pitch
+      float* r_hi = static_cast<float*>(c->arena.alloc((size_t)lr * w2 * 4));
+      float* r_lo = static_cast<float*>(c->arena.alloc((size_t)lr * w2 * 4));
       if (!q_hi || !q_lo || !r_hi || !r_lo)
         return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "outer (tf32x3): no space for hi/lo operands");
       RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, m, q_lo, m, m, w1, c->num_sms, st));
-      RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(R12op), ldr, r_hi, w1, r_lo, w1, w1, w2, c->num_sms, st));
+      RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(R12op), ldr, r_hi, lr, r_lo, lr, w1, w2, c->num_sms, st));
       c->stats.n_other_launches += 2;
-      int rc = op_outer_t<float>(c, prec, q_hi, m, r_hi, w1, A2, lda, m, w1, w2, st, q_lo, r_lo);
+      int rc = op_outer_t<float>(c, prec, q_hi, m, r_hi, lr, A2, lda, m, w1, w2, st, q_lo, r_lo);
       c->arena.release(mark);
       return rc;
     }
