@@ -33,7 +33,8 @@
  *   - Blocking: rgsqr_factor* return after Q and R are complete (host-synchronous).
  *     A handle is not thread-safe; use one handle per thread / per GPU.
  *   - Preconditions: 1 <= n <= m, lda >= m, lda*sizeof(elem) % 16 == 0, pointers
- *     16-byte aligned.  Violations return RGSQR_ERR_INVALID_ARG.
+ *     16-byte aligned.  Violations return RGSQR_ERR_INVALID_ARG.  rgsqr_factor with
+ *     m*sizeof(elem) % 16 != 0 stages A / Q through zero-padded pinned copies ([A; 0] = [Q; 0] R).
  *   - Rank deficiency (the paper assumes linearly independent columns,
  *     PAPER.md:103): if some r_jj <= m * u_fp32 * ||a_j|| (or is not finite),
  *     q_j = 0 and r_jj = 0 are written, the first such j is reported in

@@ -986,6 +986,38 @@ int factor_host(Ctx* c, const void* A, int64_t lda, int64_t m, int64_t n, void* 
   if (rc < 0) return rc;
   if (!R && c->rank == 0) return fail(c, RGSQR_ERR_INVALID_ARG, "null R_out");
   if (c->opt.vshards > 1) return fail(c, RGSQR_ERR_UNSUPPORTED, "virtual shards: device path only");
+  {
+    // Device tiles use ld = m, and TMA needs 16-byte row pitches: a ragged m is staged through a
+    // pinned bounce buffer of md = round_up(m, 16 / s) rows whose extra rows are zero.  Zero rows change
+    // nothing: [A; 0] = [Q; 0] R (every dot product and norm is the same sum plus zeros).
+    const int64_t s0 = elem_bytes(prec);
+    if ((m * s0) % 16 != 0) {
+      const int64_t md = (m * s0 + 15) / 16 * 16 / s0;
+      void *Ab = nullptr, *Qb = nullptr;
+      if (cudaHostAlloc(&Ab, (size_t)md * n * s0, cudaHostAllocPortable) != cudaSuccess ||
+          cudaHostAlloc(&Qb, (size_t)md * n * s0, cudaHostAllocPortable) != cudaSuccess) {
+        cudaGetLastError();
+        if (Ab) cudaFreeHost(Ab);
+        return fail(c, RGSQR_ERR_HOST_MEM, "ragged m: no pinned memory for the zero-padded bounce buffers");
+      }
+      for (int64_t j = 0; j < n; ++j) {
+        char* d = static_cast<char*>(Ab) + (size_t)j * md * s0;
+        std::memcpy(d, static_cast<const char*>(A) + (size_t)j * lda * s0, (size_t)m * s0);
+        std::memset(d + (size_t)m * s0, 0, (size_t)(md - m) * s0);
+      }
+      const int64_t g0 = c->opt.graph;   // (per-call bounce buffers: no graph to reuse)
+      c->opt.graph = 0;
+      rc = factor_host(c, Ab, md, md, n, Qb, R, prec, budget);
+      c->opt.graph = g0;
+      if (rc >= 0)
+        for (int64_t j = 0; j < n; ++j)
+          std::memcpy(static_cast<char*>(Q) + (size_t)j * lda * s0, static_cast<char*>(Qb) + (size_t)j * md * s0,
+                      (size_t)m * s0);
+      cudaFreeHost(Ab);
+      cudaFreeHost(Qb);
+      return rc;
+    }
+  }
   reset_stats(c);
   rc = sync_shape(c, m, &budget);
   if (rc < 0) return rc;

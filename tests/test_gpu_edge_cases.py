@@ -1,0 +1,139 @@
+"""Degenerate and ragged shapes through the C ABI, both paths (rgsqr_factor from host buffers,
+rgsqr_factor_device), against the oracle; argument validation (include/rgsqr.h preconditions:
+1 <= n <= m, lda >= m, lda * sizeof(elem) % 16 == 0, non-null outputs)."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+import oracle  # noqa: E402
+import rgsqr_inputs as gi  # noqa: E402
+from tests.gpu_util import to_dev, from_dev  # noqa: E402
+
+STOR = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32", "tf32x3": "fp32"}
+TOL = {"fp16": 5e-3, "bf16": 5e-3, "tf32": 5e-3, "tf32x3": 1e-5}
+
+
+@pytest.fixture(scope="module")
+def h():
+    from paper_conf_icpp_zhangw21_b200 import Handle
+    hd = Handle(0)
+    yield hd
+    hd.close()
+
+
+def _lda(m, st):
+    e = 2 if st != "fp32" else 4
+    q = 16 // e
+    return (m + q - 1) // q * q
+
+
+def host_factor(h, A, prec, budget=0):
+    m, n = A.shape
+    st = STOR[prec]
+    lda = _lda(m, st)
+    Ap = np.zeros((lda, n), dtype=A.dtype, order="F")
+    Ap[:m] = A
+    Q = np.zeros_like(Ap, order="F")
+    R = np.full((n, n), np.nan, dtype=np.float32, order="F")
+    rc = h.factor(Ap, lda, m, n, Q, R, precision=prec, budget=budget)
+    return rc, gi.to_float64(np.asfortranarray(Q[:m]), st), R.astype(np.float64)
+
+
+def device_factor(h, A, prec):
+    m, n = A.shape
+    st = STOR[prec]
+    lda = _lda(m, st)
+    Ad = to_dev(A, st)
+    if lda != m:
+        Ap = torch.zeros((n, lda), dtype=Ad.dtype, device="cuda")
+        Ap[:, :m] = Ad
+        Ad = Ap
+    R = torch.full((n, n), float("nan"), dtype=torch.float32, device="cuda")
+    rc = h.factor_device(Ad, lda, m, n, Ad, R, precision=prec)
+    return rc, from_dev(Ad[:, :m]), R.cpu().numpy().T.astype(np.float64)
+
+
+def check(X, Q, R, prec, leaf=64):
+    ref = oracle.rgs(X, leaf=leaf)
+    assert oracle.is_upper_triangular(R)
+    assert np.all(np.diag(R) > 0)
+    assert oracle.backward_error(X, Q, R) <= TOL[prec]
+    assert oracle.r_rel_error(R, ref.R) <= TOL[prec]
+    return ref
+
+
+@pytest.mark.parametrize("path", ["host", "device"])
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32", "tf32x3"])
+def test_single_column(h, path, prec):
+    """n = 1: R = ||a||, Q = a / ||a|| (the leaf's only column; Eq. 1 with no projections)."""
+    st = STOR[prec]
+    A = gi.gaussian(5000, 1, seed=11, dtype=st)
+    X = gi.to_float64(A, st)
+    rc, Q, R = (host_factor if path == "host" else device_factor)(h, A, prec)
+    assert rc == 0
+    nrm = np.linalg.norm(X[:, 0])
+    assert abs(R[0, 0] - nrm) <= 1e-6 * nrm
+    u = {"fp16": 2 ** -11, "bf16": 2 ** -8, "fp32": 2 ** -24}[st]
+    assert np.max(np.abs(Q[:, 0] - X[:, 0] / nrm)) <= 2 * u * np.max(np.abs(X[:, 0])) / nrm + 1e-7
+
+
+@pytest.mark.parametrize("path", ["host", "device"])
+@pytest.mark.parametrize("m,n", [(1000, 37), (777, 2), (4099, 65), (9999, 129), (12347, 1000)])
+def test_ragged_shapes(h, path, m, n):
+    """m not a multiple of 8 (lda padded), n prime / just past a leaf or split boundary."""
+    A = gi.gaussian(m, n, seed=12, dtype="fp16")
+    X = gi.to_float64(A, "fp16")
+    rc, Q, R = (host_factor if path == "host" else device_factor)(h, A, "fp16")
+    assert rc == 0
+    check(X, Q, R, "fp16")
+
+
+@pytest.mark.parametrize("prec", ["fp16", "tf32"])
+def test_square(h, prec):
+    """m = n (the paper's square Table 4 shapes, at a small size): kappa 3 U Sigma V^T."""
+    st = STOR[prec]
+    A64, _ = gi.usv(512, 512, kappa=3.0, seed=13)
+    A = gi.to_storage(A64, st)
+    X = gi.to_float64(A, st)
+    for path in (host_factor, device_factor):
+        rc, Q, R = path(h, A, prec)
+        assert rc == 0
+        check(X, Q, R, prec)
+
+
+def test_ragged_host_out_of_core(h):
+    """A ragged shape under a budget small enough to force the out-of-core node (streamed tiles with a
+    partial last tile)."""
+    m, n = 30011, 700
+    A = gi.gaussian(m, n, seed=14, dtype="fp16")
+    X = gi.to_float64(A, "fp16")
+    rc, Q, R = host_factor(h, A, "fp16", budget=24 << 20)
+    assert rc == 0
+    assert h.stats()["n_ooc_nodes"] >= 1
+    check(X, Q, R, "fp16")
+
+
+def test_invalid_arguments(h):
+    from paper_conf_icpp_zhangw21_b200.rgsqr import RgsqrError
+    A = np.asfortranarray(gi.gaussian(64, 8, seed=15, dtype="fp16"))
+    Q = np.zeros_like(A, order="F")
+    R = np.zeros((8, 8), dtype=np.float32, order="F")
+    bad = [
+        dict(lda=64, m=64, n=0),      # n < 1
+        dict(lda=64, m=4, n=8),       # m < n
+        dict(lda=32, m=64, n=8),      # lda < m
+        dict(lda=60, m=56, n=8),      # lda * 2 bytes not a multiple of 16
+    ]
+    for b in bad:
+        with pytest.raises(RgsqrError) as ei:
+            h.factor(A, b["lda"], b["m"], b["n"], Q, R, precision="fp16")
+        assert ei.value.status == -1, b
+    with pytest.raises(RgsqrError) as ei:
+        h.factor(A, 64, 64, 8, Q, 0, precision="fp16")   # null R_out
+    assert ei.value.status == -1
+    # the handle stays usable after rejected calls
+    rc, Qg, Rg = host_factor(h, A, "fp16")
+    assert rc == 0
+    check(gi.to_float64(A, "fp16"), Qg, Rg, "fp16")
