@@ -149,6 +149,9 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
   int rc = ensure_arena(c, cap);
   if (rc < 0) return rc;
   Pipe P{c, c->compute(), c->st_h2d, c->st_d2h, s, {}};
+  // device leading dimension of resident panels / column blocks: TMA needs 16-byte pitches, so a ragged m is
+  // padded (the tensor maps keep m rows; the pad rows are never read)
+  const int64_t md = (m * s + 15) / 16 * 16 / s;
   if (c->opt.serialize) P.sh = P.sd = P.sc;
   int K = (int)c->opt.ring_depth;   // (lowered to >= 2 slots when the budget is tight)
   P.freed.assign(K, nullptr);
@@ -206,25 +209,25 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
     } else if (op == 0) {
       // ---- Fig. 4: Q1 (the panel) resident, column blocks of A2, R12 blocks out ----
       const int64_t b = std::min<int64_t>(w2, block > 0 ? block : 16384);
-      char* dQ = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
-      const size_t per = (size_t)m * b * s + (size_t)w1 * b * 4 + 512;
+      char* dQ = static_cast<char*>(c->arena.alloc((size_t)md * w1 * s));
+      const size_t per = (size_t)md * b * s + (size_t)w1 * b * 4 + 512;
       if (!dQ || !fits_slots(per))
         return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc inner (blocking): panel + 2 column blocks do not fit");
       char* ring = static_cast<char*>(c->arena.alloc((size_t)K * per));
-      if ((rc = P.up(dQ, m, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
+      if ((rc = P.up(dQ, md, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
       cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
       int64_t i = 0;
       for (int64_t c0 = 0; c0 < w2; c0 += b, ++i) {
         const int64_t bw = std::min(b, w2 - c0);
         const int k = (int)(i % K);
         char* sa = ring + (size_t)k * per;
-        float* sr = reinterpret_cast<float*>(sa + (size_t)m * b * s);
+        float* sr = reinterpret_cast<float*>(sa + (size_t)md * b * s);
         if (P.freed[k]) cudaStreamWaitEvent(P.sh, P.freed[k], 0);
-        if ((rc = P.up(sa, m, ha, lda, 0, c0, m, bw, s)) < 0) return rc;
+        if ((rc = P.up(sa, md, ha, lda, 0, c0, m, bw, s)) < 0) return rc;
         cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
         if (P.freed[k]) cudaStreamWaitEvent(P.sc, P.freed[k], 0);   // the block's previous R12 is out
         cudaEvent_t a = P.seg_begin(P.sc);
-        rc = op_inner(c, prec, dQ, m, sa, m, m, w1, bw, sr, w1, nullptr, w1, 0, P.sc, false);
+        rc = op_inner(c, prec, dQ, md, sa, md, m, w1, bw, sr, w1, nullptr, w1, 0, P.sc, false);
         if (rc < 0) return rc;
         P.seg_end(2, P.sc, a);
         cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);
@@ -272,12 +275,12 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
         // ---- Fig. 6: Q1 resident too, b x b tiles of A2 in and out ----
         const int64_t b = block > 0 ? block : 16384;
         const int64_t b1 = std::min(b, (m + 127) / 128 * 128), b2 = std::min(b, w2);
-        char* dQ = static_cast<char*>(c->arena.alloc((size_t)m * w1 * s));
+        char* dQ = static_cast<char*>(c->arena.alloc((size_t)md * w1 * s));
         const size_t per = (size_t)b1 * b2 * s;
         if (!dQ || !fits_slots(per))
           return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "ooc outer (blocking): Q1 + R12 + 2 tiles do not fit");
         char* ring = static_cast<char*>(c->arena.alloc((size_t)K * per));
-        if ((rc = P.up(dQ, m, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
+        if ((rc = P.up(dQ, md, hq, ldq, 0, 0, m, w1, s)) < 0) return rc;
         cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
         int64_t i = 0;
         for (int64_t r0 = 0; r0 < m; r0 += b1)
@@ -289,7 +292,7 @@ int ooc_gemm(Ctx* c, int op, int tiling, int64_t block, const void* Q1, int64_t 
             if ((rc = P.up(sa, b1, ha, lda, r0, c0, tr, tc, s)) < 0) return rc;
             cudaStreamWaitEvent(P.sc, P.mark(P.sh), 0);
             cudaEvent_t a = P.seg_begin(P.sc);
-            rc = op_outer(c, prec, dQ + (size_t)r0 * s, m, dRop + (size_t)c0 * w1 * s, w1, sa, b1, tr, w1, tc, P.sc);
+            rc = op_outer(c, prec, dQ + (size_t)r0 * s, md, dRop + (size_t)c0 * w1 * s, w1, sa, b1, tr, w1, tc, P.sc);
             if (rc < 0) return rc;
             P.seg_end(2, P.sc, a);
             cudaStreamWaitEvent(P.sd, P.mark(P.sc), 0);

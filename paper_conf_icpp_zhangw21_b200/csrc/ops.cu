@@ -160,17 +160,18 @@ static int op_inner_local(Ctx* c, int prec, const void* Q1, int64_t ldq, const v
   if (prec != RGSQR_TF32X3)
     return op_inner_once<T>(c, prec, Q1, ldq, A2, lda, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st);
   const size_t mark = c->arena.mark();
-  float* q_hi = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
-  float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
-  float* a_hi = static_cast<float*>(c->arena.alloc((size_t)m * w2 * 4));
-  float* a_lo = static_cast<float*>(c->arena.alloc((size_t)m * w2 * 4));
+  const int64_t md = (m + 3) / 4 * 4;   // hi / lo leading dimension (16-byte TMA pitch)
+  float* q_hi = static_cast<float*>(c->arena.alloc((size_t)md * w1 * 4));
+  float* q_lo = static_cast<float*>(c->arena.alloc((size_t)md * w1 * 4));
+  float* a_hi = static_cast<float*>(c->arena.alloc((size_t)md * w2 * 4));
+  float* a_lo = static_cast<float*>(c->arena.alloc((size_t)md * w2 * 4));
   if (!q_hi || !q_lo || !a_hi || !a_lo)
     return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "inner (tf32x3): no space for the hi/lo operands");
-  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, m, q_lo, m, m, w1, c->num_sms, st));
-  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(A2), lda, a_hi, m, a_lo, m, m, w2, c->num_sms, st));
+  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, md, q_lo, md, m, w1, c->num_sms, st));
+  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(A2), lda, a_hi, md, a_lo, md, m, w2, c->num_sms, st));
   c->stats.n_other_launches += 2;
   // one GEMM over the three operand segments (K extended 3x): a single split-K reduction
-  int rc = op_inner_once<T>(c, prec, q_hi, m, a_hi, m, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st, q_lo, a_lo);
+  int rc = op_inner_once<T>(c, prec, q_hi, md, a_hi, md, m, w1, w2, R12, ldr, R12op, ldop, accumulate, st, q_lo, a_lo);
   c->arena.release(mark);
   return rc;
 }
@@ -189,8 +190,8 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
       !encode_tmap_2d(&mb, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, BK, bn, &err))
     return fail(c, RGSQR_ERR_INVALID_ARG, "inner: " + err);
   const bool x3 = Q1lo != nullptr && A2lo != nullptr;
-  if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)m * s, BK, 128, &err) ||
-             !encode_tmap_2d(&mb2, prec, A2lo, (uint64_t)m, (uint64_t)w2, (uint64_t)m * s, BK, bn, &err)))
+  if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, BK, 128, &err) ||
+             !encode_tmap_2d(&mb2, prec, A2lo, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, BK, bn, &err)))
     return fail(c, RGSQR_ERR_INVALID_ARG, "inner (tf32x3): " + err);
   GemmParams p{};
   p.M = w1;
@@ -283,7 +284,7 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
     return fail(c, RGSQR_ERR_INVALID_ARG, "outer: " + err);
   const bool x3 = Q1lo != nullptr && R12lo != nullptr;
   CUtensorMap ma2, mb2;
-  if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)m * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
+  if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
              !encode_tmap_2d(&mb2, prec, R12lo, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err)))
     return fail(c, RGSQR_ERR_INVALID_ARG, "outer (tf32x3): " + err);
   NNParams p{};
@@ -358,17 +359,18 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
       // A2 <- A2 - (Q1h R12l + Q1l R12h + Q1h R12h): one NN pass over the three segments,
       // hi = RN_tf32(x), lo = RN_tf32(x - hi) (R25)
       const size_t mark = c->arena.mark();
-      float* q_hi = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
-      float* q_lo = static_cast<float*>(c->arena.alloc((size_t)m * w1 * 4));
+      const int64_t md = (m + 3) / 4 * 4;    // 16-byte TMA pitch
+      float* q_hi = static_cast<float*>(c->arena.alloc((size_t)md * w1 * 4));
+      float* q_lo = static_cast<float*>(c->arena.alloc((size_t)md * w1 * 4));
       const int64_t lr = (w1 + 3) / 4 * 4;   // 16-byte TMA pitch
       float* r_hi = static_cast<float*>(c->arena.alloc((size_t)lr * w2 * 4));
       float* r_lo = static_cast<float*>(c->arena.alloc((size_t)lr * w2 * 4));
       if (!q_hi || !q_lo || !r_hi || !r_lo)
         return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "outer (tf32x3): no space for hi/lo operands");
-      RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, m, q_lo, m, m, w1, c->num_sms, st));
+      RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, md, q_lo, md, m, w1, c->num_sms, st));
       RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(R12op), ldr, r_hi, lr, r_lo, lr, w1, w2, c->num_sms, st));
       c->stats.n_other_launches += 2;
-      int rc = op_outer_t<float>(c, prec, q_hi, m, r_hi, lr, A2, lda, m, w1, w2, st, q_lo, r_lo);
+      int rc = op_outer_t<float>(c, prec, q_hi, md, r_hi, lr, A2, lda, m, w1, w2, st, q_lo, r_lo);
       c->arena.release(mark);
       return rc;
     }

@@ -137,3 +137,47 @@ def test_invalid_arguments(h):
     rc, Qg, Rg = host_factor(h, A, "fp16")
     assert rc == 0
     check(gi.to_float64(A, "fp16"), Qg, Rg, "fp16")
+
+
+@pytest.mark.parametrize("prec", ["fp16", "tf32"])
+@pytest.mark.parametrize("tiling,block", [(0, 2048), (1, 128)])
+def test_ooc_gemms_ragged_m(h, prec, tiling, block):
+    """The standalone OOC GEMMs (Tables 1/2 operations) with m not a multiple of the 16-byte row quantum
+    (lda padded): R12 = Q1^T A2 and A2 - Q1 R12 against fp64 products of the stored operands (bounds as
+    tests/test_gpu_ooc_gemm.py)."""
+    st = STOR[prec]
+    m, w1, w2 = 20011, 192, 264
+    lda = _lda(m, st)
+    Q = np.zeros((lda, w1), dtype=gi.storage_numpy_dtype(st), order="F")
+    A = np.zeros((lda, w2), dtype=gi.storage_numpy_dtype(st), order="F")
+    Q[:m] = gi.gaussian(m, w1, seed=21, dtype=st)
+    A[:m] = gi.gaussian(m, w2, seed=22, dtype=st)
+    Xq, Xa = gi.to_float64(np.asfortranarray(Q[:m]), st), gi.to_float64(np.asfortranarray(A[:m]), st)
+    c = 1e-4 if st != "fp32" else 2e-3
+    budget = (48 << 20) * (2 if st == "fp32" else 1)
+    R = np.full((w1, w2), np.nan, dtype=np.float32, order="F")
+    h.ooc_inner(Q, lda, A, lda, m, w1, w2, R, w1, precision=prec, tiling=tiling, block=block, budget=budget)
+    assert np.all(np.abs(R - Xq.T @ Xa) <= c * (np.abs(Xq).T @ np.abs(Xa)))
+    Rin = np.asfortranarray((np.random.default_rng(2).standard_normal((w1, w2)) / np.sqrt(w1)).astype(np.float32))
+    Rop = gi.to_float64(gi.to_storage(Rin.astype(np.float64), st), st)
+    A2 = np.array(A, order="F", copy=True)
+    h.ooc_outer(Q, lda, Rin, w1, A2, lda, m, w1, w2, precision=prec, tiling=tiling, block=block, budget=budget)
+    got = gi.to_float64(np.asfortranarray(A2[:m]), st)
+    ref = Xa - Xq @ Rop
+    u = {"fp16": 2.0 ** -11, "fp32": 2.0 ** -24}[st]
+    bound = u * np.abs(ref) + c * (np.abs(Xq) @ np.abs(Rop)) + 1e-30
+    assert np.all(np.abs(got - ref) <= bound)
+    assert np.all(A2[m:] == A[m:])   # rows past m untouched
+
+
+@pytest.mark.parametrize("path", ["host", "device"])
+@pytest.mark.parametrize("prec", ["tf32", "tf32x3"])
+@pytest.mark.parametrize("m,n", [(777, 40), (4099, 65)])
+def test_ragged_shapes_fp32_storage(h, path, prec, m, n):
+    """fp32 storage with m % 4 != 0: the TF32X3 hi / lo operand copies get a padded leading dimension."""
+    st = STOR[prec]
+    A = gi.gaussian(m, n, seed=16, dtype=st)
+    X = gi.to_float64(A, st)
+    rc, Q, R = (host_factor if path == "host" else device_factor)(h, A, prec)
+    assert rc == 0
+    check(X, Q, R, prec)
