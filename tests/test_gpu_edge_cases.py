@@ -181,3 +181,30 @@ def test_ragged_shapes_fp32_storage(h, path, prec, m, n):
     rc, Q, R = (host_factor if path == "host" else device_factor)(h, A, prec)
     assert rc == 0
     check(X, Q, R, prec)
+
+
+@pytest.mark.parametrize("path", ["host", "device"])
+@pytest.mark.parametrize("m,n", [(1, 1), (8, 8), (16, 3), (100, 100)])
+def test_tiny(h, path, m, n):
+    """Smallest problems: a 1 x 1 matrix (R = |a|, Q = sign(a)), tiny square and tiny tall ones."""
+    A64, _ = gi.usv(m, n, kappa=2.0, seed=17) if n > 1 else (np.array([[-3.0]] * m), None)
+    A = gi.to_storage(A64, "fp32")
+    X = gi.to_float64(A, "fp32")
+    rc, Q, R = (host_factor if path == "host" else device_factor)(h, A, "tf32x3")
+    assert rc == 0
+    check(X, Q, R, "tf32x3")
+
+
+@pytest.mark.parametrize("leaf", [8, 16, 24, 32])
+def test_leaf_width_option(h, leaf):
+    """RGSQR_OPT_LEAF_WIDTH (reading R3): narrower leaves give the same factorization within tolerance."""
+    A = gi.gaussian(8192, 200, seed=18, dtype="fp16")
+    X = gi.to_float64(A, "fp16")
+    h.set_option("leaf_width", leaf)
+    try:
+        rc, Q, R = device_factor(h, A, "fp16")
+    finally:
+        h.set_option("leaf_width", 64)
+    assert rc == 0
+    check(X, Q, R, "fp16", leaf=leaf)
+    assert h.stats()["n_leaf_launches"] >= 200 // leaf
