@@ -280,13 +280,18 @@ static int op_outer_t(Ctx* c, int prec, const void* Q1, int64_t ldq, const void*
   }
   if (!encode_tmap_2d(&ma, prec, Q1, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
       !encode_tmap_2d(&mb, prec, R12op, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err) ||
-      !encode_tmap_2d(&mc, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, 128, 64, &err, 2))
+      !encode_tmap_2d(&mc, prec, A2, (uint64_t)m, (uint64_t)w2, (uint64_t)lda * s, 128, 64, &err, 2)) {
+    c->arena.release(mark);
     return fail(c, RGSQR_ERR_INVALID_ARG, "outer: " + err);
+  }
   const bool x3 = Q1lo != nullptr && R12lo != nullptr;
   CUtensorMap ma2, mb2;
   if (x3 && (!encode_tmap_2d(&ma2, prec, Q1lo, (uint64_t)m, (uint64_t)w1, (uint64_t)ldq * s, EPB, BK, &err, s == 4 ? 1 : 0) ||
              !encode_tmap_2d(&mb2, prec, R12lo, (uint64_t)w1, (uint64_t)w2, (uint64_t)ldr * s, BK, bn, &err)))
+  {
+    c->arena.release(mark);
     return fail(c, RGSQR_ERR_INVALID_ARG, "outer (tf32x3): " + err);
+  }
   NNParams p{};
   p.tiles_m = (int)((m + 127) / 128);
   p.tiles_n = (int)((w2 + bn - 1) / bn);

@@ -208,3 +208,31 @@ def test_leaf_width_option(h, leaf):
     assert rc == 0
     check(X, Q, R, "fp16", leaf=leaf)
     assert h.stats()["n_leaf_launches"] >= 200 // leaf
+
+
+@pytest.mark.parametrize("algo,reorth,prec", [(1, 0, "fp16"), (2, 0, "fp16"), (0, 1, "fp16"), (0, 0, "tf32x3"),
+                                              (1, 0, "tf32"), (2, 1, "bf16")])
+def test_ragged_out_of_core_modes(h, algo, reorth, prec):
+    """Ragged m and n under an out-of-core budget through the blocked (1) / fused-blocked (2) algorithms,
+    CGS2 and TF32X3: every executor mode with a partial last row tile and odd widths."""
+    st = STOR[prec]
+    m, n = 20011, 333
+    A = gi.gaussian(m, n, seed=19, dtype=st)
+    X = gi.to_float64(A, st)
+    h.set_option("algo", algo)
+    h.set_option("block_cols", 128)
+    h.set_option("reorth", reorth)
+    try:
+        budget = (12 << 20) * (2 if st == "fp32" else 1) * (3 if prec == "tf32x3" else 1)
+        rc, Q, R = host_factor(h, A, prec, budget=budget)
+        ooc = h.stats()["n_ooc_nodes"]
+    finally:
+        h.set_option("algo", 0)
+        h.set_option("block_cols", 8192)
+        h.set_option("reorth", 0)
+    assert rc == 0
+    assert algo != 0 or ooc >= 1
+    ref = oracle.rgs(X, leaf=64)
+    assert oracle.is_upper_triangular(R)
+    assert oracle.backward_error(X, Q, R) <= TOL[prec]
+    assert oracle.r_rel_error(R, ref.R) <= max(TOL[prec], 1e-5)
