@@ -494,7 +494,10 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       const float inv = bad ? 0.0f : __frcp_rn(rtt);     // == 1/rtt (correctly rounded)
       if (bad) rtt = 0.0f;
       const float ct = ua * inv;                            // r_{t,t+1}
-      if (g == 0) {
+      // this round's R entries (CTA 0), written after the CTA has published round t+1's values:
+      // stores on CTA 0's critical path made it the last publisher of every round
+      auto write_r = [&]() {
+        if (g != 0) return;
         if (threadIdx.x == 0) {
           p.R[t + (int64_t)t * p.ldr] = rtt;
           if (bad) atomicMin(p.breakdown, (int)(p.col_offset + t));
@@ -505,7 +508,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           if (t >= 3 && more) p.R[(t - 3) + (int64_t)(t + 1) * p.ldr] = c3;
         }
         if (threadIdx.x > t && threadIdx.x < w) p.R[threadIdx.x + (int64_t)t * p.ldr] = 0.0f;
-      }
+      };
       DBG_STAMP(2);
       // ---- one pass over this thread's (at most 2) rows, both rows interleaved, the row
       //      state in registers (u_t, q_{t-1}, q_{t-2}, a_{t+2}, a_{t+3}):
@@ -590,6 +593,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
       }
       if (!more) {
+        write_r();
         // the last column: its rows of Q straight from registers (tall: from this thread's smem rows)
         if constexpr (NR == 0) {
           for (int r = threadIdx.x; r < rows; r += GROUP) P[r0 + r + (int64_t)t * p.ldp] = Elem<T>::store(sp[t * LD + r]);
@@ -634,6 +638,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         if (p.dbg2 != nullptr && lane == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 0] = gtimer();
       }
       DBG_STAMP(4);
+      write_r();
       // ---- inside round t+1's exchange wait: q_t.a_{t+4} (round t+1's value [4+t], read by this
       //      group after round t+3) reduced and added off the critical chain ----
       if (h4) {
