@@ -175,6 +175,11 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   __shared__ double fxs[LEAF_MAX_W][5], fxi[LEAF_MAX_W][5];  // fixed-point scales by (round, class)
   // last-seen exchange words persist across launches (words are never reset, see fx_exp)
   PRO_STAMP(0);
+  if (p.dbg2 != nullptr && threadIdx.x == 0) {
+    unsigned sm;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    p.dbg2[(size_t)2 * LEAF_MAX_W * LEAF_MAX_G + blockIdx.x] = sm;
+  }
   for (int i = threadIdx.x; i < LEAF_XW_WORDS; i += blockDim.x) xprev[i] = p.xprev_g[i];
 
   const int G = gridDim.x;

@@ -440,7 +440,7 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
   p.dbg = dbg ? dbg_buf : nullptr;
   static const bool dbg2 = getenv("RGSQR_LEAF_DEBUG2") != nullptr;
   static long long* dbg2_buf = nullptr;
-  if (dbg2 && !dbg2_buf) cudaMalloc(&dbg2_buf, sizeof(long long) * 2 * LEAF_MAX_W * LEAF_MAX_G);
+  if (dbg2 && !dbg2_buf) cudaMalloc(&dbg2_buf, sizeof(long long) * (2 * LEAF_MAX_W + 1) * LEAF_MAX_G);
   p.dbg2 = dbg2 ? dbg2_buf : nullptr;
   p.dbg_cta = dbg ? atoi(getenv("RGSQR_LEAF_DEBUG")) : 0;
   static const int skip = getenv("RGSQR_LEAF_SKIP") ? atoi(getenv("RGSQR_LEAF_SKIP")) : 0;
@@ -570,6 +570,47 @@ int op_leaf(Ctx* c, int prec, void* P, int64_t ldp, int64_t m, int64_t w, float*
       per += (double)(hb[((size_t)0 * LEAF_MAX_W + r) * 2] - hb[((size_t)0 * LEAF_MAX_W + r - 1) * 2]);
     }
     cnt = std::max(cnt, 1);
+    {
+      // which CTAs publish last / detect last, and each CTA's mean lateness behind the first publisher
+      std::vector<int> lastp(G, 0), lastd(G, 0);
+      std::vector<double> late(G, 0.0);
+      for (int r = 2; r + 1 < w; ++r) {
+        int gp = 0, gd = 0;
+        long long pmin = LLONG_MAX;
+        for (int q = 0; q < G; ++q) pmin = std::min(pmin, hb[((size_t)q * LEAF_MAX_W + r - 1) * 2]);
+        for (int q = 0; q < G; ++q) {
+          const long long P = hb[((size_t)q * LEAF_MAX_W + r - 1) * 2], D = hb[((size_t)q * LEAF_MAX_W + r) * 2 + 1];
+          if (P > hb[((size_t)gp * LEAF_MAX_W + r - 1) * 2]) gp = q;
+          if (D > hb[((size_t)gd * LEAF_MAX_W + r) * 2 + 1]) gd = q;
+          late[q] += (double)(P - pmin);
+        }
+        lastp[gp]++;
+        lastd[gd]++;
+      }
+      std::string sp = "", sd = "", sl = "";
+      for (int q = 0; q < G; ++q) {
+        if (lastp[q]) sp += " " + std::to_string(q) + ":" + std::to_string(lastp[q]);
+        if (lastd[q]) sd += " " + std::to_string(q) + ":" + std::to_string(lastd[q]);
+      }
+      std::vector<int> ord(G);
+      for (int q = 0; q < G; ++q) ord[q] = q;
+      std::sort(ord.begin(), ord.end(), [&](int a2, int b2) { return late[a2] > late[b2]; });
+      std::vector<long long> smid(G);
+      cudaMemcpy(smid.data(), p.dbg2 + (size_t)2 * LEAF_MAX_W * LEAF_MAX_G, sizeof(long long) * G, cudaMemcpyDeviceToHost);
+      for (int k = 0; k < G; ++k)
+        sl += " " + std::to_string(ord[k]) + "/" + std::to_string(smid[ord[k]]) + ":" +
+              std::to_string((int)(late[ord[k]] / std::max(1, cnt)));
+      fprintf(stderr, "[leaf2] last publisher (cta:rounds)%s | last detector%s | mean publish lateness (cta/smid:ns, latest first)%s\n",
+              sp.c_str(), sd.c_str(), sl.c_str());
+      std::string late_sm = "";
+      int nl = 0;
+      for (int q = 0; q < G; ++q)
+        if (late[q] / std::max(1, cnt) > 330.0) {
+          ++nl;
+          late_sm += " " + std::to_string(smid[q]);
+        }
+      fprintf(stderr, "[leaf2] late (> 330 ns) CTAs: %d, their SMs:%s\n", nl, late_sm.c_str());
+    }
     fprintf(stderr, "[leaf2 m=%lld w=%lld G=%d] ns/round %.0f | publish skew %.0f | last publish -> detect: first %.0f mean %.0f last %.0f\n",
             (long long)m, (long long)w, G, per / cnt, skew / cnt, first / cnt, mean / cnt, last / cnt);
   }
