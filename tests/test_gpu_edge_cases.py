@@ -236,3 +236,75 @@ def test_ragged_out_of_core_modes(h, algo, reorth, prec):
     assert oracle.is_upper_triangular(R)
     assert oracle.backward_error(X, Q, R) <= TOL[prec]
     assert oracle.r_rel_error(R, ref.R) <= max(TOL[prec], 1e-5)
+
+
+@pytest.mark.parametrize("path", ["host", "device"])
+def test_dependent_column_warning(h, path):
+    """Reading R4 (PAPER.md:103 assumes independent columns): a column equal to an earlier one leaves
+    u_j at rounding level, r_jj <= m u ||a_j|| -> q_j = 0, r_jj = 0, RGSQR_WARN_RANK_DEFICIENT (1) and the
+    first such column in the stats; the columns before it match the oracle."""
+    m, n = 6000, 40
+    A = gi.gaussian(m, n, seed=23, dtype="fp32")
+    A[:, 17] = A[:, 5]
+    X = gi.to_float64(A, "fp32")
+    rc, Q, R = (host_factor if path == "host" else device_factor)(h, A, "tf32x3")
+    assert rc == 1
+    assert h.stats()["first_breakdown_col"] == 17
+    assert R[17, 17] == 0 and np.all(Q[:, 17] == 0)
+    ref = oracle.rgs(X[:, :17], leaf=64)
+    assert oracle.r_rel_error(R[:17, :17], ref.R) <= 1e-5
+
+
+def test_non_finite_input_flagged(h):
+    """A NaN in the input never yields a silently wrong factorization: the column's r_jj is not finite,
+    so it is flagged (RGSQR_WARN_RANK_DEFICIENT) at or before the NaN's column."""
+    A = gi.gaussian(4096, 32, seed=24, dtype="fp32")
+    A[100, 9] = np.nan
+    rc, Q, R = device_factor(h, A, "tf32")
+    assert rc == 1
+    assert 0 <= h.stats()["first_breakdown_col"] <= 9
+
+
+def test_in_place_q_aliases_a_ragged(h):
+    """Q_out == A_host (in place) with a ragged m (staged through the zero-padded bounce buffers)."""
+    m, n = 10001, 150
+    lda = _lda(m, "fp16")
+    A = np.zeros((lda, n), dtype=np.float16, order="F")
+    A[:m] = gi.gaussian(m, n, seed=25, dtype="fp16")
+    X = gi.to_float64(np.asfortranarray(A[:m]), "fp16")
+    pad = A[m:].copy()
+    R = np.zeros((n, n), dtype=np.float32, order="F")
+    rc = h.factor(A, lda, m, n, A, R, precision="fp16")
+    assert rc == 0
+    check(X, gi.to_float64(np.asfortranarray(A[:m]), "fp16"), R.astype(np.float64), "fp16")
+    assert np.array_equal(A[m:], pad)   # rows past m untouched
+
+
+def test_distributed_context_ragged_host(h):
+    """A one-rank distributed context (every row-sharded code path: NCCL R12 all-reduce, peer exchange words,
+    round-0 all-reduce) on a ragged host problem equals the plain context bitwise."""
+    from paper_conf_icpp_zhangw21_b200 import Handle
+    m, n = 9001, 200
+    A = gi.gaussian(m, n, seed=26, dtype="fp16")
+    d = Handle(0, rank=0, nranks=1, unique_id=Handle.unique_id())
+    out = []
+    h.set_option("fuse_small", 0)   # (single-GPU-only fused bottom node: compare the same products)
+    try:
+        for hh in (h, d):
+            # the automatic split-K factor and tile heights depend on free arena space, which the
+            # rank-reduction buffers change: pin them so both contexts take the same plan (as
+            # tests/test_gpu_dist.py::test_host_ooc_dist_equals_plain)
+            hh.set_option("splitk", 2)
+            hh.set_option("tile_rows_min", 2048)
+            hh.set_option("tile_rows_max", 2048)
+            out.append(host_factor(hh, A, "fp16", budget=6 << 20))
+            hh.set_option("splitk", 0)
+            hh.set_option("tile_rows_min", 4096)
+            hh.set_option("tile_rows_max", 16384)
+    finally:
+        d.close()
+        h.set_option("fuse_small", 1)
+    (rc1, Q1, R1), (rc2, Q2, R2) = out
+    assert rc1 == 0 and rc2 == 0
+    np.testing.assert_array_equal(Q1, Q2)
+    np.testing.assert_array_equal(R1, R2)
