@@ -25,6 +25,8 @@
 // previous round sit on the critical path; the others (q_i^T a_{t+2}, i <= t-2) are added
 // two rounds early.  Round 0 uses a counter barrier + fixed-order gather of fp32 partials.
 // Measured alternatives: scripts/barrier_bench.cu, scripts/exchange_bench.cu.
+#include <type_traits>
+
 #include "dtype.cuh"
 #include "kernels.h"
 
@@ -701,32 +703,40 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           const float4* y2 = reinterpret_cast<const float4*>(sp + (g2 ? t + 5 : t) * LD);
           const float4* xa = reinterpret_cast<const float4*>(sp + kq * LD);
           const float4* xb = reinterpret_cast<const float4*>(sp + (hb ? kq + 32 : kq) * LD);
-          // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld)
-          for (int base = 8 * bw; base < nv4; base += 8 * BULK_W) {
+          // 32-row blocks: the smem slice is zero-padded to a multiple of 32 rows (leaf_ld).  The second
+          // column (lane + 32) is taken warp-uniformly when any lane has one (lanes without it compute
+          // an ignored partial), so the unrolled loop has no branch and its loads can be hoisted
+          auto gemv = [&](auto second) {
+            for (int base = 8 * bw; base < nv4; base += 8 * BULK_W) {
 #pragma unroll
-            for (int i = base; i < base + 8; ++i) {
-              const float4 u = y1[i], v = y2[i], a = xa[i];
-              a0 = fmaf(a.x, u.x, a0);
-              a1 = fmaf(a.y, u.y, a1);
-              a0 = fmaf(a.z, u.z, a0);
-              a1 = fmaf(a.w, u.w, a1);
-              c0 = fmaf(a.x, v.x, c0);
-              c1 = fmaf(a.y, v.y, c1);
-              c0 = fmaf(a.z, v.z, c0);
-              c1 = fmaf(a.w, v.w, c1);
-              if (hb) {
-                const float4 bb = xb[i];
-                b0 = fmaf(bb.x, u.x, b0);
-                b1 = fmaf(bb.y, u.y, b1);
-                b0 = fmaf(bb.z, u.z, b0);
-                b1 = fmaf(bb.w, u.w, b1);
-                d0 = fmaf(bb.x, v.x, d0);
-                d1 = fmaf(bb.y, v.y, d1);
-                d0 = fmaf(bb.z, v.z, d0);
-                d1 = fmaf(bb.w, v.w, d1);
+              for (int i = base; i < base + 8; ++i) {
+                const float4 u = y1[i], v = y2[i], a = xa[i];
+                a0 = fmaf(a.x, u.x, a0);
+                a1 = fmaf(a.y, u.y, a1);
+                a0 = fmaf(a.z, u.z, a0);
+                a1 = fmaf(a.w, u.w, a1);
+                c0 = fmaf(a.x, v.x, c0);
+                c1 = fmaf(a.y, v.y, c1);
+                c0 = fmaf(a.z, v.z, c0);
+                c1 = fmaf(a.w, v.w, c1);
+                if constexpr (decltype(second)::value) {
+                  const float4 bb = xb[i];
+                  b0 = fmaf(bb.x, u.x, b0);
+                  b1 = fmaf(bb.y, u.y, b1);
+                  b0 = fmaf(bb.z, u.z, b0);
+                  b1 = fmaf(bb.w, u.w, b1);
+                  d0 = fmaf(bb.x, v.x, d0);
+                  d1 = fmaf(bb.y, v.y, d1);
+                  d0 = fmaf(bb.z, v.z, d0);
+                  d1 = fmaf(bb.w, v.w, d1);
+                }
               }
             }
-          }
+          };
+          if (cnt > 32)
+            gemv(std::true_type{});
+          else
+            gemv(std::false_type{});
         }
         part[bw][kq] = a0 + a1;
         part[bw][kq + 32] = b0 + b1;
