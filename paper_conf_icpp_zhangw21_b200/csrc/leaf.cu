@@ -175,6 +175,9 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   __shared__ int exS[LEAF_MAX_W];                           // 2||a_j|| < 2^exS[j]
   __shared__ float tauc[LEAF_MAX_W];                        // breakdown thresholds
   __shared__ double fxs[LEAF_MAX_W][5], fxi[LEAF_MAX_W][5];  // fixed-point scales by (round, class)
+  // the same scales in fp32 when 2^+-e is a normal float (else 0: the fp64 path is taken); scaling by a
+  // power of two commutes with rounding, so both paths give bitwise-equal results for normal values
+  __shared__ float fxsf[LEAF_MAX_W][5], fxif[LEAF_MAX_W][5];
   // last-seen exchange words persist across launches (words are never reset, see fx_exp)
   PRO_STAMP(0);
   if (p.dbg2 != nullptr && threadIdx.x == 0) {
@@ -277,8 +280,19 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
   // CTA has read them: the lookahead values of round t are added two rounds early), one
   // 256-byte line per word so that concurrent atomics and polls land in different L2 slices.
   auto xw_index = [&](int t, int k) -> int { return (t & (LEAF_XW_SETS - 1)) * (LEAF_MAX_W + 2) + k; };
-  auto fx_add_scaled = [&](int t, int k, float s, double scale) {
-    long long v = __double2ll_rn((double)s * scale);
+  // value -> fixed point (s * 2^e rounded to an integer) and back (total * 2^-e rounded to fp32)
+  auto to_fx = [&](float s, float sf, double sd) -> long long {
+    return sf != 0.0f ? __float2ll_rn(s * sf) : __double2ll_rn((double)s * sd);
+  };
+  auto from_fx = [&](long long total, float xf, double xd) -> float {
+    if (xf != 0.0f) {
+      const float v = __ll2float_rn(total) * xf;
+      if (!(fabsf(v) < 1.17549435e-38f) || total == 0) return v;   // (subnormal results: the fp64 path)
+    }
+    return (float)((double)total * xd);
+  };
+  auto fx_add_scaled = [&](int t, int k, float s, float sf, double sd) {
+    long long v = to_fx(s, sf, sd);
     const long long vb = 1ll << FX_VBITS;
     v = v > vb ? vb : (v < -vb ? -vb : v);
     const unsigned long long add = (1ull << FX_CNT_SHIFT) + (unsigned long long)(v + vb);
@@ -292,7 +306,10 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
                      : "memory");
     }
   };
-  auto fx_add = [&](int t, int k, float s) { fx_add_scaled(t, k, s, fxs[t][k < 4 ? k : 4]); };
+  auto fx_add = [&](int t, int k, float s) {
+    const int c = k < 4 ? k : 4;
+    fx_add_scaled(t, k, s, fxsf[t][c], fxs[t][c]);
+  };
   // CTA total of values [0, n) of a [GEMV_PARTS][ld] partial buffer: 4 threads per value, each
   // adds a quarter of the parts, then a 2-level xor tree (fixed order).  Called by all threads;
   // the returned sum is valid on the thread with (threadIdx.x & 3) == 0 of value threadIdx.x >> 2.
@@ -404,6 +421,8 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     const int e = need < w ? fx_exp(t, c) : 0;
     fxs[t][c] = pow2d(e);
     fxi[t][c] = pow2d(-e);
+    fxsf[t][c] = (e > -120 && e < 120) ? __int_as_float((127 + e) << 23) : 0.0f;
+    fxif[t][c] = (e > -120 && e < 120) ? __int_as_float((127 - e) << 23) : 0.0f;
   }
   // (the __syncthreads at the top of the round loop publishes exS / tauc)
 
@@ -447,6 +466,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
     }
     for (int t = 0; t < w; ++t) {
       DBG_STAMP(0);
+      const float tau = tauc[t];   // (constant during the rounds: loaded before the exchange wait)
       if (t > 0) {
         // ---- round t's exchange: each of the (at most 4) values the scalars need is polled
         //      by its thread until all ranks x G CTAs have added; values [4+i] (coefficients
@@ -476,7 +496,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
           xprev[widx] = now;
           if (p.dbg2 != nullptr && k == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 1] = gtimer();
           const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
-          const float val = (float)((double)total * fxi[tr][k < 4 ? k : 4]);
+          const float val = from_fx(total, fxif[tr][k < 4 ? k : 4], fxi[tr][k < 4 ? k : 4]);
           tot[t & 1][late ? 4 : k] = val;
         }
       }
@@ -496,7 +516,6 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       const float c2 = (t >= 2 && more) ? tot[(t - 1) & 1][3] : 0.0f;   // r_{t-2,t+1} (round t-1)
       const float c3 = (t >= 3 && more) ? tt[4] : 0.0f;    // r_{t-3,t+1} (round t-2)
       float rtt = sqrtf(uu);
-      const float tau = tauc[t];
       const bool bad = !(rtt > tau) || !isfinite(rtt);
       const float inv = bad ? 0.0f : __frcp_rn(rtt);     // == 1/rtt (correctly rounded)
       if (bad) rtt = 0.0f;
@@ -613,7 +632,11 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
       // the critical reducer's lane 4c (c < 5) adds value c of round t+1: its fixed-point scale now
       const int n_crit = !h2 ? 1 : (!h3 ? 3 : 4);   // critical values of round t+1
       double crit_scale = 0.0;
-      if (warp == CRIT_W && (lane & 7) == 0 && (lane >> 3) < n_crit) crit_scale = fxs[t + 1][lane >> 3];
+      float crit_scale_f = 0.0f;
+      if (warp == CRIT_W && (lane & 7) == 0 && (lane >> 3) < n_crit) {
+        crit_scale = fxs[t + 1][lane >> 3];
+        crit_scale_f = fxsf[t + 1][lane >> 3];
+      }
       // warp sums of the 5 critical values: a transposing butterfly (6 shuffles) leaves value k
       // < 4 in lane 8k, an xor tree the fifth (fixed tree per value)
       {
@@ -640,7 +663,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         s += __shfl_xor_sync(0xffffffffu, s, 4);
         s += __shfl_xor_sync(0xffffffffu, s, 2);
         s += __shfl_xor_sync(0xffffffffu, s, 1);
-        if (j == 0 && c < n_crit) fx_add_scaled(t + 1, c, s, crit_scale);
+        if (j == 0 && c < n_crit) fx_add_scaled(t + 1, c, s, crit_scale_f, crit_scale);
         if (p.dbg != nullptr && blockIdx.x == DBG_CTA && lane == 0) p.dbg[(size_t)t * 16 + 7] = clock64();
         if (p.dbg2 != nullptr && lane == 0) p.dbg2[((size_t)g * LEAF_MAX_W + t) * 2 + 0] = gtimer();
       }
@@ -785,7 +808,7 @@ __global__ void __launch_bounds__(LEAF_THREADS, 1) leaf_cgs_kernel(LeafParams p)
         }
         xprev[pidx] = pnow;
         const long long total = (long long)(d & ((1ull << FX_CNT_SHIFT) - 1)) - (long long)cnt * (1ll << FX_VBITS);
-        const float val = (float)((double)total * fxi[t][4]);
+        const float val = from_fx(total, fxif[t][4], fxi[t][4]);
         coef[t % 3][btid] = val;
         if (g == 0) p.R[btid + (int64_t)(t + 3) * p.ldr] = val;
       }
