@@ -383,6 +383,45 @@ int op_outer(Ctx* c, int prec, const void* Q1, int64_t ldq, const void* R12op, i
   return fail(c, RGSQR_ERR_UNSUPPORTED, "outer: precision not supported");
 }
 
+// A TF32X3 recursion node, R12 = Q1^T A2 then A2 <- A2 - Q1 R12, with Q1 split into hi / lo ONCE for both
+// products (op_inner + op_outer split it twice); same kernels and operands, so bitwise equal to the pair.
+// Single-GPU contexts only (the row-sharded inner product reduces R12 across ranks first).
+static int op_node_x3(Ctx* c, const void* Q1, int64_t ldq, void* A2, int64_t lda, int64_t m, int64_t w1, int64_t w2,
+                      float* R12, int64_t ldr, void* R12op, cudaStream_t st) {
+  const size_t mark = c->arena.mark();
+  const int64_t md = (m + 3) / 4 * 4;   // hi / lo leading dimension (16-byte TMA pitch)
+  float* q_hi = static_cast<float*>(c->arena.alloc((size_t)md * w1 * 4));
+  float* q_lo = static_cast<float*>(c->arena.alloc((size_t)md * w1 * 4));
+  const size_t mark_a = c->arena.mark();
+  float* a_hi = static_cast<float*>(c->arena.alloc((size_t)md * w2 * 4));
+  float* a_lo = static_cast<float*>(c->arena.alloc((size_t)md * w2 * 4));
+  if (!q_hi || !q_lo || !a_hi || !a_lo) {
+    c->arena.release(mark);
+    return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "node (tf32x3): no space for the hi/lo operands");
+  }
+  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(Q1), ldq, q_hi, md, q_lo, md, m, w1, c->num_sms, st));
+  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(A2), lda, a_hi, md, a_lo, md, m, w2, c->num_sms, st));
+  c->stats.n_other_launches += 2;
+  int rc = op_inner_once<float>(c, RGSQR_TF32X3, q_hi, md, a_hi, md, m, w1, w2, R12, ldr, R12op, w1, 0, st, q_lo, a_lo);
+  if (rc < 0) {
+    c->arena.release(mark);
+    return rc;
+  }
+  c->arena.release(mark_a);   // (stream-ordered reuse: the outer product's buffers follow the inner product)
+  const int64_t lr = (w1 + 3) / 4 * 4;
+  float* r_hi = static_cast<float*>(c->arena.alloc((size_t)lr * w2 * 4));
+  float* r_lo = static_cast<float*>(c->arena.alloc((size_t)lr * w2 * 4));
+  if (!r_hi || !r_lo) {
+    c->arena.release(mark);
+    return fail(c, RGSQR_ERR_BUDGET_TOO_SMALL, "node (tf32x3): no space for the R12 hi/lo operands");
+  }
+  RGSQR_CUDA(c, launch_tf32_split(static_cast<const float*>(R12op), w1, r_hi, lr, r_lo, lr, w1, w2, c->num_sms, st));
+  c->stats.n_other_launches++;
+  rc = op_outer_t<float>(c, RGSQR_TF32X3, q_hi, md, r_hi, lr, A2, lda, m, w1, w2, st, q_lo, r_lo);
+  c->arena.release(mark);
+  return rc;
+}
+
 static void leaf_geometry(Ctx* c, int64_t m, int* grid, int* rp) {
   int G = c->opt.leaf_ctas > 0 ? (int)c->opt.leaf_ctas : c->num_sms;
   G = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)G, (int64_t)LEAF_MAX_G, (m + 31) / 32}));
@@ -837,10 +876,15 @@ static int incore_rec(IncoreCtx& k, int64_t c0, int64_t w) {
       return incore_rec(k, h, w2);
     }
   }
-  rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.r12op, w1, 0, k.st);
-  if (rc < 0) return rc;
-  rc = op_outer(k.c, k.prec, Q1, k.lda, k.r12op, w1, A2, k.lda, k.m, w1, w2, k.st);
-  if (rc < 0) return rc;
+  if (k.prec == RGSQR_TF32X3 && !k.S && !k.c->nccl_comm && k.c->opt.vshards <= 1) {
+    rc = op_node_x3(k.c, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.r12op, k.st);
+    if (rc < 0) return rc;
+  } else {
+    rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, R12, k.ldr, k.r12op, w1, 0, k.st);
+    if (rc < 0) return rc;
+    rc = op_outer(k.c, k.prec, Q1, k.lda, k.r12op, w1, A2, k.lda, k.m, w1, w2, k.st);
+    if (rc < 0) return rc;
+  }
   if (k.S) {
     // CGS2: S = Q1^T A2', A2' -= Q1 S, R12 += S (fixed order)
     rc = op_inner(k.c, k.prec, Q1, k.lda, A2, k.lda, k.m, w1, w2, k.S, w1, k.r12op, w1, 0, k.st);
