@@ -29,20 +29,30 @@ def handles():
 
 
 def _dev_factor(h, A, prec, m, n):
-    st = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}[prec]
+    st = {"fp16": "fp16", "bf16": "bf16", "tf32": "fp32", "tf32x3": "fp32"}[prec]
     Ad = to_dev(A, st)
     R = torch.empty((n, n), dtype=torch.float32, device="cuda")
     rc = h.factor_device(Ad, m, m, n, Ad, R, precision=prec)
     return rc, from_dev(Ad), R.cpu().numpy().T
 
 
-@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32"])
+@pytest.mark.parametrize("prec", ["fp16", "bf16", "tf32", "tf32x3"])
 def test_device_dist_equals_plain(handles, prec):
+    """(tf32x3: the plain context's nodes share one Q1 hi / lo split between both products, op_node_x3;
+    the distributed context runs the separate inner / outer products -- bitwise equal, split-K pinned
+    because the automatic factor follows the free arena, which the rank-reduction buffer changes)"""
     plain, dist = handles
     m, n = 16384, 512
-    A = gi.gaussian(m, n, seed=11, dtype={"fp16": "fp16", "bf16": "bf16", "tf32": "fp32"}[prec])
-    _, Q1, R1 = _dev_factor(plain, A, prec, m, n)
-    _, Q2, R2 = _dev_factor(dist, A, prec, m, n)
+    A = gi.gaussian(m, n, seed=11, dtype={"fp16": "fp16", "bf16": "bf16", "tf32": "fp32", "tf32x3": "fp32"}[prec])
+    sk = 4 if prec == "tf32x3" else 0
+    plain.set_option("splitk", sk)
+    dist.set_option("splitk", sk)
+    try:
+        _, Q1, R1 = _dev_factor(plain, A, prec, m, n)
+        _, Q2, R2 = _dev_factor(dist, A, prec, m, n)
+    finally:
+        plain.set_option("splitk", 0)
+        dist.set_option("splitk", 0)
     np.testing.assert_array_equal(R1, R2)
     np.testing.assert_array_equal(Q1, Q2)
 
