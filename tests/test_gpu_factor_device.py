@@ -167,3 +167,17 @@ def test_tall_panel_leaves(h, prec, m, n, leaf):
     # element-wise on R against the oracle's R (the leading block)
     k = min(n, 32)
     np.testing.assert_allclose(R[:k, :k], ref.R[:k, :k], atol=TOL[prec] * np.abs(ref.R).max())
+
+
+def test_tall_panel_tf32x3(h):
+    """Tall panels in the north star's 1e-5 mode (4-wide fp32 leaves at 1M rows: narrow TF32X3 nodes whose
+    R12 hi / lo operands need padded pitches): R error vs Gram-Cholesky of the stored A."""
+    m, n = 1048576, 20
+    A64, _ = gi.usv(m, n, kappa=100.0, seed=6)
+    A = gi.to_storage(A64, "fp32")
+    X = gi.to_float64(A, "fp32")
+    rc, Q, R = run(h, A, "fp32", "tf32x3", m, n)
+    assert rc == 0
+    assert oracle.is_upper_triangular(R)
+    assert oracle.r_rel_error(R, oracle.gram_cholesky_r(X)) <= 1e-5
+    assert oracle.backward_error(X, Q, R) <= 1e-5
