@@ -206,3 +206,21 @@ def test_budget_agreement_follows_each_call(handles):
         assert dist.factor(A, m, m, n, Q, R, precision="fp16", budget=b * MiB) == 0
         st = dist.stats()
         assert st["arena_bytes"] == b * MiB - st["ctx_device_bytes"], (b, st["arena_bytes"])
+
+
+def test_dist_tall_panel_equals_plain(handles):
+    """Tall leaf panels (> 2048 rows per CTA, leaf.cu NR = 0) through the row-sharded code paths (round-0-only
+    launch + all-reduce, peer exchange words): bitwise equal to the plain context."""
+    plain, dist = handles
+    m, n = 600000, 48
+    A = gi.gaussian(m, n, seed=13, dtype="fp16")
+    for h in (plain, dist):
+        h.set_option("splitk", 8)
+    try:
+        _, Q1, R1 = _dev_factor(plain, A, "fp16", m, n)
+        _, Q2, R2 = _dev_factor(dist, A, "fp16", m, n)
+    finally:
+        for h in (plain, dist):
+            h.set_option("splitk", 0)
+    np.testing.assert_array_equal(R1, R2)
+    np.testing.assert_array_equal(Q1, Q2)
