@@ -209,8 +209,10 @@ static int op_inner_once(Ctx* c, int prec, const void* Q1, int64_t ldq, const vo
   GemmExtra gx;
   // (TF32X3's 128 x 128 fp32 tiles need ~128 B/clk/SM of operands: grouping 4 M-tiles keeps more of
   // them in L2 there, 108 -> 105 ms at configs[1]'s shape)
+  // (16-bit, configs[1]'s top node: 16 M-tiles per group read 2.77x the algorithmic DRAM bytes vs 3.1x
+  // x-fastest, at equal time -- profiles/r2_ncu_summary.md)
   gx.group_m = env_group >= 0 ? env_group
-                              : (tiles > 8 * (int64_t)c->num_sms ? 16 : (x3 && tiles > 2 * (int64_t)c->num_sms ? 4 : 0));
+                              : (tiles > 2 * (int64_t)c->num_sms ? (x3 ? 4 : 16) : 0);
   // One wave: tiles x splits <= SMs (rounding up put 152 CTAs on 148 SMs at w1 = w2 = 512 and
   // doubled the kernel time: 57 vs 37 us, profiles/r1_splitk_scan.txt).
   int64_t splits = c->opt.splitk > 0 ? c->opt.splitk : (tiles >= c->num_sms ? 1 : c->num_sms / tiles);
